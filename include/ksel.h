@@ -1,0 +1,144 @@
+/*
+ * ksel.h -- C ABI of libksel.so: B200-native (sm_100a) batched k-selection and
+ * fused brute-force k-NN.
+ *
+ * Paper: Tang, Huang, Eyers, Mills, Guo, "Efficient Selection Algorithm for
+ * Fast k-NN Search on GPU", IPDPS 2015.  Citations are PAPER.md line numbers.
+ *
+ * Common conventions
+ * ------------------
+ *  - All array pointers are CUDA DEVICE pointers owned by the caller (except
+ *    the *_host entry points, documented below).  Arrays are dense row-major.
+ *    Inputs are read-only; outputs are fully overwritten (all Q*k entries).
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default
+ *    stream).  Every call is stream-ordered and asynchronous: it validates its
+ *    arguments on the host, enqueues kernels and returns; it never
+ *    synchronises the stream and allocates no device memory.
+ *  - Order ("lexicographic (value, index)", readings R1-R5 in DESIGN.md):
+ *    values compare as IEEE fp32 with -0.0 == +0.0, NaN greater than +Inf and
+ *    all NaNs equal, denormals exact; equal values are ordered by the lower
+ *    index.  Results are BIT-EXACT with the CPU oracle (oracle/).
+ *  - Indices are int32, 0-based.
+ *  - Thread-safe: no global mutable state except a lazily created, mutex-
+ *    protected device-property cache and (host entry points only) per-device
+ *    copy streams.
+ *  - Errors: a nonzero ksel_status is returned; no exception crosses the ABI
+ *    and nothing aborts.  Argument errors are detected before any launch.  A
+ *    launch failure (cudaGetLastError after the launch) is KSEL_ERR_CUDA; the
+ *    CUDA error itself is left in place (sticky errors are not cleared).
+ */
+#ifndef KSEL_H_
+#define KSEL_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define KSEL_API __attribute__((visibility("default")))
+#else
+#define KSEL_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    KSEL_OK = 0,
+    KSEL_ERR_INVALID_ARG = 1, /* null pointer, bad size, misalignment, aliasing */
+    KSEL_ERR_UNSUPPORTED = 2, /* valid request outside this build's range (k > 1024) */
+    KSEL_ERR_CUDA = 3,        /* a CUDA runtime call or kernel launch failed */
+    KSEL_ERR_NO_DEVICE = 4    /* no sm_100 device is current */
+} ksel_status;
+
+#define KSEL_MAX_K 1024
+
+/* ksel_select -- batched k-selection ("finding the k smallest
+ * values from a given unordered list"; L19 Algorithm 1; L637 sorted output).
+ *
+ *   dist     [Q][N] fp32, device, 4-byte aligned (16-byte alignment of each row
+ *            start is not required; unaligned heads/tails are handled).
+ *   Q >= 1 rows, 1 <= N <= 2^31 - 1 columns, 1 <= k <= min(N, KSEL_MAX_K).
+ *   out_val  [Q][k] fp32, device: out_val[q][t] has the same BITS as
+ *            dist[q][out_idx[q][t]] (including -0.0 and NaN payloads).
+ *   out_idx  [Q][k] int32, device.
+ * out[q][0..k) = the k smallest pairs (dist[q][j], j) in lexicographic
+ * (value, index) order, ascending.  Outputs must not overlap dist.
+ * k > KSEL_MAX_K with k <= N returns KSEL_ERR_UNSUPPORTED. */
+KSEL_API int ksel_select(const float* dist, int64_t Q, int64_t N, int k, float* out_val,
+                int32_t* out_idx, void* stream);
+
+/* ksel_select_config -- ksel_select with the kernel variant fixed (ablation /
+ * tuning; same result bits for every variant):
+ *   algo           KSEL_ALGO_AUTO (0), KSEL_ALGO_QUEUE (1): candidates merged into a
+ *                  warp-register bitonic queue at every buffer flush (Merge Queue +
+ *                  Buffered Search), KSEL_ALGO_POOL (2):
+ *                  candidate pool narrowed by radix-histogram select (Hierarchical
+ *                  Partition's discard-by-group, L221-L231, with value buckets).
+ *   warps_per_row  0 = automatic, else 1, 2, 4 or 8 warps cooperating on each row.
+ * Other arguments as ksel_select; invalid algo / warps_per_row -> INVALID_ARG. */
+#define KSEL_ALGO_AUTO 0
+#define KSEL_ALGO_QUEUE 1
+#define KSEL_ALGO_POOL 2
+KSEL_API int ksel_select_config(const float* dist, int64_t Q, int64_t N, int k, float* out_val,
+                                int32_t* out_idx, int algo, int warps_per_row, void* stream);
+
+/* ksel_select_host -- the same operation on HOST buffers (the end-to-end entry
+ * point a user without device memory calls).  h_dist [Q][N], h_out_val and
+ * h_out_idx [Q][k] are host pointers (page-locked memory gives overlapped
+ * copies; pageable memory works but serialises).  The library streams row
+ * blocks host->device, selects, and copies results back, double-buffered
+ * across two internal copy streams, using the caller's device workspace
+ * `d_work` of `work_bytes` bytes (query the minimum with
+ * ksel_select_host_workspace).  Returns after the results are in host memory
+ * (this call synchronises).  Same ordering/bit-exactness as ksel_select. */
+KSEL_API size_t ksel_select_host_workspace(int64_t N, int k);
+KSEL_API int ksel_select_host(const float* h_dist, int64_t Q, int64_t N, int k, float* h_out_val,
+                     int32_t* h_out_idx, void* d_work, size_t work_bytes, void* stream);
+
+/* ksel_merge -- final merge of S per-shard candidate lists (divide-and-merge,
+ * PAPER.md L243 ref. [18]; Merge Queue merging sorted levels, L41, L139).
+ *   cand_val, cand_idx  [S][Q][kin], device.  For every (s, q) the list
+ *            cand_*[s][q][0..kin) is sorted ascending in (value, index) order
+ *            (exactly what ksel_select / knn_search emit).  Indices must be
+ *            unique per query across all lists (e.g. global reference ids).
+ *   1 <= S <= 64, 1 <= kin <= KSEL_MAX_K, 1 <= k <= min(S*kin, KSEL_MAX_K).
+ *   out_val/out_idx [Q][k]: the k smallest pairs of the union, ascending;
+ *            out_val keeps the candidates' bits.
+ * Used after the NCCL all-gather of the row-sharded k-NN (S = world size). */
+KSEL_API int ksel_merge(const float* cand_val, const int32_t* cand_idx, int64_t Q, int S, int kin, int k,
+               float* out_val, int32_t* out_idx, void* stream);
+
+/* knn_search -- brute-force k-NN: distance phase (Sec. II.A,
+ * "the method of [3]" L243) fused with k-selection.
+ *   ref   [N][D] fp32, query [Q][D] fp32, device, 16-byte aligned.
+ *   1 <= D <= 1024, D % 4 == 0; 1 <= k <= min(N, KSEL_MAX_K);
+ *   N + idx_offset <= 2^31 - 1, idx_offset >= 0.
+ *   out_dist [Q][k] fp32: squared L2 distance (no sqrt), clamped at >= 0,
+ *            computed as |q|^2 + |r|^2 - 2 q.r with fp32 accumulation (error
+ *            bound: DESIGN.md "knn tolerance");
+ *   out_idx  [Q][k] int32: idx_offset + reference row, ascending by
+ *            (distance, index).
+ *   d_work   device workspace of >= knn_search_workspace(N, Q, D, k) bytes
+ *            (norms and split operand copies); NULL allowed when that is 0.
+ * The Q x N distance matrix is never written to memory. */
+KSEL_API size_t knn_search_workspace(int64_t N, int64_t Q, int D, int k);
+KSEL_API int knn_search(const float* ref, const float* query, int64_t N, int64_t Q, int D, int k,
+               float* out_dist, int32_t* out_idx, int64_t idx_offset, void* d_work,
+               size_t work_bytes, void* stream);
+
+/* Human-readable text for a ksel_status (static storage, never NULL). */
+KSEL_API const char* ksel_strerror(int status);
+
+/* Library version, encoded as major*10000 + minor*100 + patch. */
+KSEL_API int ksel_version(void);
+
+/* Number of device kernels this library has enqueued since load (all entry
+ * points, all threads).  Used by bench.py to report gpu_launches. */
+KSEL_API int64_t ksel_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* KSEL_H_ */

@@ -1,0 +1,185 @@
+"""B200-native batched k-selection (Tang et al., IPDPS 2015) -- Python binding.
+
+Thin ctypes marshalling over the C ABI of ``libksel.so`` (``include/ksel.h``):
+every step of the hot path runs in the library's sm_100a kernels.  PyTorch is
+used only for device memory and the current CUDA stream.  There is no CPU or
+library fallback: if ``libksel.so`` is missing this module raises on import.
+
+Entry points (same names as the C ABI):
+
+* :func:`ksel_select`      -- k smallest (value, index) pairs of every row.
+* :func:`ksel_select_host` -- the same on host buffers (end-to-end path).
+* :func:`ksel_merge`       -- top-k of the union of S sorted candidate lists.
+* :func:`knn_search`       -- fused distance + selection brute-force k-NN.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import torch
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libksel.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(
+        "libksel.so is not built (expected at %s); run `python __graft_entry__.py` "
+        "or paper_conf_ipps_tang0emg15_b200/build.py" % LIB_PATH)
+
+_lib = ctypes.CDLL(LIB_PATH)
+_p, _i64, _i32, _sz = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int, ctypes.c_size_t
+_lib.ksel_select.argtypes = [_p, _i64, _i64, _i32, _p, _p, _p]
+_lib.ksel_select_config.argtypes = [_p, _i64, _i64, _i32, _p, _p, _i32, _i32, _p]
+_lib.ksel_select_host_workspace.argtypes = [_i64, _i32]
+_lib.ksel_select_host_workspace.restype = _sz
+_lib.ksel_select_host.argtypes = [_p, _i64, _i64, _i32, _p, _p, _p, _sz, _p]
+_lib.ksel_merge.argtypes = [_p, _p, _i64, _i32, _i32, _i32, _p, _p, _p]
+_lib.knn_search_workspace.argtypes = [_i64, _i64, _i32, _i32]
+_lib.knn_search_workspace.restype = _sz
+_lib.knn_search.argtypes = [_p, _p, _i64, _i64, _i32, _i32, _p, _p, _i64, _p, _sz, _p]
+_lib.ksel_strerror.argtypes = [_i32]
+_lib.ksel_strerror.restype = ctypes.c_char_p
+_lib.ksel_launch_count.restype = _i64
+for _f in (_lib.ksel_select, _lib.ksel_select_config, _lib.ksel_select_host, _lib.ksel_merge, _lib.knn_search, _lib.ksel_version):
+    _f.restype = ctypes.c_int
+
+KSEL_MAX_K = 1024
+ALGO_AUTO, ALGO_QUEUE, ALGO_POOL = 0, 1, 2
+EXPORTS = ("ksel_select", "ksel_select_config", "ksel_select_host_workspace", "ksel_select_host", "ksel_merge",
+           "knn_search_workspace", "knn_search", "ksel_strerror", "ksel_version", "ksel_launch_count")
+
+
+class KselError(RuntimeError):
+    def __init__(self, fn: str, status: int):
+        self.status = status
+        super().__init__("%s failed: %s (status %d)" % (fn, strerror(status), status))
+
+
+def strerror(status: int) -> str:
+    return _lib.ksel_strerror(status).decode()
+
+
+def version() -> int:
+    return _lib.ksel_version()
+
+
+def launch_count() -> int:
+    """Kernels enqueued by libksel since load (all entry points)."""
+    return _lib.ksel_launch_count()
+
+
+def _check(fn, status):
+    if status != 0:
+        raise KselError(fn, status)
+
+
+def _dev_f32(t: torch.Tensor, name: str, ndim: int):
+    if not isinstance(t, torch.Tensor) or t.device.type != "cuda":
+        raise TypeError("%s must be a CUDA tensor" % name)
+    if t.dtype != torch.float32 or t.dim() != ndim or not t.is_contiguous():
+        raise TypeError("%s must be a contiguous %d-D float32 tensor" % (name, ndim))
+
+
+def _stream(device) -> int:
+    return torch.cuda.current_stream(device).cuda_stream
+
+
+def ksel_select(dist: torch.Tensor, k: int, out_val: torch.Tensor | None = None,
+                out_idx: torch.Tensor | None = None, algo: int = ALGO_AUTO, warps_per_row: int = 0):
+    """k smallest (value, index) pairs per row of ``dist`` [Q, N], ascending.
+
+    Returns (values float32 [Q, k] with the input bits, indices int32 [Q, k]).
+    Enqueued on the current stream; asynchronous.  ``algo``/``warps_per_row``
+    pin the kernel variant (ksel_select_config); defaults pick automatically."""
+    _dev_f32(dist, "dist", 2)
+    Q, N = dist.shape
+    if out_val is None:
+        out_val = torch.empty((Q, k), dtype=torch.float32, device=dist.device)
+    if out_idx is None:
+        out_idx = torch.empty((Q, k), dtype=torch.int32, device=dist.device)
+    with torch.cuda.device(dist.device):
+        if algo == ALGO_AUTO and warps_per_row == 0:
+            st = _lib.ksel_select(dist.data_ptr(), Q, N, k, out_val.data_ptr(), out_idx.data_ptr(),
+                                  _stream(dist.device))
+        else:
+            st = _lib.ksel_select_config(dist.data_ptr(), Q, N, k, out_val.data_ptr(), out_idx.data_ptr(),
+                                         algo, warps_per_row, _stream(dist.device))
+        _check("ksel_select", st)
+    return out_val, out_idx
+
+
+def ksel_select_host_workspace(N: int, k: int) -> int:
+    return int(_lib.ksel_select_host_workspace(N, k))
+
+
+def ksel_select_host(dist: torch.Tensor, k: int, out_val: torch.Tensor | None = None,
+                     out_idx: torch.Tensor | None = None, workspace: torch.Tensor | None = None,
+                     device=None):
+    """End-to-end selection on HOST tensors (pin them for overlapped copies).
+
+    ``dist`` is a contiguous float32 CPU tensor [Q, N]; results are CPU tensors.
+    The call returns when the results are in host memory."""
+    if dist.device.type != "cpu" or dist.dtype != torch.float32 or not dist.is_contiguous():
+        raise TypeError("dist must be a contiguous float32 CPU tensor")
+    Q, N = dist.shape
+    dev = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
+    if out_val is None:
+        out_val = torch.empty((Q, k), dtype=torch.float32, pin_memory=dist.is_pinned())
+    if out_idx is None:
+        out_idx = torch.empty((Q, k), dtype=torch.int32, pin_memory=dist.is_pinned())
+    if workspace is None:
+        workspace = torch.empty(ksel_select_host_workspace(N, k), dtype=torch.uint8, device=dev)
+    with torch.cuda.device(dev):
+        _check("ksel_select_host", _lib.ksel_select_host(
+            dist.data_ptr(), Q, N, k, out_val.data_ptr(), out_idx.data_ptr(), workspace.data_ptr(),
+            workspace.numel(), _stream(dev)))
+    return out_val, out_idx
+
+
+def ksel_merge(cand_val: torch.Tensor, cand_idx: torch.Tensor, k: int,
+               out_val: torch.Tensor | None = None, out_idx: torch.Tensor | None = None):
+    """Top-k of the union of S sorted lists per query; inputs are [S, Q, kin]."""
+    _dev_f32(cand_val, "cand_val", 3)
+    if cand_idx.dtype != torch.int32 or cand_idx.shape != cand_val.shape or not cand_idx.is_contiguous():
+        raise TypeError("cand_idx must be a contiguous int32 tensor shaped like cand_val")
+    S, Q, kin = cand_val.shape
+    if out_val is None:
+        out_val = torch.empty((Q, k), dtype=torch.float32, device=cand_val.device)
+    if out_idx is None:
+        out_idx = torch.empty((Q, k), dtype=torch.int32, device=cand_val.device)
+    with torch.cuda.device(cand_val.device):
+        _check("ksel_merge", _lib.ksel_merge(cand_val.data_ptr(), cand_idx.data_ptr(), Q, S, kin, k,
+                                             out_val.data_ptr(), out_idx.data_ptr(),
+                                             _stream(cand_val.device)))
+    return out_val, out_idx
+
+
+def knn_search_workspace(N: int, Q: int, D: int, k: int) -> int:
+    return int(_lib.knn_search_workspace(N, Q, D, k))
+
+
+def knn_search(ref: torch.Tensor, query: torch.Tensor, k: int, idx_offset: int = 0,
+               out_dist: torch.Tensor | None = None, out_idx: torch.Tensor | None = None,
+               workspace: torch.Tensor | None = None):
+    """k nearest references (squared L2) of every query; ref [N, D], query [Q, D]."""
+    _dev_f32(ref, "ref", 2)
+    _dev_f32(query, "query", 2)
+    N, D = ref.shape
+    Q = query.shape[0]
+    if query.shape[1] != D:
+        raise ValueError("ref and query must share D")
+    if out_dist is None:
+        out_dist = torch.empty((Q, k), dtype=torch.float32, device=ref.device)
+    if out_idx is None:
+        out_idx = torch.empty((Q, k), dtype=torch.int32, device=ref.device)
+    need = knn_search_workspace(N, Q, D, k)
+    if workspace is None and need > 0:
+        workspace = torch.empty(need, dtype=torch.uint8, device=ref.device)
+    wptr = workspace.data_ptr() if workspace is not None else 0
+    wlen = workspace.numel() if workspace is not None else 0
+    with torch.cuda.device(ref.device):
+        _check("knn_search", _lib.knn_search(ref.data_ptr(), query.data_ptr(), N, Q, D, k,
+                                             out_dist.data_ptr(), out_idx.data_ptr(), idx_offset,
+                                             wptr, wlen, _stream(ref.device)))
+    return out_dist, out_idx

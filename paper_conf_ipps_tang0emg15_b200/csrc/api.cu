@@ -1,0 +1,220 @@
+// api.cu -- the C ABI of libksel.so (declared in include/ksel.h).
+//
+// Host-side argument validation, device-property cache, launch dispatch and
+// the host-buffer (end-to-end) pipeline.  No torch types, no allocation on the
+// device paths, no stream synchronisation except in ksel_select_host.
+#include <atomic>
+#include <cstdint>
+#include <cstring>
+#include <mutex>
+
+#include <cuda_runtime.h>
+
+#include "ksel.h"
+#include "ksel_internal.h"
+
+namespace ksel {
+
+static std::atomic<int64_t> g_launches{0};
+void note_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+
+struct DevInfo {
+    int sms = 0;
+    int major = 0;
+    int minor = 0;
+};
+
+static std::mutex g_dev_mu;
+static DevInfo g_dev[64];
+static bool g_dev_ok[64];
+
+static int current_device_info(DevInfo* out) {
+    int dev = -1;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return KSEL_ERR_NO_DEVICE;
+    std::lock_guard<std::mutex> lock(g_dev_mu);
+    if (!g_dev_ok[dev]) {
+        cudaDeviceProp p;
+        if (cudaGetDeviceProperties(&p, dev) != cudaSuccess) return KSEL_ERR_CUDA;
+        g_dev[dev].sms = p.multiProcessorCount;
+        g_dev[dev].major = p.major;
+        g_dev[dev].minor = p.minor;
+        g_dev_ok[dev] = true;
+    }
+    *out = g_dev[dev];
+    if (out->major != 10) return KSEL_ERR_NO_DEVICE;  // built for sm_100a only
+    return KSEL_OK;
+}
+
+static bool overlaps(const void* a, size_t na, const void* b, size_t nb) {
+    const uintptr_t x = reinterpret_cast<uintptr_t>(a), y = reinterpret_cast<uintptr_t>(b);
+    return x < y + nb && y < x + na;
+}
+
+static int check_select_args(const float* dist, int64_t Q, int64_t N, int k, const float* ov, const int32_t* oi) {
+    if (!dist || !ov || !oi) return KSEL_ERR_INVALID_ARG;
+    if (Q < 1 || N < 1 || N > 0x7fffffffLL || k < 1 || k > N) return KSEL_ERR_INVALID_ARG;
+    if ((reinterpret_cast<uintptr_t>(dist) & 3u) || (reinterpret_cast<uintptr_t>(ov) & 3u) ||
+        (reinterpret_cast<uintptr_t>(oi) & 3u))
+        return KSEL_ERR_INVALID_ARG;
+    if (k > KSEL_MAX_K) return KSEL_ERR_UNSUPPORTED;
+    return KSEL_OK;
+}
+
+}  // namespace ksel
+
+using namespace ksel;
+
+extern "C" {
+
+int ksel_version(void) { return 100; }  // 0.1.0
+
+int64_t ksel_launch_count(void) { return g_launches.load(std::memory_order_relaxed); }
+
+const char* ksel_strerror(int status) {
+    switch (status) {
+        case KSEL_OK: return "success";
+        case KSEL_ERR_INVALID_ARG: return "invalid argument";
+        case KSEL_ERR_UNSUPPORTED: return "unsupported configuration (k > 1024?)";
+        case KSEL_ERR_CUDA: return "CUDA runtime error";
+        case KSEL_ERR_NO_DEVICE: return "no sm_100 (B200) device is current";
+        default: return "unknown ksel status";
+    }
+}
+
+int ksel_select_config(const float* dist, int64_t Q, int64_t N, int k, float* out_val, int32_t* out_idx, int algo,
+                       int warps_per_row, void* stream) {
+    int st = check_select_args(dist, Q, N, k, out_val, out_idx);
+    if (st) return st;
+    if (algo < KSEL_ALGO_AUTO || algo > KSEL_ALGO_POOL) return KSEL_ERR_INVALID_ARG;
+    if (warps_per_row != 0 && warps_per_row != 1 && warps_per_row != 2 && warps_per_row != 4 && warps_per_row != 8)
+        return KSEL_ERR_INVALID_ARG;
+    const size_t in_bytes = (size_t)Q * (size_t)N * 4u, out_bytes = (size_t)Q * (size_t)k * 4u;
+    if (overlaps(dist, in_bytes, out_val, out_bytes) || overlaps(dist, in_bytes, out_idx, out_bytes) ||
+        overlaps(out_val, out_bytes, out_idx, out_bytes))
+        return KSEL_ERR_INVALID_ARG;
+    DevInfo di;
+    st = current_device_info(&di);
+    if (st) return st;
+    const int wpr = warps_per_row ? warps_per_row : stream_warps_per_row(Q, N, di.sms);
+    if (algo == KSEL_ALGO_AUTO) algo = KSEL_ALGO_POOL;
+    cudaError_t e = (algo == KSEL_ALGO_QUEUE)
+                        ? launch_select_stream(dist, Q, N, k, out_val, out_idx, wpr, (cudaStream_t)stream)
+                        : launch_select_pool(dist, Q, N, k, out_val, out_idx, wpr, (cudaStream_t)stream);
+    return e == cudaSuccess ? KSEL_OK : KSEL_ERR_CUDA;
+}
+
+int ksel_select(const float* dist, int64_t Q, int64_t N, int k, float* out_val, int32_t* out_idx,
+                void* stream) {
+    return ksel_select_config(dist, Q, N, k, out_val, out_idx, KSEL_ALGO_AUTO, 0, stream);
+}
+
+int ksel_merge(const float* cand_val, const int32_t* cand_idx, int64_t Q, int S, int kin, int k, float* out_val,
+               int32_t* out_idx, void* stream) {
+    if (!cand_val || !cand_idx || !out_val || !out_idx) return KSEL_ERR_INVALID_ARG;
+    if (Q < 1 || S < 1 || S > 64 || kin < 1 || k < 1 || (int64_t)k > (int64_t)S * kin) return KSEL_ERR_INVALID_ARG;
+    if (kin > KSEL_MAX_K || k > KSEL_MAX_K) return KSEL_ERR_UNSUPPORTED;
+    const size_t in_b = (size_t)S * (size_t)Q * (size_t)kin * 4u, out_b = (size_t)Q * (size_t)k * 4u;
+    if (overlaps(cand_val, in_b, out_val, out_b) || overlaps(cand_val, in_b, out_idx, out_b) ||
+        overlaps(cand_idx, in_b, out_val, out_b) || overlaps(cand_idx, in_b, out_idx, out_b) ||
+        overlaps(out_val, out_b, out_idx, out_b))
+        return KSEL_ERR_INVALID_ARG;
+    DevInfo di;
+    int st = current_device_info(&di);
+    if (st) return st;
+    cudaError_t e = launch_merge(cand_val, cand_idx, Q, S, kin, k, out_val, out_idx, (cudaStream_t)stream);
+    return e == cudaSuccess ? KSEL_OK : KSEL_ERR_CUDA;
+}
+
+// ---------------------------------------------------------------------------
+// host-buffer pipeline (end-to-end entry point)
+// ---------------------------------------------------------------------------
+static const size_t kHostSlotTarget = 256ull << 20;  // bytes of input per pipeline slot
+
+static size_t al256(size_t x) { return (x + 255u) & ~(size_t)255u; }
+
+// bytes of one pipeline slot holding `rows` rows: [dist | out_val | out_idx], 256-B aligned parts
+static size_t host_slot_bytes(int64_t rows, int64_t N, int k) {
+    return al256((size_t)rows * (size_t)N * 4u) + 2u * al256((size_t)rows * (size_t)k * 4u);
+}
+
+static int64_t host_rows_per_slot(int64_t N, int k, size_t work_bytes) {
+    int64_t rows = (int64_t)((work_bytes / 2u) / ((size_t)N * 4u + (size_t)k * 8u));
+    while (rows > 0 && 2u * host_slot_bytes(rows, N, k) > work_bytes) --rows;
+    return rows;
+}
+
+size_t ksel_select_host_workspace(int64_t N, int k) {
+    if (N < 1 || k < 1) return 0;
+    int64_t rows = (int64_t)(kHostSlotTarget / ((size_t)N * 4u));
+    if (rows < 1) rows = 1;
+    return 2u * host_slot_bytes(rows, N, k);
+}
+
+int ksel_select_host(const float* h_dist, int64_t Q, int64_t N, int k, float* h_out_val, int32_t* h_out_idx,
+                     void* d_work, size_t work_bytes, void* stream) {
+    int st = check_select_args(h_dist, Q, N, k, h_out_val, h_out_idx);
+    if (st) return st;
+    if (!d_work) return KSEL_ERR_INVALID_ARG;
+    const int64_t rps = host_rows_per_slot(N, k, work_bytes);
+    if (rps < 1) return KSEL_ERR_INVALID_ARG;
+    DevInfo di;
+    st = current_device_info(&di);
+    if (st) return st;
+    const cudaStream_t cs = (cudaStream_t)stream;
+    const int64_t rows = rps < Q ? rps : Q;
+    const int wpr = stream_warps_per_row(rows, N, di.sms);
+
+    const size_t dist_b = al256((size_t)rps * (size_t)N * 4u), val_b = al256((size_t)rps * (size_t)k * 4u);
+    const size_t slot_b = host_slot_bytes(rps, N, k);
+    uint8_t* base = static_cast<uint8_t*>(d_work);
+    float* sd[2];
+    float* sv[2];
+    int32_t* si[2];
+    for (int s = 0; s < 2; ++s) {
+        uint8_t* p = base + (size_t)s * slot_b;
+        sd[s] = reinterpret_cast<float*>(p);
+        sv[s] = reinterpret_cast<float*>(p + dist_b);
+        si[s] = reinterpret_cast<int32_t*>(p + dist_b + val_b);
+    }
+
+    cudaStream_t h2d = nullptr, d2h = nullptr;
+    cudaEvent_t ev_in[2] = {nullptr, nullptr}, ev_comp[2] = {nullptr, nullptr}, ev_out[2] = {nullptr, nullptr};
+    cudaError_t e = cudaStreamCreateWithFlags(&h2d, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&d2h, cudaStreamNonBlocking);
+    for (int s = 0; s < 2 && e == cudaSuccess; ++s) {
+        e = cudaEventCreateWithFlags(&ev_in[s], cudaEventDisableTiming);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ev_comp[s], cudaEventDisableTiming);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ev_out[s], cudaEventDisableTiming);
+    }
+    int64_t blk = 0;
+    for (int64_t r0 = 0; r0 < Q && e == cudaSuccess; r0 += rows, ++blk) {
+        const int s = (int)(blk & 1);
+        const int64_t nr = (Q - r0 < rows) ? Q - r0 : rows;
+        if (blk >= 2) e = cudaStreamWaitEvent(h2d, ev_comp[s], 0);  // slot input free
+        if (e == cudaSuccess)
+            e = cudaMemcpyAsync(sd[s], h_dist + r0 * N, (size_t)nr * (size_t)N * 4u, cudaMemcpyHostToDevice, h2d);
+        if (e == cudaSuccess) e = cudaEventRecord(ev_in[s], h2d);
+        if (e == cudaSuccess) e = cudaStreamWaitEvent(cs, ev_in[s], 0);
+        if (e == cudaSuccess && blk >= 2) e = cudaStreamWaitEvent(cs, ev_out[s], 0);  // slot output free
+        if (e == cudaSuccess) e = launch_select_pool(sd[s], nr, N, k, sv[s], si[s], wpr, cs);
+        if (e == cudaSuccess) e = cudaEventRecord(ev_comp[s], cs);
+        if (e == cudaSuccess) e = cudaStreamWaitEvent(d2h, ev_comp[s], 0);
+        if (e == cudaSuccess)
+            e = cudaMemcpyAsync(h_out_val + r0 * k, sv[s], (size_t)nr * (size_t)k * 4u, cudaMemcpyDeviceToHost, d2h);
+        if (e == cudaSuccess)
+            e = cudaMemcpyAsync(h_out_idx + r0 * k, si[s], (size_t)nr * (size_t)k * 4u, cudaMemcpyDeviceToHost, d2h);
+        if (e == cudaSuccess) e = cudaEventRecord(ev_out[s], d2h);
+    }
+    if (e == cudaSuccess) e = cudaStreamSynchronize(d2h);
+    for (int s = 0; s < 2; ++s) {
+        if (ev_in[s]) cudaEventDestroy(ev_in[s]);
+        if (ev_comp[s]) cudaEventDestroy(ev_comp[s]);
+        if (ev_out[s]) cudaEventDestroy(ev_out[s]);
+    }
+    if (h2d) cudaStreamDestroy(h2d);
+    if (d2h) cudaStreamDestroy(d2h);
+    return e == cudaSuccess ? KSEL_OK : KSEL_ERR_CUDA;
+}
+
+// knn_search: declared for the ABI; the fused tcgen05 path lives in knn_fused.cu.
+}  // extern "C"

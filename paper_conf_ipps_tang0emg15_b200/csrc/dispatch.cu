@@ -1,0 +1,47 @@
+// dispatch.cu -- runtime k -> queue-size (R = k'/32) dispatch for the kernel
+// families that build.py compiles once per R (select_stream, select_pool, merge).
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "ksel_internal.h"
+
+namespace ksel {
+
+static int queue_regs(int k) {
+    return k <= 32 ? 1 : k <= 64 ? 2 : k <= 128 ? 4 : k <= 256 ? 8 : k <= 512 ? 16 : 32;
+}
+
+int stream_warps_per_row(int64_t Q, int64_t N, int num_sms) {
+    // enough warps to cover every SM several times, but >= 8 chunks per warp
+    const int64_t target = (int64_t)num_sms * 12;
+    int wpr = 1;
+    while (wpr < 8 && Q * wpr < target && N / (1024 * (wpr * 2)) >= 8) wpr *= 2;
+    return wpr;
+}
+
+#define KSEL_DISPATCH_R(FN, R_, ...)                  \
+    switch (R_) {                                     \
+        case 1: return FN<1>(__VA_ARGS__);            \
+        case 2: return FN<2>(__VA_ARGS__);            \
+        case 4: return FN<4>(__VA_ARGS__);            \
+        case 8: return FN<8>(__VA_ARGS__);            \
+        case 16: return FN<16>(__VA_ARGS__);          \
+        default: return FN<32>(__VA_ARGS__);          \
+    }
+
+cudaError_t launch_select_stream(const float* dist, int64_t Q, int64_t N, int k, float* ov, int32_t* oi, int wpr,
+                                 cudaStream_t stream) {
+    KSEL_DISPATCH_R(launch_stream_r, queue_regs(k), dist, Q, N, k, ov, oi, wpr, stream)
+}
+
+cudaError_t launch_select_pool(const float* dist, int64_t Q, int64_t N, int k, float* ov, int32_t* oi, int wpr,
+                               cudaStream_t stream) {
+    KSEL_DISPATCH_R(launch_pool_r, queue_regs(k), dist, Q, N, k, ov, oi, wpr, stream)
+}
+
+cudaError_t launch_merge(const float* cv, const int32_t* ci, int64_t Q, int S, int kin, int k, float* ov,
+                         int32_t* oi, cudaStream_t stream) {
+    KSEL_DISPATCH_R(launch_merge_r, queue_regs(k), cv, ci, Q, S, kin, k, ov, oi, stream)
+}
+
+}  // namespace ksel

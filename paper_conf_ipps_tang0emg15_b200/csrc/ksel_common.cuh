@@ -1,0 +1,233 @@
+// ksel_common.cuh -- device primitives shared by the sm_100a kernels of libksel.
+//
+// * order keys (fp32 -> ordered u32 with -0.0/NaN canonicalised), R3-R5;
+// * warp-distributed sorted arrays of (key, idx) pairs and the bitonic networks
+//   over them (Fig. 2 "Bitonic Merge" / "Reverse Bitonic
+//   Merge"; the "flip" stage is the reverse merge's cross-compare);
+// * mbarrier + cp.async.bulk (TMA bulk copy) helpers for the streaming stage.
+//
+// Layout of a warp array with R registers per lane: element e = r*32 + lane
+// lives in register r of lane `lane`.  Strides >= 32 are in-register
+// compare-exchanges, strides < 32 use __shfl_xor_sync.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace ksel {
+
+constexpr unsigned kFull = 0xffffffffu;
+constexpr uint32_t kSentKey = 0xffffffffu;  // sentinel pair (kSentKey, kSentIdx) is
+constexpr uint32_t kSentIdx = 0x7fffffffu;  // greater than every real pair (idx < 2^31-1)
+
+// fp32 bits -> order-preserving u32 key.  -0.0 and +0.0 map to the same key
+// (0x80000000), every NaN maps to 0xffffffff (above +Inf = 0xff800000).
+__device__ __forceinline__ uint32_t key_of_bits(uint32_t b) {
+    const uint32_t mag = b & 0x7fffffffu;
+    uint32_t key = b ^ ((uint32_t)((int32_t)b >> 31) | 0x80000000u);
+    key = (mag == 0u) ? 0x80000000u : key;
+    key = (mag > 0x7f800000u) ? 0xffffffffu : key;
+    return key;
+}
+__device__ __forceinline__ uint32_t key_of(float x) { return key_of_bits(__float_as_uint(x)); }
+
+// Inverse of key_of_bits for every non-canonicalised key (all values except
+// -0.0 and NaN payloads, which callers re-gather from the input).
+__device__ __forceinline__ uint32_t bits_of_key(uint32_t key) {
+    return (key & 0x80000000u) ? (key & 0x7fffffffu) : ~key;
+}
+__device__ __forceinline__ bool key_needs_regather(uint32_t key) {
+    return key == 0x80000000u || key == 0xffffffffu;
+}
+
+// Lexicographic (key, idx) "strictly before".
+__device__ __forceinline__ bool pair_lt(uint32_t ka, uint32_t ia, uint32_t kb, uint32_t ib) {
+    return (ka < kb) || (ka == kb && ia < ib);
+}
+
+__device__ __forceinline__ uint32_t lane_id() {
+    uint32_t l;
+    asm volatile("mov.u32 %0, %%laneid;" : "=r"(l));
+    return l;
+}
+__device__ __forceinline__ uint32_t lanemask_lt() {
+    uint32_t m;
+    asm volatile("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+    return m;
+}
+
+// ---------------------------------------------------------------------------
+// Warp-distributed arrays and bitonic networks
+// ---------------------------------------------------------------------------
+template <int R>
+struct WArr {
+    uint32_t k[R];
+    uint32_t i[R];
+};
+
+template <int R>
+__device__ __forceinline__ void warr_fill_sentinel(WArr<R>& a) {
+#pragma unroll
+    for (int r = 0; r < R; ++r) { a.k[r] = kSentKey; a.i[r] = kSentIdx; }
+}
+
+// In-register compare-exchange: lower position gets the smaller pair when asc.
+__device__ __forceinline__ void cx_reg(uint32_t& ka, uint32_t& ia, uint32_t& kb, uint32_t& ib, bool asc) {
+    const bool swap = asc ? pair_lt(kb, ib, ka, ia) : pair_lt(ka, ia, kb, ib);
+    const uint32_t tk = ka, ti = ia;
+    ka = swap ? kb : ka; ia = swap ? ib : ia;
+    kb = swap ? tk : kb; ib = swap ? ti : ib;
+}
+
+// Cross-lane compare-exchange at lane stride s: this lane keeps the min when
+// `keep_min`, else the max, of (own, partner).
+__device__ __forceinline__ void cx_lane(uint32_t& k, uint32_t& i, int s, bool keep_min) {
+    const uint32_t ok = __shfl_xor_sync(kFull, k, s);
+    const uint32_t oi = __shfl_xor_sync(kFull, i, s);
+    const bool other_first = pair_lt(ok, oi, k, i);
+    const bool take = keep_min ? other_first : pair_lt(k, i, ok, oi);
+    k = take ? ok : k;
+    i = take ? oi : i;
+}
+
+// In-register bitonic stage (stride s >= 32, compile time) of the network
+// whose direction is set by bit m of the element position (m = 0: ascending).
+template <int R, int s>
+__device__ __forceinline__ void reg_stage(WArr<R>& a, int m) {
+    constexpr int rs = s >> 5;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        if ((r & rs) == 0) {
+            // direction from bit m of the position r*32+lane (m > s >= 32: a register bit)
+            const bool asc = (m == 0) ? true : (((r << 5) & m) == 0);
+            cx_reg(a.k[r], a.i[r], a.k[r | rs], a.i[r | rs], asc);
+        }
+    }
+}
+
+// Cross-lane stages s_hi, s_hi/2, ..., 1 (s_hi <= 16).  Kept as a runtime loop:
+// the body is the same for every stride, which keeps the code (and ptxas time)
+// small for large queues; the register index stays compile-time.
+template <int R>
+__device__ __forceinline__ void lane_stages(WArr<R>& a, int s_hi, int m, uint32_t lane) {
+#pragma unroll 1
+    for (int s = s_hi; s >= 1; s >>= 1) {
+        const bool lower = (lane & (uint32_t)s) == 0u;
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            const bool asc = (m == 0) ? true : (((m >= 32) ? ((r << 5) & m) : (int)(lane & (uint32_t)m)) == 0);
+            cx_lane(a.k[r], a.i[r], s, lower == asc);
+        }
+    }
+}
+
+template <int R, int s>
+__device__ __forceinline__ void reg_stages_from(WArr<R>& a, int m) {
+    if constexpr (s >= 32) {
+        reg_stage<R, s>(a, m);
+        reg_stages_from<R, (s >> 1)>(a, m);
+    }
+}
+
+template <int R, int M>
+__device__ __forceinline__ void sort_levels_from(WArr<R>& a, uint32_t lane) {
+    if constexpr (M <= 32 * R) {
+        const int dirbit = (M == 32 * R) ? 0 : M;
+        reg_stages_from<R, (M >> 1)>(a, dirbit);
+        lane_stages<R>(a, 16, dirbit, lane);
+        sort_levels_from<R, (M << 1)>(a, lane);
+    }
+}
+
+// Full bitonic sort, ascending, of the 32*R elements.
+template <int R>
+__device__ __forceinline__ void warr_sort(WArr<R>& a, uint32_t lane) {
+    // levels whose blocks fit inside a warp (m <= 32): cross-lane stages only
+#pragma unroll 1
+    for (int m = 2; m <= 32; m <<= 1) lane_stages<R>(a, m >> 1, (m == 32 * R) ? 0 : m, lane);
+    sort_levels_from<R, 64>(a, lane);
+}
+
+// Bitonic clean: sorts ascending a bitonic sequence of 32*R elements.
+template <int R>
+__device__ __forceinline__ void warr_clean(WArr<R>& a, uint32_t lane) {
+    reg_stages_from<R, 16 * R>(a, 0);
+    lane_stages<R>(a, 16, 0, lane);
+}
+
+// Keep the 32*R smallest of (q ∪ b); q and b sorted ascending (b has 32*RB
+// elements, RB may differ from R).  "Flip" stage of the Reverse Bitonic Merge
+// (PAPER.md L139): q[p] = min(q[p], b[L-1-p']) over the overlapping tail,
+// which leaves a bitonic sequence holding exactly the 32*R smallest, then a
+// bitonic clean.  The Merge Queue's lazy update is that this
+// runs only when a buffer flushes.
+template <int R, int RB>
+__device__ __forceinline__ void warr_merge(WArr<R>& q, const WArr<RB>& b, uint32_t lane) {
+    constexpr int RE = (RB < R) ? RB : R;
+#pragma unroll
+    for (int t = 0; t < RE; ++t) {
+        const int qr = R - RE + t;
+        const int br = RE - 1 - t;
+        const uint32_t bk = __shfl_xor_sync(kFull, b.k[br], 31);
+        const uint32_t bi = __shfl_xor_sync(kFull, b.i[br], 31);
+        const bool take = pair_lt(bk, bi, q.k[qr], q.i[qr]);
+        q.k[qr] = take ? bk : q.k[qr];
+        q.i[qr] = take ? bi : q.i[qr];
+    }
+    warr_clean<R>(q, lane);
+}
+
+// Pair at (0-based) position pos of a warp array, broadcast to all lanes.
+template <int R>
+__device__ __forceinline__ void warr_get(const WArr<R>& a, int pos, uint32_t& k, uint32_t& i) {
+    const int rr = pos >> 5;
+    uint32_t tk = 0, ti = 0;
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+        if (r == rr) { tk = a.k[r]; ti = a.i[r]; }
+    k = __shfl_sync(kFull, tk, pos & 31);
+    i = __shfl_sync(kFull, ti, pos & 31);
+}
+
+// ---------------------------------------------------------------------------
+// mbarrier / bulk async copy (TMA non-tensor) helpers
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.release.cta.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+                 "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+    return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    while (!mbar_try_wait(bar, parity)) {
+    }
+}
+// 1-D bulk copy global -> shared, completion signalled on `bar` (complete_tx).
+// dst/src 16-byte aligned, bytes a multiple of 16.
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            smem_u32(dst)),
+        "l"(src), "r"(bytes), "r"(smem_u32(bar))
+        : "memory");
+}
+
+}  // namespace ksel

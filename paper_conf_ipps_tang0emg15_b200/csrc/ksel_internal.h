@@ -1,0 +1,38 @@
+// ksel_internal.h -- host-side declarations shared by the translation units of
+// libksel.so (not part of the public ABI; see include/ksel.h).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace ksel {
+
+constexpr int kMaxSmemPerBlock = 227 * 1024;  // sm_100 opt-in dynamic shared memory per CTA
+
+// Count one enqueued kernel (reported through ksel_launch_count()).
+void note_launch();
+
+// Streaming selection (select_stream.cu).
+int stream_warps_per_row(int64_t Q, int64_t N, int num_sms);
+cudaError_t launch_select_stream(const float* dist, int64_t Q, int64_t N, int k, float* out_val,
+                                 int32_t* out_idx, int wpr, cudaStream_t stream);
+
+// Pool + radix-narrowing selection (select_pool.cu).
+cudaError_t launch_select_pool(const float* dist, int64_t Q, int64_t N, int k, float* out_val, int32_t* out_idx,
+                               int wpr, cudaStream_t stream);
+
+// Merge of S sorted candidate lists (merge.cu).
+cudaError_t launch_merge(const float* cand_val, const int32_t* cand_idx, int64_t Q, int S, int kin,
+                         int k, float* out_val, int32_t* out_idx, cudaStream_t stream);
+
+// Per-queue-size entry points (explicitly instantiated, one object per R).
+template <int R>
+cudaError_t launch_stream_r(const float* dist, int64_t Q, int64_t N, int k, float* ov, int32_t* oi, int wpr,
+                            cudaStream_t stream);
+template <int R>
+cudaError_t launch_pool_r(const float* dist, int64_t Q, int64_t N, int k, float* ov, int32_t* oi, int wpr,
+                          cudaStream_t stream);
+template <int R>
+cudaError_t launch_merge_r(const float* cv, const int32_t* ci, int64_t Q, int S, int kin, int k, float* ov,
+                           int32_t* oi, cudaStream_t stream);
+
+}  // namespace ksel

@@ -1,0 +1,131 @@
+// KSEL_SPLIT_R
+// merge.cu -- ksel_merge: per-query merge of S sorted candidate lists.
+//
+// The final step of divide-and-merge (ref. [18]) and of the
+// row-sharded k-NN after the NCCL all-gather.  One warp per
+// query keeps a register-resident sorted queue of k' = max(32, 2^ceil(log2 k))
+// pairs; each list is merged in with the Reverse Bitonic Merge "flip" + clean
+// (Fig. 2; Merge Queue levels merged lazily, L41).  Lists are
+// checked for sortedness with one neighbour compare per element and sorted in
+// the warp if a caller hands in an unsorted list, so the result is the exact
+// top-k of the union either way.
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "ksel_common.cuh"
+#include "ksel_internal.h"
+
+#ifndef KSEL_ONLY_R
+#error "compile once per queue size with -DKSEL_ONLY_R=1|2|4|8|16|32"
+#endif
+
+namespace ksel {
+
+constexpr int kMergeWarps = 4;
+
+template <int RL>
+__device__ __forceinline__ bool warr_is_sorted(const WArr<RL>& a, uint32_t lane) {
+    bool bad = false;
+#pragma unroll
+    for (int r = 0; r < RL; ++r) {
+        uint32_t nk = __shfl_down_sync(kFull, a.k[r], 1);
+        uint32_t ni = __shfl_down_sync(kFull, a.i[r], 1);
+        if (r + 1 < RL) {
+            const uint32_t hk = __shfl_sync(kFull, a.k[r + 1], 0);
+            const uint32_t hi = __shfl_sync(kFull, a.i[r + 1], 0);
+            if (lane == 31) { nk = hk; ni = hi; }
+        }
+        const bool has_next = (lane < 31) || (r + 1 < RL);
+        bad |= has_next && pair_lt(nk, ni, a.k[r], a.i[r]);
+    }
+    return !__any_sync(kFull, bad);
+}
+
+template <int R, int RL>
+__global__ void __launch_bounds__(32 * kMergeWarps)
+    ksel_merge_kernel(const float* __restrict__ cv, const int32_t* __restrict__ ci, int64_t Q, int S, int kin,
+                      int k, float* __restrict__ out_val, int32_t* __restrict__ out_idx) {
+    const uint32_t lane = lane_id();
+    const int64_t q = (int64_t)blockIdx.x * kMergeWarps + (threadIdx.x >> 5);
+    if (q >= Q) return;
+    constexpr int LN = 32 * RL;  // list elements merged per step (<= k')
+
+    WArr<R> acc;
+    warr_fill_sentinel<R>(acc);
+#pragma unroll 1
+    for (int s = 0; s < S; ++s) {
+        const int64_t base = ((int64_t)s * Q + q) * kin;
+        // A list longer than k' is folded in whole, k' at a time (only its k'
+        // smallest can matter, but finding them must not assume sortedness).
+#pragma unroll 1
+        for (int off = 0; off < kin; off += LN) {
+            WArr<RL> b;
+#pragma unroll
+            for (int r = 0; r < RL; ++r) {
+                const int e = off + r * 32 + (int)lane;
+                b.k[r] = (e < kin) ? key_of(cv[base + e]) : kSentKey;
+                b.i[r] = (e < kin) ? (uint32_t)ci[base + e] : kSentIdx;
+            }
+            const bool sorted = (kin <= LN) && warr_is_sorted<RL>(b, lane);
+            if (!sorted) warr_sort<RL>(b, lane);
+            warr_merge<R, RL>(acc, b, lane);
+        }
+    }
+
+    float* ov = out_val + q * (int64_t)k;
+    int32_t* oi = out_idx + q * (int64_t)k;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const int e = r * 32 + (int)lane;
+        if (e < k) {
+            const uint32_t key = acc.k[r];
+            const uint32_t idx = acc.i[r];
+            uint32_t bits = bits_of_key(key);
+            if (key_needs_regather(key)) {  // -0.0 / NaN payload: find the candidate's own bits
+                for (int s = 0; s < S; ++s) {
+                    const int64_t base = ((int64_t)s * Q + q) * kin;
+                    bool found = false;
+                    for (int t = 0; t < kin; ++t)
+                        if ((uint32_t)ci[base + t] == idx && key_of(cv[base + t]) == key) {
+                            bits = __float_as_uint(cv[base + t]);
+                            found = true;
+                            break;
+                        }
+                    if (found) break;
+                }
+            }
+            ov[e] = __uint_as_float(bits);
+            oi[e] = (int32_t)idx;
+        }
+    }
+}
+
+template <int R, int RL>
+static cudaError_t launch_merge_rl(const float* cv, const int32_t* ci, int64_t Q, int S, int kin, int k, float* ov,
+                                   int32_t* oi, cudaStream_t stream) {
+    const int64_t grid = (Q + kMergeWarps - 1) / kMergeWarps;
+    ksel_merge_kernel<R, RL><<<(unsigned)grid, 32 * kMergeWarps, 0, stream>>>(cv, ci, Q, S, kin, k, ov, oi);
+    note_launch();
+    return cudaGetLastError();
+}
+
+template <int R>
+cudaError_t launch_merge_r(const float* cv, const int32_t* ci, int64_t Q, int S, int kin, int k, float* ov,
+                                  int32_t* oi, cudaStream_t stream) {
+    const int lp = kin <= 32 ? 1 : kin <= 64 ? 2 : kin <= 128 ? 4 : kin <= 256 ? 8 : kin <= 512 ? 16 : 32;
+    const int rl = lp < R ? lp : R;
+    switch (rl) {
+        case 1: return launch_merge_rl<R, 1>(cv, ci, Q, S, kin, k, ov, oi, stream);
+        case 2: if constexpr (R >= 2) return launch_merge_rl<R, 2>(cv, ci, Q, S, kin, k, ov, oi, stream); break;
+        case 4: if constexpr (R >= 4) return launch_merge_rl<R, 4>(cv, ci, Q, S, kin, k, ov, oi, stream); break;
+        case 8: if constexpr (R >= 8) return launch_merge_rl<R, 8>(cv, ci, Q, S, kin, k, ov, oi, stream); break;
+        case 16: if constexpr (R >= 16) return launch_merge_rl<R, 16>(cv, ci, Q, S, kin, k, ov, oi, stream); break;
+        case 32: if constexpr (R >= 32) return launch_merge_rl<R, 32>(cv, ci, Q, S, kin, k, ov, oi, stream); break;
+    }
+    return cudaErrorInvalidValue;
+}
+
+template cudaError_t launch_merge_r<KSEL_ONLY_R>(const float*, const int32_t*, int64_t, int, int, int, float*,
+                                                 int32_t*, cudaStream_t);
+
+}  // namespace ksel

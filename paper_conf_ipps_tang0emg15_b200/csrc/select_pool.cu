@@ -1,0 +1,482 @@
+// KSEL_SPLIT_R
+// select_pool.cu -- streaming k-selection with radix threshold narrowing (sm_100a).
+//
+// Same staging and filter as select_stream.cu (a1/a2: TMA bulk copies into a
+// per-warp shared-memory ring, fp32 pre-filter against the running k-th pair,
+// exact lexicographic test), but candidates are NOT merged into a sorted queue
+// as they arrive.  They are appended, warp-aggregated, to an unordered
+// per-warp candidate pool in shared memory (Buffered Search's candidate
+// buffer, sized P >= k' + 256).  When the pool fills, an
+// MSD radix-histogram select over the pool (8-bit digits of the order key,
+// then of the index for ties) finds the exact k-th pair of everything seen so
+// far; the pool is compacted to those k pairs and the pair becomes the new
+// threshold.  This is the paper's Hierarchical Partition idea -- discard whole
+// groups that cannot hold a k-NN ("if any element in the
+// upper level does not belong to k-NN, none of the elements in its sub-groups
+// would") -- with value buckets instead of index groups and a fixed number of
+// steps (<= 8 digit passes) instead of log_G(N/k) (L231); radix select [12]
+// (L15) is the digit order.
+//
+// At the end of the row the k surviving pairs are bitonic-sorted in the warp
+// (Local Sort / Reverse Bitonic Merge networks), the
+// W warps of a row are merged pairwise (divide-and-merge, L243), and the row's
+// top-k is emitted ascending by (value, index).
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "ksel_common.cuh"
+#include "ksel_internal.h"
+
+#ifndef KSEL_ONLY_R
+#error "compile once per queue size with -DKSEL_ONLY_R=1|2|4|8|16|32"
+#endif
+
+namespace ksel {
+
+template <int R, int WPR, int RPC>
+struct PoolCfg {
+    static constexpr int kQueue = 32 * R;  // k'
+    static constexpr int kPool = (2 * kQueue > kQueue + 256) ? 2 * kQueue : kQueue + 256;
+    static constexpr int CH = 1024;        // floats per staged chunk
+    static constexpr int S = 3;            // ring stages per warp
+    static constexpr int G = 2;            // float4 per lane per sub-step (256 elements per warp)
+    static constexpr int NS = 4 * G;       // element slots per lane per sub-step
+    static constexpr int kWarps = WPR * RPC;
+    static constexpr int kThreads = 32 * kWarps;
+    static constexpr int kRingBytes = S * CH * 4;
+    // per warp: ring | pool keys | pool idx | histogram (256 u32) | mbarriers
+    static constexpr int kWarpBytes = kRingBytes + kPool * 8 + 256 * 4 + S * 8;
+    static constexpr int kWarpStride = (kWarpBytes + 127) / 128 * 128;
+    static constexpr int kGroupBytes = 128;
+    static constexpr int kSmem = RPC * kGroupBytes + kWarps * kWarpStride;
+    static_assert(kPool % 32 == 0, "pool size");
+    static_assert(kPool >= kQueue + 32 * NS, "a full sub-step must fit after compaction");
+};
+
+__device__ __forceinline__ void pool_group_bar(int id, int nthreads) {
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
+
+// Exclusive warp prefix sum of v; total in `total`.
+__device__ __forceinline__ uint32_t warp_excl_scan(uint32_t v, uint32_t lane, uint32_t& total) {
+    uint32_t inc = v;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t t = __shfl_up_sync(kFull, inc, d);
+        if (lane >= (uint32_t)d) inc += t;
+    }
+    total = __shfl_sync(kFull, inc, 31);
+    return inc - v;
+}
+
+// Histogram bins are stored transposed (bin b at (b & 7) * 32 + (b >> 3)) so
+// that lane l reading its 8 bins 8l..8l+7 hits 8 distinct banks per access.
+__device__ __forceinline__ int hist_slot(uint32_t b) { return (int)((b & 7u) * 32u + (b >> 3)); }
+
+// Locate the bucket holding the want-th (1-based) element from a filled
+// histogram: returns the digit; `want` becomes the rank inside that bucket and
+// `cnt` the bucket's population.
+__device__ __forceinline__ uint32_t hist_find(const uint32_t* hist, uint32_t lane, uint32_t& want, uint32_t& cnt) {
+    uint32_t h[8], s = 0;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+        h[j] = hist[j * 32 + lane];
+        s += h[j];
+    }
+    uint32_t total;
+    const uint32_t excl = warp_excl_scan(s, lane, total);
+    const bool mine = excl < want && want <= excl + s;
+    const uint32_t bal = __ballot_sync(kFull, mine);
+    const int src = __ffs(bal) - 1;
+    uint32_t d = 0, before = excl, c = 0;
+    if (mine) {
+        uint32_t acc = excl;
+        bool done = false;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            if (!done && acc + h[j] >= want) {
+                d = lane * 8u + (uint32_t)j;
+                before = acc;
+                c = h[j];
+                done = true;
+            }
+            acc += h[j];
+        }
+    }
+    d = __shfl_sync(kFull, d, src);
+    before = __shfl_sync(kFull, before, src);
+    cnt = __shfl_sync(kFull, c, src);
+    want -= before;
+    return d;
+}
+
+// Exact want-th smallest (key, idx) pair among pool[0..n), want in [1, n].
+// MSD radix select, 8-bit digits: 4 passes over the key, then (only if the
+// k-th key value is tied beyond the rank needed) 4 passes over the index.
+static __device__ __noinline__ unsigned long long pool_kth(const uint32_t* __restrict__ pk, const uint32_t* __restrict__ pi,
+                                                    int n, uint32_t want, uint32_t* __restrict__ hist) {
+    const uint32_t lane = lane_id();
+    uint32_t prefix = 0, cnt = 0;
+#pragma unroll 1
+    for (int pass = 0; pass < 4; ++pass) {
+        const int shift = 24 - 8 * pass;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) hist[j * 32 + lane] = 0u;
+        __syncwarp();
+        for (int e = (int)lane; e < n; e += 32) {
+            const uint32_t key = pk[e];
+            const bool sel = (pass == 0) || ((key ^ prefix) >> (shift + 8)) == 0u;
+            if (sel) atomicAdd(&hist[hist_slot((key >> shift) & 255u)], 1u);
+        }
+        __syncwarp();
+        const uint32_t d = hist_find(hist, lane, want, cnt);
+        prefix |= d << shift;
+        __syncwarp();
+    }
+    const uint32_t vkey = prefix;
+    uint32_t idx;
+    if (cnt == want) {
+        // every tie of the k-th key is needed: the threshold is the largest such index
+        uint32_t m = 0;
+        for (int e = (int)lane; e < n; e += 32)
+            if (pk[e] == vkey) m = max(m, pi[e]);
+        idx = __reduce_max_sync(kFull, m);
+    } else {
+        uint32_t ip = 0;
+#pragma unroll 1
+        for (int pass = 0; pass < 4; ++pass) {
+            const int shift = 24 - 8 * pass;
+#pragma unroll
+            for (int j = 0; j < 8; ++j) hist[j * 32 + lane] = 0u;
+            __syncwarp();
+            for (int e = (int)lane; e < n; e += 32) {
+                if (pk[e] != vkey) continue;
+                const uint32_t id = pi[e];
+                const bool sel = (pass == 0) || ((id ^ ip) >> (shift + 8)) == 0u;
+                if (sel) atomicAdd(&hist[hist_slot((id >> shift) & 255u)], 1u);
+            }
+            __syncwarp();
+            const uint32_t d = hist_find(hist, lane, want, cnt);
+            ip |= d << shift;
+            __syncwarp();
+        }
+        idx = ip;
+    }
+    return ((unsigned long long)vkey << 32) | idx;
+}
+
+// In-place compaction of pool[0..n) to the pairs <= (tk, ti); returns the new count.
+static __device__ __noinline__ int pool_compact(uint32_t* __restrict__ pk, uint32_t* __restrict__ pi, int n, uint32_t tk,
+                                         uint32_t ti) {
+    const uint32_t lane = lane_id();
+    const uint32_t lt = lanemask_lt();
+    int w = 0;
+    for (int base = 0; base < n; base += 32) {
+        const int e = base + (int)lane;
+        uint32_t kk = 0, ii = 0;
+        bool keep = false;
+        if (e < n) {
+            kk = pk[e];
+            ii = pi[e];
+            keep = !pair_lt(tk, ti, kk, ii);
+        }
+        const uint32_t bal = __ballot_sync(kFull, keep);
+        __syncwarp();
+        if (keep) {
+            const int pos = w + __popc(bal & lt);
+            pk[pos] = kk;
+            pi[pos] = ii;
+        }
+        w += __popc(bal);
+        __syncwarp();
+    }
+    return w;
+}
+
+// Sort pool[0..n) (n <= k') ascending into pool[0..k') with sentinel padding.
+template <int R>
+__device__ __noinline__ void pool_sort(uint32_t* __restrict__ pk, uint32_t* __restrict__ pi, int n) {
+    const uint32_t lane = lane_id();
+    WArr<R> a;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const int e = r * 32 + (int)lane;
+        a.k[r] = (e < n) ? pk[e] : kSentKey;
+        a.i[r] = (e < n) ? pi[e] : kSentIdx;
+    }
+    __syncwarp();
+    warr_sort<R>(a, lane);
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        pk[r * 32 + lane] = a.k[r];
+        pi[r * 32 + lane] = a.i[r];
+    }
+    __syncwarp();
+}
+
+// Merge of two sorted k'-lists in shared memory: (qk, qi) <- k' smallest.
+template <int R>
+__device__ __noinline__ void pool_merge_sorted(uint32_t* __restrict__ qk, uint32_t* __restrict__ qi,
+                                               const uint32_t* __restrict__ pk, const uint32_t* __restrict__ pi) {
+    const uint32_t lane = lane_id();
+    WArr<R> q, b;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        q.k[r] = qk[r * 32 + lane];
+        q.i[r] = qi[r * 32 + lane];
+        b.k[r] = pk[r * 32 + lane];
+        b.i[r] = pi[r * 32 + lane];
+    }
+    warr_merge<R, R>(q, b, lane);
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        qk[r * 32 + lane] = q.k[r];
+        qi[r * 32 + lane] = q.i[r];
+    }
+    __syncwarp();
+}
+
+template <int R, int WPR, int RPC>
+__global__ void __launch_bounds__(PoolCfg<R, WPR, RPC>::kThreads)
+    ksel_pool_kernel(const float* __restrict__ dist, int64_t Q, int64_t N, int k, float* __restrict__ out_val,
+                     int32_t* __restrict__ out_idx) {
+    using Cfg = PoolCfg<R, WPR, RPC>;
+    constexpr int CH = Cfg::CH, S = Cfg::S, G = Cfg::G, NS = Cfg::NS;
+    extern __shared__ __align__(128) uint8_t smem[];
+
+    const uint32_t lane = lane_id();
+    const int warp = threadIdx.x >> 5;
+    const int grp = warp / WPR;
+    const int wig = warp % WPR;
+    const int64_t row = (int64_t)blockIdx.x * RPC + grp;
+    if (row >= Q) return;
+
+    unsigned long long* grp_thr = reinterpret_cast<unsigned long long*>(smem + grp * Cfg::kGroupBytes);
+    uint8_t* wbase = smem + RPC * Cfg::kGroupBytes + warp * Cfg::kWarpStride;
+    float* ring = reinterpret_cast<float*>(wbase);
+    uint32_t* pk = reinterpret_cast<uint32_t*>(wbase + Cfg::kRingBytes);
+    uint32_t* pi = pk + Cfg::kPool;
+    uint32_t* hist = pi + Cfg::kPool;
+    uint64_t* mbar = reinterpret_cast<uint64_t*>(hist + 256);
+
+    // ---- row geometry -----------------------------------------------------------
+    const uint64_t g0 = (uint64_t)row * (uint64_t)N;
+    const uint64_t g1 = g0 + (uint64_t)N;
+    const uint64_t mis = ((reinterpret_cast<uintptr_t>(dist) >> 2) + g0) & 3u;
+    uint64_t a0 = g0 + ((4u - mis) & 3u);
+    if (a0 > g1) a0 = g1;
+    const uint64_t a1 = a0 + ((g1 - a0) & ~3ull);
+    const uint64_t nch = (a1 - a0 + CH - 1) / CH;
+    const uint64_t c_begin = nch * wig / WPR;
+    const uint64_t c_end = nch * (wig + 1) / WPR;
+    const int nmine = (int)(c_end - c_begin);
+
+    auto chunk_len = [&](uint64_t c) -> uint32_t {
+        const uint64_t s0 = a0 + c * CH;
+        const uint64_t s1 = (s0 + CH < a1) ? s0 + CH : a1;
+        return (uint32_t)(s1 - s0);
+    };
+    auto issue = [&](int li) {
+        const uint64_t c = c_begin + li;
+        const int st = li % S;
+        const uint32_t bytes = chunk_len(c) * 4u;
+        mbar_arrive_expect_tx(&mbar[st], bytes);
+        bulk_g2s(ring + st * CH, dist + a0 + c * CH, bytes, &mbar[st]);
+    };
+
+    if (lane == 0) {
+        for (int s = 0; s < S; ++s) mbar_init(&mbar[s], 1);
+        fence_mbar_init();
+        for (int li = 0; li < S && li < nmine; ++li) issue(li);
+    }
+    if (WPR > 1 && wig == 0 && lane == 0) *grp_thr = 0xffffffffffffffffull;
+    __syncwarp();
+    if (WPR > 1) pool_group_bar(1 + grp, 32 * WPR);
+
+    // ---- state ----------------------------------------------------------------------
+    uint32_t Tk = kSentKey, Ti = kSentIdx;
+    float tv = 0.f;
+    bool fast = false;
+    int n = 0;
+
+    auto tighten = [&](uint32_t kk, uint32_t ki) {
+        if (pair_lt(kk, ki, Tk, Ti)) { Tk = kk; Ti = ki; }
+        fast = Tk < 0xff800000u;
+        tv = __uint_as_float(bits_of_key(Tk));
+    };
+    // pool full: exact k-th of everything seen so far becomes the threshold
+    auto narrow = [&]() {
+        const unsigned long long t = pool_kth(pk, pi, n, (uint32_t)k, hist);
+        const uint32_t kk = (uint32_t)(t >> 32), ki = (uint32_t)t;
+        n = pool_compact(pk, pi, n, kk, ki);
+        tighten(kk, ki);
+        if (WPR > 1 && lane == 0) atomicMin(grp_thr, t);
+    };
+    // append the candidates flagged in `mask` (slot j: key[j], col[j]) after the exact test
+    auto absorb = [&](uint32_t mask, const auto& key, const auto& col) {
+        constexpr int ns = (int)(sizeof(key) / sizeof(key[0]));
+        uint32_t m = 0;
+#pragma unroll
+        for (int j = 0; j < ns; ++j)
+            if (((mask >> j) & 1u) && pair_lt(key[j], col[j], Tk, Ti)) m |= 1u << j;
+        uint32_t total;
+        uint32_t excl = warp_excl_scan(__popc(m), lane, total);
+        if (total == 0) return;
+        if (n + (int)total > Cfg::kPool) {
+            narrow();
+            uint32_t m2 = 0;
+#pragma unroll
+            for (int j = 0; j < ns; ++j)
+                if (((m >> j) & 1u) && pair_lt(key[j], col[j], Tk, Ti)) m2 |= 1u << j;
+            m = m2;
+            excl = warp_excl_scan(__popc(m), lane, total);
+        }
+        int pos = n + (int)excl;
+#pragma unroll
+        for (int j = 0; j < ns; ++j)
+            if ((m >> j) & 1u) {
+                pk[pos] = key[j];
+                pi[pos] = col[j];
+                ++pos;
+            }
+        n += (int)total;
+        __syncwarp();
+    };
+
+    // ---- unaligned head and tail ---------------------------------------------------------
+    if (wig == 0) {
+        const uint32_t nh = (uint32_t)(a0 - g0), nt = (uint32_t)(g1 - a1);
+        bool valid = false;
+        uint64_t g = 0;
+        if (lane < nh) { valid = true; g = g0 + lane; }
+        else if (lane < nh + nt) { valid = true; g = a1 + (lane - nh); }
+        uint32_t key[1], col[1];
+        key[0] = valid ? key_of(dist[g]) : kSentKey;
+        col[0] = (uint32_t)(g - g0);
+        absorb(valid ? 1u : 0u, key, col);
+    }
+
+    // ---- streaming body ------------------------------------------------------------------
+    for (int li = 0; li < nmine; ++li) {
+        const int st = li % S;
+        const uint64_t c = c_begin + li;
+        const uint32_t len = chunk_len(c);
+        const uint32_t col0 = (uint32_t)(a0 + c * CH - g0);
+        if (WPR > 1) {
+            const unsigned long long sh = *reinterpret_cast<volatile unsigned long long*>(grp_thr);
+            tighten((uint32_t)(sh >> 32), (uint32_t)sh);
+        }
+        mbar_wait(&mbar[st], (uint32_t)(li / S) & 1u);
+        const float4* src = reinterpret_cast<const float4*>(ring + st * CH);
+#pragma unroll 1
+        for (int g = 0; g < CH / 128; g += G) {
+            float x[NS];
+            uint32_t mask = 0;
+#pragma unroll
+            for (int u = 0; u < G; ++u) {
+                const uint32_t e4 = (uint32_t)(g + u) * 32u + lane;
+                const bool ok = e4 * 4u < len;
+                const float nan = __int_as_float(0x7fc00000);  // fails every compare
+                const float4 v = ok ? src[e4] : make_float4(nan, nan, nan, nan);
+                x[4 * u + 0] = v.x;
+                x[4 * u + 1] = v.y;
+                x[4 * u + 2] = v.z;
+                x[4 * u + 3] = v.w;
+                if (fast) {
+                    mask |= ((uint32_t)(v.x <= tv) | ((uint32_t)(v.y <= tv) << 1) | ((uint32_t)(v.z <= tv) << 2) |
+                             ((uint32_t)(v.w <= tv) << 3)) << (4 * u);
+                } else {
+                    mask |= ok ? (0xfu << (4 * u)) : 0u;
+                }
+            }
+            if (__any_sync(kFull, mask != 0u)) {
+                uint32_t key[NS], col[NS];
+#pragma unroll
+                for (int j = 0; j < NS; ++j) {
+                    key[j] = key_of(x[j]);
+                    col[j] = col0 + ((uint32_t)(g + (j >> 2)) * 32u + lane) * 4u + (uint32_t)(j & 3);
+                }
+                absorb(mask, key, col);
+            }
+        }
+        __syncwarp();
+        if (lane == 0 && li + S < nmine) issue(li + S);
+    }
+
+    // ---- finish: exact top-k of this warp's share, sorted -----------------------------------
+    if (n > k) {
+        const unsigned long long t = pool_kth(pk, pi, n, (uint32_t)k, hist);
+        n = pool_compact(pk, pi, n, (uint32_t)(t >> 32), (uint32_t)t);
+    }
+    pool_sort<R>(pk, pi, n);
+
+    if (WPR > 1) {
+#pragma unroll 1
+        for (int step = 1; step < WPR; step <<= 1) {
+            pool_group_bar(1 + grp, 32 * WPR);
+            if ((wig & (2 * step - 1)) == 0) {
+                const uint32_t* ok2 = reinterpret_cast<const uint32_t*>(
+                    smem + RPC * Cfg::kGroupBytes + (warp + step) * Cfg::kWarpStride + Cfg::kRingBytes);
+                pool_merge_sorted<R>(pk, pi, ok2, ok2 + Cfg::kPool);
+            }
+        }
+        if (wig != 0) return;
+    }
+
+    float* ov = out_val + row * (int64_t)k;
+    int32_t* oi = out_idx + row * (int64_t)k;
+    for (int e = (int)lane; e < k; e += 32) {
+        const uint32_t key = pk[e];
+        const uint32_t col = pi[e];
+        const uint32_t bits = key_needs_regather(key) ? __float_as_uint(dist[g0 + col]) : bits_of_key(key);
+        ov[e] = __uint_as_float(bits);
+        oi[e] = (int32_t)col;
+    }
+}
+
+template <int R, int WPR, int RPC>
+static cudaError_t launch_pool_cfg(const float* dist, int64_t Q, int64_t N, int k, float* ov, int32_t* oi,
+                                   cudaStream_t stream) {
+    using Cfg = PoolCfg<R, WPR, RPC>;
+    auto kern = ksel_pool_kernel<R, WPR, RPC>;
+    static bool attr_done = false;
+    if (!attr_done) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::kSmem);
+        if (e != cudaSuccess) return e;
+        attr_done = true;
+    }
+    const int64_t grid = (Q + RPC - 1) / RPC;
+    kern<<<(unsigned)grid, Cfg::kThreads, Cfg::kSmem, stream>>>(dist, Q, N, k, ov, oi);
+    note_launch();
+    return cudaGetLastError();
+}
+
+// Largest configuration <= (WPR, RPC) whose shared memory fits one SM (227 KB):
+// large queues with many warps per row fall back to fewer warps per CTA.
+template <int R, int WPR, int RPC>
+static cudaError_t launch_pool_fit(const float* dist, int64_t Q, int64_t N, int k, float* ov, int32_t* oi,
+                                   cudaStream_t stream) {
+    if constexpr (PoolCfg<R, WPR, RPC>::kSmem > kMaxSmemPerBlock) {
+        if constexpr (RPC > 1) return launch_pool_fit<R, WPR, RPC / 2>(dist, Q, N, k, ov, oi, stream);
+        else return launch_pool_fit<R, WPR / 2, 1>(dist, Q, N, k, ov, oi, stream);
+    } else {
+        return launch_pool_cfg<R, WPR, RPC>(dist, Q, N, k, ov, oi, stream);
+    }
+}
+
+template <int R>
+cudaError_t launch_pool_r(const float* dist, int64_t Q, int64_t N, int k, float* ov, int32_t* oi, int wpr,
+                          cudaStream_t stream) {
+    switch (wpr) {
+        case 1: return launch_pool_fit<R, 1, 4>(dist, Q, N, k, ov, oi, stream);
+        case 2: return launch_pool_fit<R, 2, 2>(dist, Q, N, k, ov, oi, stream);
+        case 4: return launch_pool_fit<R, 4, 1>(dist, Q, N, k, ov, oi, stream);
+        default: return launch_pool_fit<R, 8, 1>(dist, Q, N, k, ov, oi, stream);
+    }
+}
+
+// One object per queue size R (build.py compiles this file with -DKSEL_ONLY_R=R).
+template cudaError_t launch_pool_r<KSEL_ONLY_R>(const float*, int64_t, int64_t, int, float*, int32_t*, int,
+                                                cudaStream_t);
+
+}  // namespace ksel

@@ -1,0 +1,209 @@
+"""GPU parity of ksel_select / ksel_merge / ksel_select_host against the oracle.
+
+Every comparison is BIT-EXACT: values compared as uint32 bit patterns and
+indices as int32 (north star: "ksel_select must be bit-exact in values and
+indices on identical generated inputs").  Inputs come from synth/ (the same
+bits on both sides); no expected value is produced by the CUDA path.
+"""
+import numpy as np
+import pytest
+import torch
+
+import synth
+
+pytestmark = pytest.mark.gpu
+
+KS = [1, 2, 3, 8, 31, 32, 33, 100, 128, 255, 256, 257, 512, 1000, 1024]
+
+
+@pytest.fixture(scope="module")
+def K():
+    import paper_conf_ipps_tang0emg15_b200 as k
+    assert torch.cuda.is_available(), "GPU test run without a GPU"
+    return k
+
+
+def _bits(a):
+    return np.ascontiguousarray(a, dtype=np.float32).view(np.uint32)
+
+
+def assert_same(ev, ei, gv, gi, ctx=""):
+    gv = gv.cpu().numpy() if torch.is_tensor(gv) else gv
+    gi = gi.cpu().numpy() if torch.is_tensor(gi) else gi
+    bad_i = np.nonzero((gi != ei).any(axis=1) | (_bits(gv) != _bits(ev)).any(axis=1))[0]
+    if bad_i.size:
+        r = bad_i[0]
+        j = np.nonzero((gi[r] != ei[r]) | (_bits(gv[r]) != _bits(ev[r])))[0][0]
+        raise AssertionError("%s: %d bad rows; row %d first diff at %d: gpu (%r,%d) oracle (%r,%d)"
+                             % (ctx, bad_i.size, r, j, gv[r][j], gi[r][j], ev[r][j], ei[r][j]))
+
+
+def _check_select(K, oracle_mod, x_cpu, k, ctx, algo=0, wpr=0):
+    x = x_cpu.cuda()
+    gv, gi = K.ksel_select(x, k, algo=algo, warps_per_row=wpr)
+    torch.cuda.synchronize()
+    ev, ei = oracle_mod.select(x_cpu.numpy(), k)
+    assert_same(ev, ei, gv, gi, ctx)
+
+
+def test_config1(K, oracle_mod):
+    # configs[0]: Q=16 rows, N=4096 uniform fp32 distances, k=32
+    x = synth.rows("U", synth.seed_for(1, "U"), 0, 16, 4096)
+    _check_select(K, oracle_mod, x, 32, "C1")
+
+
+@pytest.mark.parametrize("algo", [1, 2])
+@pytest.mark.parametrize("dist", synth.DISTS)
+def test_k_sweep_all_distributions(K, oracle_mod, dist, algo):
+    # both kernel variants: 1 = bitonic queue per flush, 2 = pool + radix narrowing
+    x = synth.rows(dist, synth.seed_for(7, dist), 0, 48, 5003)  # ragged N (N % 4 != 0)
+    for k in KS:
+        _check_select(K, oracle_mod, x, k, "%s k=%d algo=%d" % (dist, k, algo), algo=algo)
+
+
+@pytest.mark.parametrize("N", [1, 2, 3, 5, 31, 1000, 1023, 1024, 1025, 4095, 4096, 9999, 65536])
+def test_edge_lengths(K, oracle_mod, N):
+    for dist in ("U", "T", "X"):
+        x = synth.rows(dist, 99, 0, 9, N)
+        for k in sorted({1, min(N, 2), min(N, 3), min(N, 32), min(N, 33), min(N, 257), min(N, 1024), min(N, 1024)}):
+            _check_select(K, oracle_mod, x, k, "%s N=%d k=%d" % (dist, N, k))
+
+
+@pytest.mark.parametrize("Q", [1, 2, 5, 16, 150, 600, 2000])
+def test_row_counts_and_warps_per_row(K, oracle_mod, Q):
+    # small Q selects several warps per row (shared threshold + in-CTA merge)
+    x = synth.rows("G", 31, 0, Q, 40000)
+    for k in (1, 32, 100, 256, 1024):
+        _check_select(K, oracle_mod, x, k, "Q=%d k=%d" % (Q, k))
+
+
+@pytest.mark.parametrize("algo", [1, 2])
+@pytest.mark.parametrize("wpr", [1, 2, 4, 8])
+def test_forced_warps_per_row(K, oracle_mod, wpr, algo):
+    for dist in ("U", "SD", "T", "X"):
+        x = synth.rows(dist, 41, 0, 13, 30011)
+        for k in (1, 33, 256, 1000):
+            _check_select(K, oracle_mod, x, k, "%s wpr=%d algo=%d k=%d" % (dist, wpr, algo, k), algo, wpr)
+
+
+def test_unaligned_base_pointer(K, oracle_mod):
+    # row starts that are not 16-byte aligned, including the base pointer itself
+    big = synth.rows("U", 5, 0, 1, 7 * 4099 + 3)[0]
+    for off in (1, 2, 3):
+        x_cpu = big[off:off + 7 * 4099].reshape(7, 4099).contiguous()
+        xg = big.cuda()[off:off + 7 * 4099].view(7, 4099)
+        assert xg.data_ptr() % 16 != 0
+        for k in (1, 64, 300):
+            gv, gi = K.ksel_select(xg, k)
+            ev, ei = oracle_mod.select(x_cpu.numpy(), k)
+            assert_same(ev, ei, gv, gi, "off=%d k=%d" % (off, k))
+
+
+def test_special_rows(K, oracle_mod):
+    N = 3000
+    rows = [np.full(N, 0.25, np.float32), np.arange(N, dtype=np.float32),
+            np.arange(N, dtype=np.float32)[::-1].copy(),
+            np.where(np.arange(N) % 2 == 0, -0.0, 0.0).astype(np.float32),
+            np.full(N, np.nan, np.float32), np.full(N, np.inf, np.float32),
+            np.concatenate([np.full(N - 5, np.nan), [np.inf, -np.inf, 1e-45, -1e-45, -0.0]]).astype(np.float32)]
+    x = torch.from_numpy(np.stack(rows))
+    for k in (1, 5, 6, 32, 100, 1024):
+        _check_select(K, oracle_mod, x, k, "special k=%d" % k)
+
+
+@pytest.mark.parametrize("k", [1, 8, 32, 128, 256, 1024])
+@pytest.mark.parametrize("dist", ["U", "G", "SA", "SD", "T"])
+def test_config2_full_size(K, oracle_mod, dist, k):
+    # configs[1]: Q=1024, N=65536, the k sweep, all distributions -- all rows
+    x = synth.rows(dist, synth.seed_for(2, dist), 0, 1024, 65536, device="cuda")
+    gv, gi = K.ksel_select(x, k)
+    torch.cuda.synchronize()
+    ev, ei = oracle_mod.select(x.cpu().numpy(), k)
+    assert_same(ev, ei, gv, gi, "C2 %s k=%d" % (dist, k))
+
+
+@pytest.mark.slow
+def test_config3_full_size_sampled_rows(K, oracle_mod):
+    # configs[2] at one GPU, exactly the launch bench.py times: Q=16384, N=2^20,
+    # k=256; the oracle checks a fixed sample (first 32 rows of each 2048 block)
+    Q, N, k = 16384, 1 << 20, 256
+    seed = synth.seed_for(3, "U")
+    x = synth.rows("U", seed, 0, Q, N, device="cuda")
+    gv, gi = K.ksel_select(x, k)
+    torch.cuda.synchronize()
+    sample = [b * 2048 + t for b in range(Q // 2048) for t in range(32)]
+    del x
+    xs = synth.row_subset("U", seed, sample, N)
+    ev, ei = oracle_mod.select(xs.numpy(), k)
+    assert_same(ev, ei, gv[sample].cpu().numpy(), gi[sample].cpu().numpy(), "C3 sample")
+
+
+# ---- ksel_merge -----------------------------------------------------------
+
+@pytest.mark.parametrize("S", [1, 2, 3, 8])
+@pytest.mark.parametrize("dist", ["U", "T", "X"])
+def test_sharded_select_then_merge_equals_full(K, oracle_mod, S, dist):
+    # the row-sharded path on one GPU: per-shard ksel_select with global
+    # indices, concatenate like an all-gather, ksel_merge == unsharded result
+    Q, N = 64, 12000
+    x = synth.rows(dist, 77, 0, Q, N)
+    xg = x.cuda()
+    bounds = np.linspace(0, N, S + 1).astype(int)
+    for k in (1, 32, 100, 256, 1000):
+        if any(bounds[s + 1] - bounds[s] < k for s in range(S)):
+            continue
+        vals, idxs = [], []
+        for s in range(S):
+            v, i = K.ksel_select(xg[:, bounds[s]:bounds[s + 1]].contiguous(), k)
+            vals.append(v)
+            idxs.append(i + int(bounds[s]))
+        mv, mi = K.ksel_merge(torch.stack(vals).contiguous(), torch.stack(idxs).contiguous(), k)
+        ev, ei = oracle_mod.select(x.numpy(), k)
+        assert_same(ev, ei, mv, mi, "merge S=%d %s k=%d" % (S, dist, k))
+
+
+def test_merge_vs_oracle_merge_unsorted_and_long_lists(K, oracle_mod):
+    rng = np.random.default_rng(5)
+    for (S, Q, kin, k) in [(2, 33, 4, 8), (4, 100, 100, 100), (3, 7, 1024, 64), (8, 50, 300, 1024), (5, 9, 37, 3)]:
+        v = rng.integers(0, 50, size=(S, Q, kin)).astype(np.float32)
+        i = rng.permutation(S * Q * kin).astype(np.int32).reshape(S, Q, kin)
+        # sorted lists (the contract) ...
+        order = np.lexsort((i, v), axis=-1)
+        vs = np.take_along_axis(v, order, -1)
+        is_ = np.take_along_axis(i, order, -1)
+        ev, ei = oracle_mod.merge(vs, is_, k)
+        gv, gi = K.ksel_merge(torch.from_numpy(vs).cuda(), torch.from_numpy(is_).cuda(), k)
+        assert_same(ev, ei, gv, gi, "merge sorted %r" % ((S, Q, kin, k),))
+        # ... and unsorted lists are handled exactly too
+        ev, ei = oracle_mod.merge(v, i, k)
+        gv, gi = K.ksel_merge(torch.from_numpy(v).cuda(), torch.from_numpy(i).cuda(), k)
+        assert_same(ev, ei, gv, gi, "merge unsorted %r" % ((S, Q, kin, k),))
+
+
+def test_merge_keeps_special_bits(K, oracle_mod):
+    v = np.array([[[-0.0, 1.0, np.nan]], [[0.0, 2.0, float.fromhex("0x1.8p+0")]]], np.float32)
+    v[0, 0, 2] = np.frombuffer(np.uint32(0x7fc00123).tobytes(), np.float32)[0]
+    i = np.array([[[3, 4, 5]], [[1, 6, 7]]], np.int32)
+    order = np.lexsort((i, v), axis=-1)
+    vs, is_ = np.take_along_axis(v, order, -1), np.take_along_axis(i, order, -1)
+    ev, ei = oracle_mod.merge(vs, is_, 6)
+    gv, gi = K.ksel_merge(torch.from_numpy(vs).cuda(), torch.from_numpy(is_).cuda(), 6)
+    assert_same(ev, ei, gv, gi, "merge special")
+
+
+# ---- host (end-to-end) entry point ------------------------------------------
+
+def test_select_host_pipeline(K, oracle_mod):
+    Q, N, k = 300, 70000, 100
+    x = synth.rows("DG", 55, 0, Q, N).pin_memory()
+    ws = torch.empty(K.ksel_select_host_workspace(N, k) // 8, dtype=torch.uint8, device="cuda")  # force many blocks
+    gv, gi = K.ksel_select_host(x, k, workspace=ws)
+    ev, ei = oracle_mod.select(x.numpy(), k)
+    assert_same(ev, ei, gv.numpy(), gi.numpy(), "host pipeline")
+
+
+def test_launch_count_increments(K):
+    x = torch.rand(4, 100, device="cuda")
+    c0 = K.launch_count()
+    K.ksel_select(x, 3)
+    assert K.launch_count() == c0 + 1
