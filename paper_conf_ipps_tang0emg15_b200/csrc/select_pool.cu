@@ -36,10 +36,10 @@ namespace ksel {
 template <int R, int WPR, int RPC>
 struct PoolCfg {
     static constexpr int kQueue = 32 * R;  // k'
-    static constexpr int kPool = (2 * kQueue > kQueue + 256) ? 2 * kQueue : kQueue + 256;
-    static constexpr int CH = 1024;        // floats per staged chunk
-    static constexpr int S = 3;            // ring stages per warp
-    static constexpr int G = 2;            // float4 per lane per sub-step (256 elements per warp)
+    static constexpr int kPool = (2 * kQueue > kQueue + 512) ? 2 * kQueue : kQueue + 512;
+    static constexpr int CH = 512;         // floats per staged chunk (2 KB bulk copy)
+    static constexpr int S = 4;            // ring stages per warp
+    static constexpr int G = 4;            // float4 per lane per sub-step (512 elements per warp)
     static constexpr int NS = 4 * G;       // element slots per lane per sub-step
     static constexpr int kWarps = WPR * RPC;
     static constexpr int kThreads = 32 * kWarps;
@@ -312,48 +312,64 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC>::kThreads)
         tighten(kk, ki);
         if (WPR > 1 && lane == 0) atomicMin(grp_thr, t);
     };
-    // append the candidates flagged in `mask` (slot j: key[j], col[j]) after the exact test
-    auto absorb = [&](uint32_t mask, const auto& key, const auto& col) {
-        constexpr int ns = (int)(sizeof(key) / sizeof(key[0]));
+    // Exact path of one sub-step: the elements of this lane are the 4*G floats at
+    // e(j) = ((g + j/4)*32 + lane)*4 + j%4 of the staged chunk `srcf` (x[j] in
+    // registers).  Pre-filter again per element, run the exact lexicographic
+    // test only on the flagged ones (re-read from shared memory), then append
+    // the admitted pairs to the pool at warp-scanned positions.
+    auto exact = [&](const float* srcf, uint32_t g, uint32_t len, uint32_t col0, const float(&x)[NS]) {
         uint32_t m = 0;
 #pragma unroll
-        for (int j = 0; j < ns; ++j)
-            if (((mask >> j) & 1u) && pair_lt(key[j], col[j], Tk, Ti)) m |= 1u << j;
+        for (int j = 0; j < NS; ++j) {
+            const uint32_t e = ((g + (uint32_t)(j >> 2)) * 32u + lane) * 4u + (uint32_t)(j & 3);
+            const bool cand = (e < len) && (!fast || x[j] <= tv);
+            m |= (uint32_t)cand << j;
+        }
+        auto elem = [&](int j) { return ((g + (uint32_t)(j >> 2)) * 32u + lane) * 4u + (uint32_t)(j & 3); };
+        auto refine = [&](uint32_t mm) {
+            uint32_t adm = 0;
+            for (uint32_t t = mm; t; t &= t - 1u) {
+                const int j = __ffs(t) - 1;
+                const uint32_t e = elem(j);
+                if (pair_lt(key_of(srcf[e]), col0 + e, Tk, Ti)) adm |= 1u << j;
+            }
+            return adm;
+        };
+        uint32_t adm = refine(m);
         uint32_t total;
-        uint32_t excl = warp_excl_scan(__popc(m), lane, total);
+        uint32_t excl = warp_excl_scan(__popc(adm), lane, total);
         if (total == 0) return;
         if (n + (int)total > Cfg::kPool) {
             narrow();
-            uint32_t m2 = 0;
-#pragma unroll
-            for (int j = 0; j < ns; ++j)
-                if (((m >> j) & 1u) && pair_lt(key[j], col[j], Tk, Ti)) m2 |= 1u << j;
-            m = m2;
-            excl = warp_excl_scan(__popc(m), lane, total);
+            adm = refine(adm);
+            excl = warp_excl_scan(__popc(adm), lane, total);
         }
         int pos = n + (int)excl;
-#pragma unroll
-        for (int j = 0; j < ns; ++j)
-            if ((m >> j) & 1u) {
-                pk[pos] = key[j];
-                pi[pos] = col[j];
-                ++pos;
-            }
+        for (uint32_t t = adm; t; t &= t - 1u) {
+            const uint32_t e = elem(__ffs(t) - 1);
+            pk[pos] = key_of(srcf[e]);
+            pi[pos] = col0 + e;
+            ++pos;
+        }
         n += (int)total;
         __syncwarp();
     };
 
-    // ---- unaligned head and tail ---------------------------------------------------------
+    // ---- unaligned head and tail (< 4 elements each; pool is empty, cannot overflow) ---------
     if (wig == 0) {
         const uint32_t nh = (uint32_t)(a0 - g0), nt = (uint32_t)(g1 - a1);
         bool valid = false;
         uint64_t g = 0;
         if (lane < nh) { valid = true; g = g0 + lane; }
         else if (lane < nh + nt) { valid = true; g = a1 + (lane - nh); }
-        uint32_t key[1], col[1];
-        key[0] = valid ? key_of(dist[g]) : kSentKey;
-        col[0] = (uint32_t)(g - g0);
-        absorb(valid ? 1u : 0u, key, col);
+        const uint32_t bal = __ballot_sync(kFull, valid);
+        if (valid) {
+            const int pos = n + __popc(bal & lanemask_lt());
+            pk[pos] = key_of(dist[g]);
+            pi[pos] = (uint32_t)(g - g0);
+        }
+        n += __popc(bal);
+        __syncwarp();
     }
 
     // ---- streaming body ------------------------------------------------------------------
@@ -367,37 +383,30 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC>::kThreads)
             tighten((uint32_t)(sh >> 32), (uint32_t)sh);
         }
         mbar_wait(&mbar[st], (uint32_t)(li / S) & 1u);
-        const float4* src = reinterpret_cast<const float4*>(ring + st * CH);
+        const float* srcf = ring + st * CH;
+        const float4* src = reinterpret_cast<const float4*>(srcf);
 #pragma unroll 1
         for (int g = 0; g < CH / 128; g += G) {
             float x[NS];
-            uint32_t mask = 0;
+            const float inf = __int_as_float(0x7f800000);  // never passes x <= tv in fast mode
 #pragma unroll
             for (int u = 0; u < G; ++u) {
                 const uint32_t e4 = (uint32_t)(g + u) * 32u + lane;
-                const bool ok = e4 * 4u < len;
-                const float nan = __int_as_float(0x7fc00000);  // fails every compare
-                const float4 v = ok ? src[e4] : make_float4(nan, nan, nan, nan);
+                const float4 v = (len == (uint32_t)CH || e4 * 4u < len) ? src[e4] : make_float4(inf, inf, inf, inf);
                 x[4 * u + 0] = v.x;
                 x[4 * u + 1] = v.y;
                 x[4 * u + 2] = v.z;
                 x[4 * u + 3] = v.w;
-                if (fast) {
-                    mask |= ((uint32_t)(v.x <= tv) | ((uint32_t)(v.y <= tv) << 1) | ((uint32_t)(v.z <= tv) << 2) |
-                             ((uint32_t)(v.w <= tv) << 3)) << (4 * u);
-                } else {
-                    mask |= ok ? (0xfu << (4 * u)) : 0u;
-                }
             }
-            if (__any_sync(kFull, mask != 0u)) {
-                uint32_t key[NS], col[NS];
+            bool go = true;
+            if (fast) {
+                // one compare per lane: the sub-step minimum (fminf skips NaN, which is never a candidate)
+                float mn = x[0];
 #pragma unroll
-                for (int j = 0; j < NS; ++j) {
-                    key[j] = key_of(x[j]);
-                    col[j] = col0 + ((uint32_t)(g + (j >> 2)) * 32u + lane) * 4u + (uint32_t)(j & 3);
-                }
-                absorb(mask, key, col);
+                for (int j = 1; j < NS; ++j) mn = fminf(mn, x[j]);
+                go = __any_sync(kFull, mn <= tv);
             }
+            if (go) exact(srcf, (uint32_t)g, len, col0, x);
         }
         __syncwarp();
         if (lane == 0 && li + S < nmine) issue(li + S);
@@ -468,7 +477,7 @@ template <int R>
 cudaError_t launch_pool_r(const float* dist, int64_t Q, int64_t N, int k, float* ov, int32_t* oi, int wpr,
                           cudaStream_t stream) {
     switch (wpr) {
-        case 1: return launch_pool_fit<R, 1, 4>(dist, Q, N, k, ov, oi, stream);
+        case 1: return launch_pool_fit<R, 1, 1>(dist, Q, N, k, ov, oi, stream);
         case 2: return launch_pool_fit<R, 2, 2>(dist, Q, N, k, ov, oi, stream);
         case 4: return launch_pool_fit<R, 4, 1>(dist, Q, N, k, ov, oi, stream);
         default: return launch_pool_fit<R, 8, 1>(dist, Q, N, k, ov, oi, stream);
