@@ -5,6 +5,7 @@
 // device paths, no stream synchronisation except in ksel_select_host.
 #include <atomic>
 #include <cstdint>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 
@@ -17,6 +18,14 @@ namespace ksel {
 
 static std::atomic<int64_t> g_launches{0};
 void note_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+
+int chunk_order_mode() {
+    static const int mode = [] {
+        const char* e = std::getenv("KSEL_ORDER");
+        return (e && (e[0] == '0' || e[0] == '1' || e[0] == '2')) ? e[0] - '0' : 2;
+    }();
+    return mode;
+}
 
 struct DevInfo {
     int sms = 0;

@@ -8,6 +8,10 @@ namespace ksel {
 
 constexpr int kMaxSmemPerBlock = 227 * 1024;  // sm_100 opt-in dynamic shared memory per CTA
 
+// Chunk visit order of the streaming kernels (experiments only; env KSEL_ORDER):
+// 0 = address order, 1 = spread prologue + address order, 2 = strided permutation (default).
+int chunk_order_mode();
+
 // Count one enqueued kernel (reported through ksel_launch_count()).
 void note_launch();
 

@@ -44,8 +44,8 @@ struct PoolCfg {
     static constexpr int kWarps = WPR * RPC;
     static constexpr int kThreads = 32 * kWarps;
     static constexpr int kRingBytes = S * CH * 4;
-    // per warp: ring | pool keys | pool idx | histogram (256 u32) | mbarriers
-    static constexpr int kWarpBytes = kRingBytes + kPool * 8 + 256 * 4 + S * 8;
+    // per warp: ring | pool keys | pool idx | histogram (256 u32) | mbarriers | stage chunk ids
+    static constexpr int kWarpBytes = kRingBytes + kPool * 8 + 256 * 4 + S * 8 + S * 4;
     static constexpr int kWarpStride = (kWarpBytes + 127) / 128 * 128;
     static constexpr int kGroupBytes = 128;
     static constexpr int kSmem = RPC * kGroupBytes + kWarps * kWarpStride;
@@ -239,7 +239,7 @@ __device__ __noinline__ void pool_merge_sorted(uint32_t* __restrict__ qk, uint32
 template <int R, int WPR, int RPC>
 __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC>::kThreads)
     ksel_pool_kernel(const float* __restrict__ dist, int64_t Q, int64_t N, int k, float* __restrict__ out_val,
-                     int32_t* __restrict__ out_idx) {
+                     int32_t* __restrict__ out_idx, int order_mode) {
     using Cfg = PoolCfg<R, WPR, RPC>;
     constexpr int CH = Cfg::CH, S = Cfg::S, G = Cfg::G, NS = Cfg::NS;
     extern __shared__ __align__(128) uint8_t smem[];
@@ -258,6 +258,7 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC>::kThreads)
     uint32_t* pi = pk + Cfg::kPool;
     uint32_t* hist = pi + Cfg::kPool;
     uint64_t* mbar = reinterpret_cast<uint64_t*>(hist + 256);
+    uint32_t* cid = reinterpret_cast<uint32_t*>(mbar + S);  // chunk id of each stage
 
     // ---- row geometry -----------------------------------------------------------
     const uint64_t g0 = (uint64_t)row * (uint64_t)N;
@@ -271,14 +272,49 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC>::kThreads)
     const uint64_t c_end = nch * (wig + 1) / WPR;
     const int nmine = (int)(c_end - c_begin);
 
+    // Visit order: first a "spread prologue" of NP chunks evenly spaced over the
+    // warp's range (c = i * step), then every other chunk in address order.  The
+    // prologue gives the running threshold a representative sample of the whole
+    // range early, so sorted or trending rows (which an in-order scan would
+    // admit entirely, e.g. descending rows) are filtered like random ones, while
+    // the bulk of the traffic stays sequential for DRAM locality.  The result
+    // does not depend on the order.  Only the issuing lane walks the order
+    // (incrementally, no divisions); the chunk id travels with the stage.
+    const uint32_t nm = (uint32_t)nmine;
+    uint32_t np = (nm >= 64u) ? 16u : nm / 4u;
+    if (order_mode == 0) np = 0;
+    const uint32_t step = np ? nm / np : 1u;
+    uint32_t pstride = 1;
+    if (order_mode == 2 && nm > 2u && lane == 0) {
+        pstride = ((uint32_t)((double)nm * 0.6180339887498949)) | 1u;
+        auto gcd = [](uint32_t a, uint32_t b) { while (b) { const uint32_t t = a % b; a = b; b = t; } return a; };
+        while (gcd(pstride, nm) != 1u) pstride += 2;
+    }
+    uint32_t it_i = 0, it_blk = 0, it_off = 1, it_tail = np * step, it_p = 0;
+    auto next_chunk = [&]() -> uint32_t {  // lane 0 only; chunk index relative to c_begin
+        if (order_mode == 2) {
+            const uint32_t c = it_p;
+            it_p += pstride;
+            if (it_p >= nm) it_p -= nm;
+            return c;
+        }
+        if (it_i < np) return (it_i++) * step;
+        if (it_blk < np) {
+            const uint32_t c = it_blk * step + it_off;
+            if (++it_off == step) { it_off = 1; ++it_blk; }
+            return c;
+        }
+        return it_tail++;
+    };
     auto chunk_len = [&](uint64_t c) -> uint32_t {
         const uint64_t s0 = a0 + c * CH;
         const uint64_t s1 = (s0 + CH < a1) ? s0 + CH : a1;
         return (uint32_t)(s1 - s0);
     };
     auto issue = [&](int li) {
-        const uint64_t c = c_begin + li;
+        const uint64_t c = c_begin + next_chunk();
         const int st = li % S;
+        cid[st] = (uint32_t)c;
         const uint32_t bytes = chunk_len(c) * 4u;
         mbar_arrive_expect_tx(&mbar[st], bytes);
         bulk_g2s(ring + st * CH, dist + a0 + c * CH, bytes, &mbar[st]);
@@ -319,11 +355,14 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC>::kThreads)
     // the admitted pairs to the pool at warp-scanned positions.
     auto exact = [&](const float* srcf, uint32_t g, uint32_t len, uint32_t col0, const float(&x)[NS]) {
         uint32_t m = 0;
+        if (fast) {
+            // invalid slots of a partial chunk hold +Inf and never pass
 #pragma unroll
-        for (int j = 0; j < NS; ++j) {
-            const uint32_t e = ((g + (uint32_t)(j >> 2)) * 32u + lane) * 4u + (uint32_t)(j & 3);
-            const bool cand = (e < len) && (!fast || x[j] <= tv);
-            m |= (uint32_t)cand << j;
+            for (int j = 0; j < NS; ++j) m |= (uint32_t)(x[j] <= tv) << j;
+        } else {
+#pragma unroll
+            for (int u = 0; u < G; ++u)
+                if (((g + (uint32_t)u) * 32u + lane) * 4u < len) m |= 0xfu << (4 * u);
         }
         auto elem = [&](int j) { return ((g + (uint32_t)(j >> 2)) * 32u + lane) * 4u + (uint32_t)(j & 3); };
         auto refine = [&](uint32_t mm) {
@@ -375,14 +414,14 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC>::kThreads)
     // ---- streaming body ------------------------------------------------------------------
     for (int li = 0; li < nmine; ++li) {
         const int st = li % S;
-        const uint64_t c = c_begin + li;
-        const uint32_t len = chunk_len(c);
-        const uint32_t col0 = (uint32_t)(a0 + c * CH - g0);
         if (WPR > 1) {
             const unsigned long long sh = *reinterpret_cast<volatile unsigned long long*>(grp_thr);
             tighten((uint32_t)(sh >> 32), (uint32_t)sh);
         }
         mbar_wait(&mbar[st], (uint32_t)(li / S) & 1u);
+        const uint64_t c = cid[st];
+        const uint32_t len = chunk_len(c);
+        const uint32_t col0 = (uint32_t)(a0 + c * CH - g0);
         const float* srcf = ring + st * CH;
         const float4* src = reinterpret_cast<const float4*>(srcf);
 #pragma unroll 1
@@ -455,7 +494,7 @@ static cudaError_t launch_pool_cfg(const float* dist, int64_t Q, int64_t N, int 
         attr_done = true;
     }
     const int64_t grid = (Q + RPC - 1) / RPC;
-    kern<<<(unsigned)grid, Cfg::kThreads, Cfg::kSmem, stream>>>(dist, Q, N, k, ov, oi);
+    kern<<<(unsigned)grid, Cfg::kThreads, Cfg::kSmem, stream>>>(dist, Q, N, k, ov, oi, chunk_order_mode());
     note_launch();
     return cudaGetLastError();
 }
