@@ -136,11 +136,14 @@ def cpu_count():
         return os.cpu_count() or 1
 
 
-def oracle_rows_per_s(dist: str, seed: int, N: int, k: int, rows: list, threads: int):
-    """Time the oracle (as it stands) on a bounded sample of rows; returns rows/s."""
+def oracle_rows_per_s(dist: str, seed: int, N: int, k: int, rows: list, threads: int, device="cpu"):
+    """Time the oracle (as it stands) on a bounded sample of rows; returns rows/s.
+
+    The sample rows are generated (bit-identically) on `device` and copied to
+    the host; only the oracle call is timed."""
     import oracle
     import synth
-    x = synth.row_subset(dist, seed, rows, N).numpy()
+    x = synth.row_subset(dist, seed, rows, N, device=device).cpu().numpy()
     oracle.build()
     t0 = time.perf_counter()
     oracle.select(x, k, nthreads=threads)
@@ -279,7 +282,7 @@ def main():
             "hbm_gbs": achieved,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
-                         "kernel": "ksel_stream_kernel",
+                         "kernel": "ksel_pool_kernel",
                          "bytes_per_launch": alg_bytes, "bytes_formula": "Q*(4N+8k)"},
             "gpu_launches": launches,
             "clocks": clocks,
@@ -310,10 +313,11 @@ def main():
     # ---- CPU baseline: the oracle on this host's cores (rank 0, N=1 only) --------
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         threads = cpu_count()
-        nrows = args.cpu_sample_rows or min(256, max(16, 4 * threads))
-        sample = [(b * 2048 + t) % Qr for b in range(max(1, Qr // 2048)) for t in range(2048)][:nrows]
-        sample = sorted(set(sample))
-        rps, dt = oracle_rows_per_s(dist, seed, N, k, [row0 + r for r in sample], threads)
+        # ~10-30 s of CPU work: 64 rows per host thread (first rows of each 2048-row block)
+        nrows = args.cpu_sample_rows or min(Qr, 64 * threads)
+        per_blk = max(1, nrows // max(1, Qr // 2048))
+        sample = sorted({(b * 2048 + t) % Qr for b in range(max(1, Qr // 2048)) for t in range(per_blk)})[:nrows]
+        rps, dt = oracle_rows_per_s(dist, seed, N, k, [row0 + r for r in sample], threads, device=dev)
         line["cpu_baseline"] = {"value": rps, "unit": "rows/s", "cores": threads, "kind": "oracle",
                                 "sample": "%d rows of the same workload (%.1f s)" % (len(sample), dt)}
 

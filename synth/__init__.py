@@ -113,8 +113,10 @@ def row_subset(dist: str, seed: int, row_ids, N: int, device="cpu") -> torch.Ten
     """Arbitrary (sampled) global rows, bit-identical to those in rows()."""
     ids = torch.as_tensor(list(row_ids), dtype=torch.int64)
     out = torch.empty((len(ids), N), dtype=torch.float32, device=device)
-    for t, r in enumerate(ids.tolist()):
-        out[t:t + 1] = _gen_block(dist, seed, torch.tensor([[r]], device=device), N, device)
+    step = max(1, _CHUNK // max(N, 1))
+    for a in range(0, len(ids), step):
+        r = ids[a:a + step].to(device).unsqueeze(1)
+        out[a:a + len(r)] = _gen_block(dist, seed, r, N, device)
     return out
 
 

@@ -207,3 +207,15 @@ def test_launch_count_increments(K):
     c0 = K.launch_count()
     K.ksel_select(x, 3)
     assert K.launch_count() == c0 + 1
+
+
+@pytest.mark.parametrize("dist", synth.DISTS)
+def test_synth_same_bits_on_gpu_and_cpu(dist):
+    # the oracle may regenerate rows on the host: the generator must be device-independent
+    a = synth.rows(dist, 123, 5000, 6, 7777, device="cuda").cpu()
+    b = synth.rows(dist, 123, 5000, 6, 7777)
+    assert torch.equal(a.view(torch.int32), b.view(torch.int32))
+    for kind in ("knn-U", "knn-S"):
+        p = synth.knn_points(kind, 9, 100, 50, 128, device="cuda").cpu()
+        q = synth.knn_points(kind, 9, 100, 50, 128)
+        assert torch.equal(p.view(torch.int32), q.view(torch.int32))
