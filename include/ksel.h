@@ -111,8 +111,8 @@ KSEL_API int ksel_merge(const float* cand_val, const int32_t* cand_idx, int64_t 
 
 /* knn_search -- brute-force k-NN: distance phase (Sec. II.A,
  * "the method of [3]" L243) fused with k-selection.
- *   ref   [N][D] fp32, query [Q][D] fp32, device, 16-byte aligned.
- *   1 <= D <= 1024, D % 4 == 0; 1 <= k <= min(N, KSEL_MAX_K);
+ *   ref   [N][D] fp32, query [Q][D] fp32, device, 4-byte aligned, row-major.
+ *   1 <= D <= 256 (D > 256 -> KSEL_ERR_UNSUPPORTED); 1 <= k <= min(N, KSEL_MAX_K);
  *   N + idx_offset <= 2^31 - 1, idx_offset >= 0.
  *   out_dist [Q][k] fp32: squared L2 distance (no sqrt), clamped at >= 0,
  *            computed as |q|^2 + |r|^2 - 2 q.r with fp32 accumulation (error
@@ -126,6 +126,15 @@ KSEL_API size_t knn_search_workspace(int64_t N, int64_t Q, int D, int k);
 KSEL_API int knn_search(const float* ref, const float* query, int64_t N, int64_t Q, int D, int k,
                float* out_dist, int32_t* out_idx, int64_t idx_offset, void* d_work,
                size_t work_bytes, void* stream);
+
+/* knn_distances -- DIAGNOSTIC (not the hot path): the same tcgen05 distance
+ * computation as knn_search, but every d(q, r) is written to out[Q][N] (device,
+ * fp32) instead of being selected.  Lets tests pin the tensor-core distance
+ * against the oracle's definition independently of selection.
+ * Workspace from knn_distances_workspace(N, Q, D). */
+KSEL_API size_t knn_distances_workspace(int64_t N, int64_t Q, int D);
+KSEL_API int knn_distances(const float* ref, const float* query, int64_t N, int64_t Q, int D, float* out,
+                           void* d_work, size_t work_bytes, void* stream);
 
 /* Human-readable text for a ksel_status (static storage, never NULL). */
 KSEL_API const char* ksel_strerror(int status);

@@ -38,6 +38,10 @@ _lib.ksel_merge.argtypes = [_p, _p, _i64, _i32, _i32, _i32, _p, _p, _p]
 _lib.knn_search_workspace.argtypes = [_i64, _i64, _i32, _i32]
 _lib.knn_search_workspace.restype = _sz
 _lib.knn_search.argtypes = [_p, _p, _i64, _i64, _i32, _i32, _p, _p, _i64, _p, _sz, _p]
+_lib.knn_distances_workspace.argtypes = [_i64, _i64, _i32]
+_lib.knn_distances_workspace.restype = _sz
+_lib.knn_distances.argtypes = [_p, _p, _i64, _i64, _i32, _p, _p, _sz, _p]
+_lib.knn_distances.restype = ctypes.c_int
 _lib.ksel_strerror.argtypes = [_i32]
 _lib.ksel_strerror.restype = ctypes.c_char_p
 _lib.ksel_launch_count.restype = _i64
@@ -47,7 +51,8 @@ for _f in (_lib.ksel_select, _lib.ksel_select_config, _lib.ksel_select_host, _li
 KSEL_MAX_K = 1024
 ALGO_AUTO, ALGO_QUEUE, ALGO_POOL = 0, 1, 2
 EXPORTS = ("ksel_select", "ksel_select_config", "ksel_select_host_workspace", "ksel_select_host", "ksel_merge",
-           "knn_search_workspace", "knn_search", "ksel_strerror", "ksel_version", "ksel_launch_count")
+           "knn_search_workspace", "knn_search", "knn_distances_workspace", "knn_distances", "ksel_strerror",
+           "ksel_version", "ksel_launch_count")
 
 
 class KselError(RuntimeError):
@@ -183,3 +188,18 @@ def knn_search(ref: torch.Tensor, query: torch.Tensor, k: int, idx_offset: int =
                                              out_dist.data_ptr(), out_idx.data_ptr(), idx_offset,
                                              wptr, wlen, _stream(ref.device)))
     return out_dist, out_idx
+
+
+def knn_distances(ref: torch.Tensor, query: torch.Tensor, out: torch.Tensor | None = None):
+    """DIAGNOSTIC: the tensor-core squared distances [Q, N] (materialised)."""
+    _dev_f32(ref, "ref", 2)
+    _dev_f32(query, "query", 2)
+    N, D = ref.shape
+    Q = query.shape[0]
+    if out is None:
+        out = torch.empty((Q, N), dtype=torch.float32, device=ref.device)
+    ws = torch.empty(max(1, int(_lib.knn_distances_workspace(N, Q, D))), dtype=torch.uint8, device=ref.device)
+    with torch.cuda.device(ref.device):
+        _check("knn_distances", _lib.knn_distances(ref.data_ptr(), query.data_ptr(), N, Q, D, out.data_ptr(),
+                                                   ws.data_ptr(), ws.numel(), _stream(ref.device)))
+    return out

@@ -19,6 +19,26 @@ namespace ksel {
 static std::atomic<int64_t> g_launches{0};
 void note_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
 
+cudaError_t ensure_smem_attr(const void* func, int bytes) {
+    static std::mutex mu;
+    struct Entry {
+        const void* f;
+        int dev;
+        int bytes;
+    };
+    static Entry done[256];
+    static int ndone = 0;
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    std::lock_guard<std::mutex> lock(mu);
+    for (int i = 0; i < ndone; ++i)
+        if (done[i].f == func && done[i].dev == dev && done[i].bytes >= bytes) return cudaSuccess;
+    e = cudaFuncSetAttribute(func, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    if (e == cudaSuccess && ndone < 256) done[ndone++] = Entry{func, dev, bytes};
+    return e;
+}
+
 int chunk_order_mode() {
     static const int mode = [] {
         const char* e = std::getenv("KSEL_ORDER");
@@ -27,23 +47,18 @@ int chunk_order_mode() {
     return mode;
 }
 
-struct DevInfo {
-    int sms = 0;
-    int major = 0;
-    int minor = 0;
-};
-
 static std::mutex g_dev_mu;
 static DevInfo g_dev[64];
 static bool g_dev_ok[64];
 
-static int current_device_info(DevInfo* out) {
+int current_device_info(DevInfo* out) {
     int dev = -1;
     if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return KSEL_ERR_NO_DEVICE;
     std::lock_guard<std::mutex> lock(g_dev_mu);
     if (!g_dev_ok[dev]) {
         cudaDeviceProp p;
         if (cudaGetDeviceProperties(&p, dev) != cudaSuccess) return KSEL_ERR_CUDA;
+        g_dev[dev].dev = dev;
         g_dev[dev].sms = p.multiProcessorCount;
         g_dev[dev].major = p.major;
         g_dev[dev].minor = p.minor;

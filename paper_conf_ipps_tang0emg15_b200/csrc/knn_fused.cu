@@ -1,23 +1,701 @@
 // knn_fused.cu -- knn_search: tcgen05/TMEM distance GEMM fused with k-selection.
-// (placeholder entry points until the fused kernel lands)
+//
+// The k-NN of the paper has two phases (Sec. II.A): Euclidean
+// distances between every query and reference, then k-selection over each
+// query's row of N distances.  The paper computes the Q x N matrix with "the
+// method of [3]" and stores it in global memory (L243); here the matrix never
+// exists.  d(q, r) = |q|^2 + |r|^2 - 2 q.r (reading R9: squared L2), with the dot
+// products on the 5th-gen tensor cores:
+//
+//   * operands split once into bf16 hi/lo pairs (x ~ hi + lo, hi = bf16(x),
+//     lo = bf16(x - hi)); q.r ~ qh.rh + qh.rl + ql.rh -- three kind::f16 MMAs
+//     into one fp32 TMEM accumulator (the dropped ql.rl term is ~2^-16 relative;
+//     SURVEY 7.3 emulation: 8.8e-6 max relative error vs the 1e-4 bar).
+//     Integer data in [0,255] is exact (lo = 0).
+//   * the norms ride in the same accumulation: A holds -2q and one extra
+//     16-wide K block [n1, n2, n3, 1, 1, 1, 0...] with |q|^2 = n1+n2+n3 split
+//     three ways in bf16 (24 significant bits), B holds [1, 1, 1, m1, m2, m3, 0...]
+//     for |r|^2 -- so the accumulator IS d(q, r) and the epilogue touches each
+//     distance once (no per-element norm adds).
+//   * CTA = one tile of 128 queries (TMEM lanes, A operand resident in shared
+//     memory) x a contiguous range of 256-reference tiles (TMEM columns, B
+//     operand streamed by 1-D TMA bulk copies from a pre-tiled image);
+//     warp 0 = producer, warp 1 = TMEM allocator + single-thread MMA issuer,
+//     warps 2-5 = epilogue (one thread per query: the paper's thread-per-query
+//     layout, L243), double-buffered 2 x 256-column accumulators.
+//   * epilogue: tcgen05.ld 32 columns at a time, d = fma(-2, acc, |q|^2+|r|^2),
+//     clamp at 0, and the same pool/threshold selection as select_pool.cu: a
+//     per-query candidate pool (global memory), exact (key, idx) admission test,
+//     warp-cooperative radix narrowing (pool_kth) when a pool fills.
+//   * each CTA leaves the exact top-k of its reference range per query; the
+//     splits are combined by ksel_merge (divide-and-merge, L243).
 #include <cstdint>
+#include <cstdlib>
+#include <cstring>
+
+#include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
 #include "ksel.h"
+#include "ksel_common.cuh"
 #include "ksel_internal.h"
+#include "ksel_pool.cuh"
+
+namespace ksel {
+
+constexpr int KNN_BM = 128;                              // queries per tile (TMEM lanes)
+constexpr int KNN_BN = 256;                              // references per tile (accumulator columns)
+constexpr int KNN_KS = 32;                               // dims per pipeline stage
+constexpr int KNN_STAGE_BYTES = 2 * KNN_KS * KNN_BN * 2;  // hi + lo bf16 = 32 KB
+constexpr int KNN_NORM_B_BYTES = 16 * KNN_BN * 2;         // norm block of a reference tile (hi only)
+constexpr int KNN_NORM_A_BYTES = 16 * KNN_BM * 2;         // norm block of a query tile
+constexpr int KNN_THREADS = 192;                         // 6 warps
+constexpr int KNN_MAX_D = 256;
+constexpr int kNarrowRegs = 40;  // register-resident narrowing: pools of <= 1280 pairs
+constexpr unsigned long long kSentPair = ((unsigned long long)kSentKey << 32) | kSentIdx;
+
+struct KnnGeom {
+    int64_t N, Q;
+    int D, Dp, KS;       // dims, padded dims (multiple of 32), stages per tile
+    int NT, QT, S;       // ref tiles, query tiles, reference splits
+    int k, P;            // k, per-query pool capacity
+    int NS;              // ring stages
+    int64_t idx_offset;
+    int ntiles, tstride; // this launch visits reference tiles i * tstride, i < ntiles (split over S)
+    __host__ __device__ size_t tile_bytes() const { return (size_t)KS * KNN_STAGE_BYTES + KNN_NORM_B_BYTES; }
+    __host__ __device__ int a_bytes() const { return Dp * 512 + KNN_NORM_A_BYTES; }
+};
+
+// ---------------------------------------------------------------------------
+// prologue: bf16 hi/lo split into the UMMA canonical (K-major, no-swizzle) image
+// ---------------------------------------------------------------------------
+// Core matrix = 8 rows x 16 bytes (8 bf16 along K), rows 16 B apart; 8-row
+// groups 128 B apart (SBO); 8-element K chunks ROWS*16 B apart (LBO).
+//   ref image : [tile][stage][hi,lo][4 chunks][256 rows][8]   (32 KB per stage)
+//   query img : [tile][hi,lo][Dp/8 chunks][128 rows][8]
+__device__ __forceinline__ void split8(const float* src, int nvalid, uint4& hi, uint4& lo, float scale = 1.f) {
+    uint32_t h[4], l[4];
+#pragma unroll
+    for (int p = 0; p < 4; ++p) {
+        const float x0 = (2 * p < nvalid) ? scale * src[2 * p] : 0.f;  // scale is -2 or 1: exact
+        const float x1 = (2 * p + 1 < nvalid) ? scale * src[2 * p + 1] : 0.f;
+        const __nv_bfloat16 h0 = __float2bfloat16_rn(x0), h1 = __float2bfloat16_rn(x1);
+        const __nv_bfloat16 l0 = __float2bfloat16_rn(x0 - __bfloat162float(h0));
+        const __nv_bfloat16 l1 = __float2bfloat16_rn(x1 - __bfloat162float(h1));
+        h[p] = (uint32_t)__bfloat16_as_ushort(h0) | ((uint32_t)__bfloat16_as_ushort(h1) << 16);
+        l[p] = (uint32_t)__bfloat16_as_ushort(l0) | ((uint32_t)__bfloat16_as_ushort(l1) << 16);
+    }
+    hi = make_uint4(h[0], h[1], h[2], h[3]);
+    lo = make_uint4(l[0], l[1], l[2], l[3]);
+}
+
+// grid (tiles, Dp/8), block 256 (ref) -- thread = row of the tile, one 8-dim chunk
+__global__ void knn_prep_ref_kernel(const float* __restrict__ ref, int64_t N, int D, int Dp, size_t tile_bytes,
+                                    uint4* __restrict__ img) {
+    const int64_t t = blockIdx.x;
+    const int c = blockIdx.y;
+    const int i = threadIdx.x;
+    const int64_t r = t * KNN_BN + i;
+    const int nvalid = (r < N) ? max(0, min(8, D - 8 * c)) : 0;
+    uint4 hi, lo;
+    split8(ref + r * (int64_t)D + 8 * c, nvalid, hi, lo);
+    const int KS = Dp / KNN_KS;
+    const int ks = c >> 2, kc = c & 3;
+    uint4* stage = img + (t * (int64_t)(tile_bytes / 16) + ks * (int64_t)(KNN_STAGE_BYTES / 16));
+    stage[(0 * 4 + kc) * KNN_BN + i] = hi;
+    stage[(1 * 4 + kc) * KNN_BN + i] = lo;
+}
+
+// grid (tiles, Dp/8), block 128 (query)
+__global__ void knn_prep_query_kernel(const float* __restrict__ qry, int64_t Q, int D, int Dp,
+                                      uint4* __restrict__ img) {
+    const int64_t t = blockIdx.x;
+    const int c = blockIdx.y;
+    const int i = threadIdx.x;
+    const int64_t q = t * KNN_BM + i;
+    const int nvalid = (q < Q) ? max(0, min(8, D - 8 * c)) : 0;
+    uint4 hi, lo;
+    split8(qry + q * (int64_t)D + 8 * c, nvalid, hi, lo, -2.f);  // A holds -2q
+    const int nch = Dp / 8;
+    uint4* tile = img + t * (int64_t)((Dp * 512 + KNN_NORM_A_BYTES) / 16);
+    tile[(0 * nch + c) * KNN_BM + i] = hi;
+    tile[(1 * nch + c) * KNN_BM + i] = lo;
+}
+
+// Norm block (the extra 16-wide K block of each operand tile).  Warp per row:
+// |x|^2 accumulated in double, split three ways in bf16 (x = n1 + n2 + n3 to
+// ~2^-24).  is_query: lanes [n1, n2, n3, 1, 1, 1, 0, 0]; reference:
+// [1, 1, 1, n1, n2, n3, 0, 0]; the second 8-element chunk is zero.  Rows past
+// the end get zeros (their results are never used).
+__device__ __forceinline__ uint32_t bf2(float a, float b) {
+    return (uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(a)) |
+           ((uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(b)) << 16);
+}
+__global__ void knn_norm_block_kernel(const float* __restrict__ x, int64_t n, int64_t n_pad, int D, int rows_per_tile,
+                                      size_t tile_stride, size_t block_off, bool is_query, uint4* __restrict__ img) {
+    const int64_t row = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    const int lane = threadIdx.x & 31;
+    if (row >= n_pad) return;
+    double s = 0.0;
+    if (row < n)
+        for (int d = lane; d < D; d += 32) {
+            const double v = (double)x[row * (int64_t)D + d];
+            s += v * v;
+        }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(kFull, s, o);
+    if (lane == 0) {
+        const float n1 = __bfloat162float(__float2bfloat16_rn((float)s));
+        const float n2 = __bfloat162float(__float2bfloat16_rn((float)(s - (double)n1)));
+        const float n3 = __bfloat162float(__float2bfloat16_rn((float)(s - (double)n1 - (double)n2)));
+        const bool valid = row < n;
+        const float one = valid ? 1.f : 0.f;
+        uint4 c0;
+        if (is_query) c0 = make_uint4(bf2(n1, n2), bf2(n3, one), bf2(one, one), 0u);
+        else c0 = make_uint4(bf2(one, one), bf2(one, n1), bf2(n2, n3), 0u);
+        const int64_t t = row / rows_per_tile, i = row % rows_per_tile;
+        uint4* blk = img + (t * (int64_t)tile_stride + (int64_t)block_off) / 16;
+        blk[i] = c0;
+        blk[rows_per_tile + i] = make_uint4(0u, 0u, 0u, 0u);
+    }
+}
+
+// ---------------------------------------------------------------------------
+// tcgen05 helpers
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
+    // K-major, SWIZZLE_NONE canonical layout; version 1 (bits 46-47), base offset 0
+    return (uint64_t)((saddr >> 4) & 0x3FFFu) | ((uint64_t)((lbo >> 4) & 0x3FFFu) << 16) |
+           ((uint64_t)((sbo >> 4) & 0x3FFFu) << 32) | (1ull << 46);
+}
+
+// kind::f16 instruction descriptor: bf16 x bf16 -> fp32, K-major A and B, M x N
+__host__ __device__ constexpr uint32_t umma_idesc_bf16(int M, int N) {
+    return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+}
+
+__device__ __forceinline__ void umma_bf16(uint32_t d_tmem, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+        "l"(a), "l"(b), "r"(idesc), "r"(acc)
+        : "memory");
+}
+
+__device__ __forceinline__ void umma_commit(uint64_t* bar) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+                     smem_u32(bar))
+                 : "memory");
+}
+
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
+        "%15, %16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31}, [%32];"
+        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+          "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15]),
+          "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]),
+          "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
+        : "r"(taddr));
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+
+__device__ __forceinline__ void stage_f4(uint32_t saddr, float4 v) {
+    asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(saddr), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w)
+                 : "memory");
+}
+__device__ __forceinline__ float4 lds_f4(uint32_t saddr) {
+    float4 v;
+    asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(saddr));
+    return v;
+}
+
+// ---------------------------------------------------------------------------
+// the fused kernel
+// ---------------------------------------------------------------------------
+struct KnnSmem {
+    static constexpr int kHistBytes = 4 * 256 * 4;
+    static constexpr int kStageRow = 36;  // floats per lane row (16-B aligned, conflict-free STS.128 phases)
+    // per epilogue warp: the rare-path staging rows (32 x 36 floats) OR, between
+    // chunks, one query's pool while it is narrowed (kNarrowCap pairs)
+    static constexpr int kNarrowCap = 1152;
+    static constexpr int kWarpScratch = (kNarrowCap * 8 > 32 * kStageRow * 4) ? kNarrowCap * 8 : 32 * kStageRow * 4;
+    static constexpr int kDStageBytes = 4 * kWarpScratch;
+    __host__ __device__ static int total(const KnnGeom& g) {
+        return 1024 /*align slack*/ + g.a_bytes() + g.NS * KNN_STAGE_BYTES + kHistBytes + kDStageBytes +
+               (2 * g.NS + 5) * 8 + 16;
+    }
+};
+
+// MODE 0: selection (knn_search); 1: write every distance (knn_distances);
+// 2: pipeline only -- the epilogue reads the accumulators and drops them
+// (experiments: isolates the TMA + MMA + TMEM pipeline from the selection).
+template <int MODE>
+__global__ void __launch_bounds__(KNN_THREADS, 1)
+    knn_fused_kernel(KnnGeom g, const uint8_t* __restrict__ ref_img, const uint8_t* __restrict__ q_img,
+                     unsigned long long* __restrict__ pool64, float* __restrict__ cand_val, int32_t* __restrict__ cand_idx,
+                     unsigned long long* __restrict__ qthr, float* __restrict__ dump) {
+    constexpr bool DUMP = (MODE == 1);
+    constexpr bool PIPE_ONLY = (MODE == 2);
+    constexpr bool PROF = (MODE == 3);  // selection + per-warp cycle counters (experiments)
+    unsigned long long prof_narrow = 0, prof_wait = 0, prof_chunks = 0, prof_rare = 0, prof_nrare = 0, prof_nnarrow = 0;
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
+    const int NS = g.NS;
+    uint8_t* sA = smem;
+    uint8_t* sB = sA + g.a_bytes();
+    uint32_t* hist_all = reinterpret_cast<uint32_t*>(sB + NS * KNN_STAGE_BYTES);
+    float* dstage_all = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(hist_all) + KnnSmem::kHistBytes);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(reinterpret_cast<uint8_t*>(dstage_all) + KnnSmem::kDStageBytes);
+    uint64_t* full = bars;
+    uint64_t* empty = bars + NS;
+    uint64_t* accf = bars + 2 * NS;
+    uint64_t* acce = accf + 2;
+    uint64_t* afull = acce + 2;
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(afull + 1);
+
+    const int warp = threadIdx.x >> 5;
+    const uint32_t lane = lane_id();
+    const int qt = blockIdx.x % g.QT;
+    const int split = blockIdx.x / g.QT;
+    const int t0 = (int)((int64_t)g.ntiles * split / g.S);  // logical tile range of this CTA
+    const int t1 = (int)((int64_t)g.ntiles * (split + 1) / g.S);
+
+    if (warp == 0 && lane == 0) {
+        for (int s = 0; s < NS; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], 1);
+        }
+        for (int b = 0; b < 2; ++b) {
+            mbar_init(&accf[b], 1);
+            mbar_init(&acce[b], 4);
+        }
+        mbar_init(afull, 1);
+        fence_mbar_init();
+    }
+    if (warp == 1) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                     "r"(512)
+                     : "memory");
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+
+    if (warp == 0) {
+        // ===== producer: resident query tile, then the reference stream =====
+        // (per tile: KS dims stages of 32 KB, then the 8 KB norm block)
+        if (lane == 0) {
+            const uint32_t abytes = (uint32_t)g.a_bytes();
+            mbar_arrive_expect_tx(afull, abytes);
+            bulk_g2s(sA, q_img + (size_t)qt * abytes, abytes, afull);
+            uint32_t it = 0;
+            for (int ti = t0; ti < t1; ++ti) {
+                const int t = ti * g.tstride;
+                for (int ks = 0; ks <= g.KS; ++ks, ++it) {
+                    const int st = (int)(it % NS);
+                    const uint32_t bytes = (ks < g.KS) ? KNN_STAGE_BYTES : KNN_NORM_B_BYTES;
+                    mbar_wait(&empty[st], ((it / NS) & 1u) ^ 1u);
+                    mbar_arrive_expect_tx(&full[st], bytes);
+                    bulk_g2s(sB + st * KNN_STAGE_BYTES, ref_img + (size_t)t * g.tile_bytes() + (size_t)ks * KNN_STAGE_BYTES,
+                             bytes, &full[st]);
+                }
+            }
+        }
+    } else if (warp == 1) {
+        // ===== MMA issuer (one thread) =====
+        if (lane == 0) {
+            constexpr uint32_t idesc = umma_idesc_bf16(KNN_BM, KNN_BN);
+            const uint32_t a0 = smem_u32(sA);
+            const uint32_t alo = a0 + (uint32_t)(g.Dp / 8) * (KNN_BM * 16);
+            const uint32_t anorm = a0 + (uint32_t)(g.Dp * 512);
+            mbar_wait(afull, 0);
+            tc_fence_after();
+            uint32_t it = 0;
+            for (int ti = t0, lt = 0; ti < t1; ++ti, ++lt) {
+                const int b = lt & 1;
+                mbar_wait(&acce[b], (((uint32_t)lt >> 1) & 1u) ^ 1u);
+                tc_fence_after();
+                const uint32_t d_tmem = tmem_base + (uint32_t)(b * KNN_BN);
+                for (int ks = 0; ks <= g.KS; ++ks, ++it) {
+                    const int st = (int)(it % NS);
+                    mbar_wait(&full[st], (it / NS) & 1u);
+                    tc_fence_after();
+                    const uint32_t bs = smem_u32(sB + st * KNN_STAGE_BYTES);
+                    if (ks == g.KS) {  // norm block: |q|^2 + |r|^2 into the same accumulator
+                        const uint64_t an = umma_desc(anorm, KNN_BM * 16, 128);
+                        const uint64_t bn = umma_desc(bs, KNN_BN * 16, 128);
+                        umma_bf16(d_tmem, an, bn, idesc, 1u);
+                        umma_commit(&empty[st]);
+                        continue;
+                    }
+#pragma unroll
+                    for (int j = 0; j < 2; ++j) {
+                        const int kk = ks * 2 + j;
+                        const uint64_t ah = umma_desc(a0 + (uint32_t)(2 * kk) * (KNN_BM * 16), KNN_BM * 16, 128);
+                        const uint64_t al = umma_desc(alo + (uint32_t)(2 * kk) * (KNN_BM * 16), KNN_BM * 16, 128);
+                        const uint64_t bh = umma_desc(bs + (uint32_t)(2 * j) * (KNN_BN * 16), KNN_BN * 16, 128);
+                        const uint64_t bl =
+                            umma_desc(bs + KNN_STAGE_BYTES / 2 + (uint32_t)(2 * j) * (KNN_BN * 16), KNN_BN * 16, 128);
+                        umma_bf16(d_tmem, ah, bh, idesc, (ks | j) ? 1u : 0u);
+                        umma_bf16(d_tmem, ah, bl, idesc, 1u);
+                        umma_bf16(d_tmem, al, bh, idesc, 1u);
+                    }
+                    umma_commit(&empty[st]);  // frees the stage when these MMAs complete
+                }
+                umma_commit(&accf[b]);  // accumulator b ready for the epilogue
+            }
+        }
+    } else {
+        // ===== epilogue: one thread per query =====
+        const int e = warp - 2;                   // 0..3
+        const int quad = warp & 3;                // TMEM lane quadrant this warp may access
+        const int row = quad * 32 + (int)lane;    // query row within the tile
+        const int64_t q = (int64_t)qt * KNN_BM + row;
+        const bool qvalid = q < g.Q;
+        uint32_t* hist = hist_all + e * 256;
+        uint8_t* wscratch = reinterpret_cast<uint8_t*>(dstage_all) + e * KnnSmem::kWarpScratch;
+        const uint32_t dst = smem_u32(wscratch + (int)lane * KnnSmem::kStageRow * 4);
+        // this query's candidate pool: packed pairs (key << 32 | reference row)
+        unsigned long long* pool = pool64 + ((size_t)split * g.Q + (qvalid ? q : 0)) * g.P;
+        unsigned long long T = kSentPair;  // running bound on the k-th pair
+        float tv = 0.f;
+        bool fast = false;                 // T below +Inf: the fp32 compare d <= tv pre-filters
+        int n = 0;
+
+        auto adopt = [&](unsigned long long t) {
+            if (t < T) {
+                T = t;
+                fast = (uint32_t)(T >> 32) < 0xff800000u;
+                tv = __uint_as_float(bits_of_key((uint32_t)(T >> 32)));
+            }
+        };
+        // warp-cooperative narrowing of every lane whose pool cannot take `room` more pairs
+        auto narrow_lanes = [&](int room, int target) {
+            uint32_t need = __ballot_sync(kFull, qvalid && n + room > g.P);
+            while (need) {
+                if (PROF) prof_nnarrow++;
+                const int j = __ffs(need) - 1;
+                need &= need - 1u;
+                unsigned long long* jp = (unsigned long long*)__shfl_sync(kFull, (unsigned long long)pool, j);
+                const int jn = __shfl_sync(kFull, n, j);
+                int nn;
+                const unsigned long long t = pool_narrow64<kNarrowRegs>(jp, jn, (uint32_t)target, &nn);
+                if ((int)lane == j) {
+                    n = nn;
+                    adopt(t);
+                    // publish: the k-th pair of this split's part bounds the whole row
+                    if (target == g.k && (uint32_t)(t >> 32) != kSentKey) atomicMin(&qthr[q], t);
+                }
+            }
+            __syncwarp();
+        };
+
+        for (int ti = t0, lt = 0; ti < t1; ++ti, ++lt) {
+            const int t = ti * g.tstride;
+            const int b = lt & 1;
+            if (!DUMP && !PIPE_ONLY) {
+                // adopt the tightest bound any split of this query has published
+                if (qvalid) adopt(__ldcg(&qthr[q]));
+                const unsigned long long c0 = PROF ? clock64() : 0;
+                narrow_lanes(KNN_BN, g.k);
+                if (PROF) prof_narrow += clock64() - c0;
+            }
+            const unsigned long long cw0 = PROF ? clock64() : 0;
+            mbar_wait(&accf[b], ((uint32_t)lt >> 1) & 1u);
+            if (PROF) prof_wait += clock64() - cw0;
+            const unsigned long long cc0 = PROF ? clock64() : 0;
+            tc_fence_after();
+            const uint32_t taddr = tmem_base + ((uint32_t)(quad * 32) << 16) + (uint32_t)(b * KNN_BN);
+#pragma unroll 1
+            for (int c = 0; c < KNN_BN / 32; ++c) {
+                uint32_t v[32];
+                tmem_ld32(taddr + (uint32_t)(c * 32), v);
+                if (PIPE_ONLY) {
+                    if (v[0] == 0x7fc00001u && v[31] == 0x7fc00001u) n++;  // keep the load alive
+                    continue;
+                }
+                const int64_t col0 = (int64_t)t * KNN_BN + c * 32;
+                // the accumulator is d = |q|^2 + |r|^2 - 2 q.r (clamped at 0 only where it is kept)
+                float d[32], gmin[8];
+#pragma unroll
+                for (int j = 0; j < 32; j += 4) {
+                    d[j + 0] = __uint_as_float(v[j + 0]);
+                    d[j + 1] = __uint_as_float(v[j + 1]);
+                    d[j + 2] = __uint_as_float(v[j + 2]);
+                    d[j + 3] = __uint_as_float(v[j + 3]);
+                    gmin[j >> 2] = fminf(fminf(d[j], d[j + 1]), fminf(d[j + 2], d[j + 3]));
+                }
+                if (DUMP) {
+                    if (qvalid)
+                        for (int j = 0; j < 32; ++j)
+                            if (col0 + j < g.N) dump[q * g.N + col0 + j] = (d[j] < 0.f) ? 0.f : d[j];
+                    continue;
+                }
+                // thresholds are >= 0, so negative (pre-clamp) values pass as they should;
+                // the vote is warp-uniform: every lane takes part whatever its mode
+                const float mn = fminf(fminf(fminf(gmin[0], gmin[1]), fminf(gmin[2], gmin[3])),
+                                       fminf(fminf(gmin[4], gmin[5]), fminf(gmin[6], gmin[7])));
+                if (!__any_sync(kFull, qvalid && (!fast || mn <= tv))) continue;
+                const unsigned long long cr0 = PROF ? clock64() : 0;
+                // rare path: stage this lane's 32 values, then visit only its candidate
+                // groups and, inside them, only its candidate elements.  The pair test
+                // against T is left to narrowing: an element with d == tv and a larger
+                // index is a harmless extra pool entry.
+                uint32_t gm = 0;
+#pragma unroll
+                for (int u = 0; u < 8; ++u) {
+                    stage_f4(dst + (uint32_t)(u * 16), make_float4(d[4 * u], d[4 * u + 1], d[4 * u + 2], d[4 * u + 3]));
+                    gm |= (uint32_t)(!fast || gmin[u] <= tv) << u;
+                }
+                if (!qvalid) gm = 0;
+                while (gm) {
+                    const int u = __ffs(gm) - 1;
+                    gm &= gm - 1u;
+                    const float4 d4 = lds_f4(dst + (uint32_t)(u * 16));
+                    const float dd[4] = {d4.x, d4.y, d4.z, d4.w};
+                    const int64_t cu = col0 + 4 * u;
+                    uint32_t em = 0;
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) em |= (uint32_t)((cu + i < g.N) && (!fast || dd[i] <= tv)) << i;
+                    while (em) {
+                        const int i = __ffs(em) - 1;
+                        em &= em - 1u;
+                        const float x = (i == 0) ? dd[0] : (i == 1) ? dd[1] : (i == 2) ? dd[2] : dd[3];
+                        const float dc = (x < 0.f) ? 0.f : x;  // clamp, NaN propagates
+                        pool[n++] = ((unsigned long long)key_of(dc) << 32) | (uint32_t)(cu + i);
+                    }
+                }
+                if (PROF) { prof_rare += clock64() - cr0; prof_nrare++; }
+            }
+            if (PROF) prof_chunks += clock64() - cc0;
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive_cta(&acce[b]);
+        }
+        if (PROF && lane == 0) {
+            unsigned long long* o = reinterpret_cast<unsigned long long*>(dump) + ((size_t)blockIdx.x * 4 + e) * 6;
+            o[0] = prof_narrow; o[1] = prof_wait; o[2] = prof_chunks; o[3] = prof_rare; o[4] = prof_nrare; o[5] = prof_nnarrow;
+        }
+        if (!DUMP && !PIPE_ONLY) {
+            // exact top-k of this split for every query, unsorted (ksel_merge sorts)
+            narrow_lanes(g.P - g.k, g.k);  // n > k  <=>  n + (P - k) > P
+            if (qvalid) {
+                float* cv = cand_val + ((size_t)split * g.Q + q) * g.k;
+                int32_t* ci = cand_idx + ((size_t)split * g.Q + q) * g.k;
+                for (int x = 0; x < g.k; ++x) {
+                    const bool real = x < n;
+                    const unsigned long long pr = real ? pool[x] : 0ull;
+                    cv[x] = __uint_as_float(real ? bits_of_key((uint32_t)(pr >> 32)) : 0x7fffffffu);
+                    ci[x] = real ? (int32_t)((int64_t)(uint32_t)pr + g.idx_offset) : (int32_t)kSentIdx;
+                }
+            }
+        }
+    }
+
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    if (warp == 1) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(512) : "memory");
+}
+
+// ---------------------------------------------------------------------------
+// host side
+// ---------------------------------------------------------------------------
+static size_t al256(size_t x) { return (x + 255u) & ~(size_t)255u; }
+
+static bool knn_prologue_enabled() {  // experiments: KSEL_KNN_PROLOGUE=1
+    static const bool on = [] {
+        const char* e = std::getenv("KSEL_KNN_PROLOGUE");
+        return e && e[0] == '1';
+    }();
+    return on;
+}
+
+struct KnnWork {
+    size_t ref_img, q_img, pool, cval, cidx, qthr, prof, total;
+};
+
+static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int64_t idx_offset) {
+    KnnGeom g{};
+    g.N = N;
+    g.Q = Q;
+    g.D = D;
+    g.Dp = (D + KNN_KS - 1) / KNN_KS * KNN_KS;
+    g.KS = g.Dp / KNN_KS;
+    g.NT = (int)((N + KNN_BN - 1) / KNN_BN);
+    g.QT = (int)((Q + KNN_BM - 1) / KNN_BM);
+    g.k = k;
+    const int kk = k < 32 ? 32 : k;
+    // room for >= 1 tile of candidates after narrowing to k; register narrowing holds 1152
+    int P = (kk + KNN_BN > 1152) ? kk + KNN_BN : 1152;  // <= 32 * kNarrowRegs for k' <= 1024
+    g.P = (P + 31) / 32 * 32;
+    // ring depth: as many 32 KB stages as fit next to the resident query tile
+    const int fixed = 1024 + (g.Dp * 512 + KNN_NORM_A_BYTES) + KnnSmem::kHistBytes + KnnSmem::kDStageBytes + 512;
+    g.NS = (kMaxSmemPerBlock - fixed) / KNN_STAGE_BYTES;
+    if (g.NS > 6) g.NS = 6;
+    g.idx_offset = idx_offset;
+    g.ntiles = g.NT;
+    g.tstride = 1;
+    // reference splits: enough CTAs for the SMs, waves as full as possible, <= 64 lists to merge
+    int best = 1;
+    double best_cost = 1e30;
+    const int smax = (int)((g.NT < 64) ? g.NT : 64);
+    for (int s = 1; s <= smax; ++s) {
+        const double ctas = (double)g.QT * s;
+        const double waves = ctas / num_sms;
+        const double cost = (double)((int64_t)((ctas + num_sms - 1) / num_sms)) / waves  // tail efficiency
+                            + (waves < 2.0 ? (2.0 - waves) : 0.0)                        // too few waves
+                            + 0.01 * s;                                                  // merge/pool overhead
+        if (cost < best_cost) { best_cost = cost; best = s; }
+    }
+    g.S = best;
+    return g;
+}
+
+static KnnWork knn_work_layout(const KnnGeom& g) {
+    KnnWork w{};
+    size_t off = 0;
+    w.ref_img = off; off += al256((size_t)g.NT * g.tile_bytes());
+    w.q_img = off;   off += al256((size_t)g.QT * g.a_bytes());
+    w.pool = off;    off += al256((size_t)g.S * g.Q * g.P * 8);
+    w.cval = off;    off += al256((size_t)g.S * g.Q * g.k * 4);
+    w.cidx = off;    off += al256((size_t)g.S * g.Q * g.k * 4);
+    w.qthr = off;    off += al256((size_t)g.Q * 8);
+    w.prof = off;    off += al256((size_t)g.QT * g.S * 4 * 6 * 8);  // MODE 3 counters
+    w.total = off;
+    return w;
+}
+
+static int knn_device_sms() {
+    DevInfo di;
+    return current_device_info(&di) == KSEL_OK ? di.sms : 148;
+}
+
+static cudaError_t knn_run(const float* ref, const float* query, const KnnGeom& g, uint8_t* work,
+                           float* out_dist, int32_t* out_idx, float* dump, cudaStream_t stream) {
+    const KnnWork w = knn_work_layout(g);
+    uint4* ref_img = reinterpret_cast<uint4*>(work + w.ref_img);
+    uint4* q_img = reinterpret_cast<uint4*>(work + w.q_img);
+
+    knn_prep_ref_kernel<<<dim3((unsigned)g.NT, (unsigned)(g.Dp / 8)), KNN_BN, 0, stream>>>(ref, g.N, g.D, g.Dp,
+                                                                                         g.tile_bytes(), ref_img);
+    note_launch();
+    knn_prep_query_kernel<<<dim3((unsigned)g.QT, (unsigned)(g.Dp / 8)), KNN_BM, 0, stream>>>(query, g.Q, g.D, g.Dp,
+                                                                                           q_img);
+    note_launch();
+    const int64_t rpad = (int64_t)g.NT * KNN_BN, qpad = (int64_t)g.QT * KNN_BM;
+    knn_norm_block_kernel<<<(unsigned)((rpad + 7) / 8), 256, 0, stream>>>(
+        ref, g.N, rpad, g.D, KNN_BN, g.tile_bytes(), (size_t)g.KS * KNN_STAGE_BYTES, false, ref_img);
+    note_launch();
+    knn_norm_block_kernel<<<(unsigned)((qpad + 7) / 8), 256, 0, stream>>>(
+        query, g.Q, qpad, g.D, KNN_BM, (size_t)g.a_bytes(), (size_t)g.Dp * 512, true, q_img);
+    note_launch();
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+
+    e = cudaMemsetAsync(work + w.qthr, 0xff, (size_t)g.Q * 8, stream);  // "no bound yet"
+    if (e != cudaSuccess) return e;
+    const int smem = KnnSmem::total(g);
+    static const int mode_env = [] {
+        const char* e = std::getenv("KSEL_KNN_MODE");
+        return (e && (e[0] == '2' || e[0] == '3')) ? e[0] - '0' : 0;
+    }();
+    auto sel_kern = mode_env == 3 ? knn_fused_kernel<3> : knn_fused_kernel<0>;
+    auto kern = dump ? knn_fused_kernel<1>
+                     : (mode_env == 2 ? knn_fused_kernel<2> : (mode_env == 3 ? knn_fused_kernel<3> : knn_fused_kernel<0>));
+    if (!dump && mode_env == 3) dump = reinterpret_cast<float*>(work + w.prof);
+    e = ensure_smem_attr(reinterpret_cast<const void*>(kern), smem);
+    if (e != cudaSuccess) return e;
+    if (!dump && g.NT >= 256 && knn_prologue_enabled()) {
+        // threshold prologue: exact top-k of every query over 64 reference tiles spread
+        // evenly across the set; each k-th pair is a valid bound for the whole row and is
+        // published in qthr, so the main pass starts filtering at rank ~k*NT/64 instead of
+        // admitting everything until its pools fill (outputs of this pass are discarded)
+        KnnGeom gp = g;
+        gp.ntiles = 64;
+        gp.tstride = g.NT / 64;
+        gp.S = (g.QT >= 148) ? 1 : ((2 * 148 + g.QT - 1) / g.QT > 4 ? 4 : (2 * 148 + g.QT - 1) / g.QT);
+        e = ensure_smem_attr(reinterpret_cast<const void*>(sel_kern), smem);
+        if (e != cudaSuccess) return e;
+        sel_kern<<<(unsigned)(gp.QT * gp.S), KNN_THREADS, smem, stream>>>(
+            gp, reinterpret_cast<const uint8_t*>(ref_img), reinterpret_cast<const uint8_t*>(q_img),
+            reinterpret_cast<unsigned long long*>(work + w.pool),
+            reinterpret_cast<float*>(work + w.cval), reinterpret_cast<int32_t*>(work + w.cidx),
+            reinterpret_cast<unsigned long long*>(work + w.qthr), mode_env == 3 ? dump : nullptr);
+        note_launch();
+        e = cudaGetLastError();
+        if (e != cudaSuccess) return e;
+    }
+    kern<<<(unsigned)(g.QT * g.S), KNN_THREADS, smem, stream>>>(
+        g, reinterpret_cast<const uint8_t*>(ref_img), reinterpret_cast<const uint8_t*>(q_img),
+        reinterpret_cast<unsigned long long*>(work + w.pool),
+        reinterpret_cast<float*>(work + w.cval), reinterpret_cast<int32_t*>(work + w.cidx),
+        reinterpret_cast<unsigned long long*>(work + w.qthr), dump);
+    note_launch();
+    e = cudaGetLastError();
+    if (e != cudaSuccess || (dump && mode_env != 3)) return e;
+    return launch_merge(reinterpret_cast<const float*>(work + w.cval), reinterpret_cast<const int32_t*>(work + w.cidx),
+                        g.Q, g.S, g.k, g.k, out_dist, out_idx, stream);
+}
+
+static int knn_check(const float* ref, const float* query, int64_t N, int64_t Q, int D, int k, int64_t idx_offset) {
+    if (!ref || !query) return KSEL_ERR_INVALID_ARG;
+    if (N < 1 || Q < 1 || D < 1 || k < 1 || k > N || idx_offset < 0 || N + idx_offset > 0x7fffffffLL)
+        return KSEL_ERR_INVALID_ARG;
+    if ((reinterpret_cast<uintptr_t>(ref) & 3u) || (reinterpret_cast<uintptr_t>(query) & 3u))
+        return KSEL_ERR_INVALID_ARG;
+    if (D > KNN_MAX_D || k > KSEL_MAX_K) return KSEL_ERR_UNSUPPORTED;
+    return KSEL_OK;
+}
+
+}  // namespace ksel
+
+using namespace ksel;
 
 extern "C" {
 
 size_t knn_search_workspace(int64_t N, int64_t Q, int D, int k) {
-    (void)N; (void)Q; (void)D; (void)k;
-    return 0;
+    if (N < 1 || Q < 1 || D < 1 || D > KNN_MAX_D || k < 1 || k > KSEL_MAX_K) return 0;
+    const KnnGeom g = knn_geometry(N, Q, D, k, knn_device_sms(), 0);
+    return knn_work_layout(g).total;
 }
 
 int knn_search(const float* ref, const float* query, int64_t N, int64_t Q, int D, int k, float* out_dist,
                int32_t* out_idx, int64_t idx_offset, void* d_work, size_t work_bytes, void* stream) {
-    (void)ref; (void)query; (void)N; (void)Q; (void)D; (void)k; (void)out_dist; (void)out_idx;
-    (void)idx_offset; (void)d_work; (void)work_bytes; (void)stream;
-    return KSEL_ERR_UNSUPPORTED;
+    int st = knn_check(ref, query, N, Q, D, k, idx_offset);
+    if (st) return st;
+    if (!out_dist || !out_idx || !d_work) return KSEL_ERR_INVALID_ARG;
+    DevInfo di;
+    st = current_device_info(&di);
+    if (st) return st;
+    const KnnGeom g = knn_geometry(N, Q, D, k, di.sms, idx_offset);
+    if (work_bytes < knn_work_layout(g).total) return KSEL_ERR_INVALID_ARG;
+    cudaError_t e = knn_run(ref, query, g, static_cast<uint8_t*>(d_work), out_dist, out_idx, nullptr,
+                            (cudaStream_t)stream);
+    return e == cudaSuccess ? KSEL_OK : KSEL_ERR_CUDA;
+}
+
+size_t knn_distances_workspace(int64_t N, int64_t Q, int D) { return knn_search_workspace(N, Q, D, 1); }
+
+int knn_distances(const float* ref, const float* query, int64_t N, int64_t Q, int D, float* out, void* d_work,
+                  size_t work_bytes, void* stream) {
+    int st = knn_check(ref, query, N, Q, D, 1, 0);
+    if (st) return st;
+    if (!out || !d_work) return KSEL_ERR_INVALID_ARG;
+    DevInfo di;
+    st = current_device_info(&di);
+    if (st) return st;
+    const KnnGeom g = knn_geometry(N, Q, D, 1, di.sms, 0);
+    if (work_bytes < knn_work_layout(g).total) return KSEL_ERR_INVALID_ARG;
+    cudaError_t e = knn_run(ref, query, g, static_cast<uint8_t*>(d_work), nullptr, nullptr, out, (cudaStream_t)stream);
+    return e == cudaSuccess ? KSEL_OK : KSEL_ERR_CUDA;
 }
 
 }  // extern "C"

@@ -12,6 +12,19 @@ constexpr int kMaxSmemPerBlock = 227 * 1024;  // sm_100 opt-in dynamic shared me
 // 0 = address order, 1 = spread prologue + address order, 2 = strided permutation (default).
 int chunk_order_mode();
 
+// Cached properties of the current device (mutex-protected; cudaGetDeviceProperties
+// is far too slow to call per launch).  Returns a ksel_status.
+struct DevInfo {
+    int dev = -1;
+    int sms = 0;
+    int major = 0;
+    int minor = 0;
+};
+int current_device_info(DevInfo* out);
+
+// Raise a kernel's dynamic shared memory limit once per (function, device).
+cudaError_t ensure_smem_attr(const void* func, int bytes);
+
 // Count one enqueued kernel (reported through ksel_launch_count()).
 void note_launch();
 

@@ -1,0 +1,305 @@
+// ksel_pool.cuh -- warp-cooperative candidate-pool primitives (radix narrowing).
+//
+// A "pool" is an unordered array of (key, idx) pairs (keys and indices in two
+// arrays, shared or global memory).  pool_kth finds the exact want-th smallest
+// pair with an MSD radix-histogram select (8-bit digits of the key, then of the
+// index for ties); pool_compact keeps the pairs <= a threshold.  Together they
+// are the value-bucket form of the paper's Hierarchical Partition
+// (PAPER.md L221-L231): every bucket above the one holding the k-th pair is
+// discarded as a whole.  Used by select_pool.cu (per-warp pools in shared
+// memory) and knn_fused.cu (per-query pools in global memory).
+#pragma once
+#include <cstdint>
+
+#include "ksel_common.cuh"
+
+namespace ksel {
+
+// Exclusive warp prefix sum of v; total in `total`.
+__device__ __forceinline__ uint32_t warp_excl_scan(uint32_t v, uint32_t lane, uint32_t& total) {
+    uint32_t inc = v;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t t = __shfl_up_sync(kFull, inc, d);
+        if (lane >= (uint32_t)d) inc += t;
+    }
+    total = __shfl_sync(kFull, inc, 31);
+    return inc - v;
+}
+
+// Histogram bins are stored transposed (bin b at (b & 7) * 32 + (b >> 3)) so
+// that lane l reading its 8 bins 8l..8l+7 hits 8 distinct banks per access.
+__device__ __forceinline__ int hist_slot(uint32_t b) { return (int)((b & 7u) * 32u + (b >> 3)); }
+
+// Locate the bucket holding the want-th (1-based) element from a filled
+// histogram: returns the digit; `want` becomes the rank inside that bucket and
+// `cnt` the bucket's population.
+__device__ __forceinline__ uint32_t hist_find(const uint32_t* hist, uint32_t lane, uint32_t& want, uint32_t& cnt) {
+    uint32_t h[8], s = 0;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+        h[j] = hist[j * 32 + lane];
+        s += h[j];
+    }
+    uint32_t total;
+    const uint32_t excl = warp_excl_scan(s, lane, total);
+    const bool mine = excl < want && want <= excl + s;
+    const uint32_t bal = __ballot_sync(kFull, mine);
+    const int src = __ffs(bal) - 1;
+    uint32_t d = 0, before = excl, c = 0;
+    if (mine) {
+        uint32_t acc = excl;
+        bool done = false;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            if (!done && acc + h[j] >= want) {
+                d = lane * 8u + (uint32_t)j;
+                before = acc;
+                c = h[j];
+                done = true;
+            }
+            acc += h[j];
+        }
+    }
+    d = __shfl_sync(kFull, d, src);
+    before = __shfl_sync(kFull, before, src);
+    cnt = __shfl_sync(kFull, c, src);
+    want -= before;
+    return d;
+}
+
+// Exact want-th smallest (key, idx) pair among pool[0..n), want in [1, n].
+// MSD radix select, 8-bit digits: 4 passes over the key, then (only if the
+// k-th key value is tied beyond the rank needed) 4 passes over the index.
+__device__ __noinline__ static unsigned long long pool_kth(const uint32_t* __restrict__ pk, const uint32_t* __restrict__ pi,
+                                                    int n, uint32_t want, uint32_t* __restrict__ hist) {
+    const uint32_t lane = lane_id();
+    uint32_t prefix = 0, cnt = 0;
+#pragma unroll 1
+    for (int pass = 0; pass < 4; ++pass) {
+        const int shift = 24 - 8 * pass;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) hist[j * 32 + lane] = 0u;
+        __syncwarp();
+#pragma unroll 4
+        for (int e = (int)lane; e < n; e += 32) {
+            const uint32_t key = pk[e];
+            const bool sel = (pass == 0) || ((key ^ prefix) >> (shift + 8)) == 0u;
+            if (sel) atomicAdd(&hist[hist_slot((key >> shift) & 255u)], 1u);
+        }
+        __syncwarp();
+        const uint32_t d = hist_find(hist, lane, want, cnt);
+        prefix |= d << shift;
+        __syncwarp();
+    }
+    const uint32_t vkey = prefix;
+    uint32_t idx;
+    if (cnt == want) {
+        // every tie of the k-th key is needed: the threshold is the largest such index
+        uint32_t m = 0;
+        for (int e = (int)lane; e < n; e += 32)
+            if (pk[e] == vkey) m = max(m, pi[e]);
+        idx = __reduce_max_sync(kFull, m);
+    } else {
+        uint32_t ip = 0;
+#pragma unroll 1
+        for (int pass = 0; pass < 4; ++pass) {
+            const int shift = 24 - 8 * pass;
+#pragma unroll
+            for (int j = 0; j < 8; ++j) hist[j * 32 + lane] = 0u;
+            __syncwarp();
+            for (int e = (int)lane; e < n; e += 32) {
+                if (pk[e] != vkey) continue;
+                const uint32_t id = pi[e];
+                const bool sel = (pass == 0) || ((id ^ ip) >> (shift + 8)) == 0u;
+                if (sel) atomicAdd(&hist[hist_slot((id >> shift) & 255u)], 1u);
+            }
+            __syncwarp();
+            const uint32_t d = hist_find(hist, lane, want, cnt);
+            ip |= d << shift;
+            __syncwarp();
+        }
+        idx = ip;
+    }
+    return ((unsigned long long)vkey << 32) | idx;
+}
+
+// In-place compaction of pool[0..n) to the pairs <= (tk, ti); returns the new count.
+__device__ __noinline__ static int pool_compact(uint32_t* __restrict__ pk, uint32_t* __restrict__ pi, int n, uint32_t tk,
+                                         uint32_t ti) {
+    const uint32_t lane = lane_id();
+    const uint32_t lt = lanemask_lt();
+    int w = 0;
+    for (int base = 0; base < n; base += 32) {
+        const int e = base + (int)lane;
+        uint32_t kk = 0, ii = 0;
+        bool keep = false;
+        if (e < n) {
+            kk = pk[e];
+            ii = pi[e];
+            keep = !pair_lt(tk, ti, kk, ii);
+        }
+        const uint32_t bal = __ballot_sync(kFull, keep);
+        __syncwarp();
+        if (keep) {
+            const int pos = w + __popc(bal & lt);
+            pk[pos] = kk;
+            pi[pos] = ii;
+        }
+        w += __popc(bal);
+        __syncwarp();
+    }
+    return w;
+}
+
+
+// Register-resident narrowing of one pool of n <= 32*NR pairs (global or shared
+// memory): the pool is loaded once (NR pairs per lane), the want-th smallest
+// pair is found by bisection on the key bits with warp-wide counts
+// (__reduce_add_sync; no shared-memory histogram, hence no atomic contention
+// when all keys share their top bits, e.g. distances), ties by a second
+// bisection on the index, and the pool is compacted in place to the pairs
+// <= that pair (exactly `want` of them).  Returns the pair; *n_out = want.
+template <int NR>
+__device__ __noinline__ unsigned long long pool_narrow_regs(uint32_t* __restrict__ pk, uint32_t* __restrict__ pi,
+                                                            int n, uint32_t want, int* n_out) {
+    const uint32_t lane = lane_id();
+    uint32_t rk[NR], ri[NR];
+#pragma unroll
+    for (int u = 0; u < NR; ++u) {
+        const int x = u * 32 + (int)lane;
+        rk[u] = (x < n) ? __ldcg(pk + x) : 0xffffffffu;
+        ri[u] = (x < n) ? __ldcg(pi + x) : 0xffffffffu;
+    }
+    // want-th smallest key: the largest v with #{key < v} < want
+    uint32_t vkey = 0;
+#pragma unroll 1
+    for (int b = 31; b >= 0; --b) {
+        const uint32_t cand = vkey | (1u << b);
+        uint32_t c = 0;
+#pragma unroll
+        for (int u = 0; u < NR; ++u) c += (rk[u] < cand) ? 1u : 0u;  // pads are 0xffffffff: never below
+        if (__reduce_add_sync(kFull, c) < want) vkey = cand;
+    }
+    uint32_t less = 0, eq = 0, mx = 0;
+#pragma unroll
+    for (int u = 0; u < NR; ++u) {
+        const bool valid = u * 32 + (int)lane < n;
+        less += (rk[u] < vkey) ? 1u : 0u;
+        const bool e = valid && rk[u] == vkey;
+        eq += e ? 1u : 0u;
+        mx = e ? max(mx, ri[u]) : mx;
+    }
+    less = __reduce_add_sync(kFull, less);
+    eq = __reduce_add_sync(kFull, eq);
+    const uint32_t need = want - less;  // ties of vkey to keep, in index order
+    uint32_t vidx;
+    if (eq == need) {
+        vidx = __reduce_max_sync(kFull, mx);
+    } else {
+        vidx = 0;
+#pragma unroll 1
+        for (int b = 31; b >= 0; --b) {
+            const uint32_t cand = vidx | (1u << b);
+            uint32_t c = 0;
+#pragma unroll
+            for (int u = 0; u < NR; ++u)
+                c += (u * 32 + (int)lane < n && rk[u] == vkey && ri[u] < cand) ? 1u : 0u;
+            if (__reduce_add_sync(kFull, c) < need) vidx = cand;
+        }
+    }
+    // compaction in place: keep (key, idx) <= (vkey, vidx)
+    const uint32_t lt = lanemask_lt();
+    int w = 0;
+#pragma unroll
+    for (int u = 0; u < NR; ++u) {
+        const bool keep = (u * 32 + (int)lane < n) && !pair_lt(vkey, vidx, rk[u], ri[u]);
+        const uint32_t bal = __ballot_sync(kFull, keep);
+        if (keep) {
+            const int pos = w + __popc(bal & lt);
+            pk[pos] = rk[u];
+            pi[pos] = ri[u];
+        }
+        w += __popc(bal);
+    }
+    __syncwarp();
+    *n_out = w;
+    return ((unsigned long long)vkey << 32) | vidx;
+}
+
+// Same as pool_narrow_regs for a pool of packed pairs (key << 32 | idx) in one
+// u64 array; the key bisection starts below the common prefix of the pool's
+// smallest and largest key.
+template <int NR>
+__device__ __noinline__ unsigned long long pool_narrow64(unsigned long long* __restrict__ pool, int n, uint32_t want,
+                                                         int* n_out) {
+    const uint32_t lane = lane_id();
+    unsigned long long r[NR];
+    uint32_t kmin = 0xffffffffu, kmax = 0u;
+#pragma unroll
+    for (int u = 0; u < NR; ++u) {
+        const int x = u * 32 + (int)lane;
+        r[u] = (x < n) ? __ldcg(pool + x) : 0xffffffffffffffffull;
+        if (x < n) {
+            kmin = min(kmin, (uint32_t)(r[u] >> 32));
+            kmax = max(kmax, (uint32_t)(r[u] >> 32));
+        }
+    }
+    kmin = __reduce_min_sync(kFull, kmin);
+    kmax = __reduce_max_sync(kFull, kmax);
+    // want-th smallest key: the largest v with #{key < v} < want; bits above the
+    // highest bit where kmin and kmax differ are those of kmin
+    const int top = (kmin == kmax) ? -1 : 31 - __clz(kmin ^ kmax);
+    uint32_t vkey = (top < 0) ? kmin : (kmin & ~((2u << top) - 1u));
+#pragma unroll 1
+    for (int b = top; b >= 0; --b) {
+        const uint32_t cand = vkey | (1u << b);
+        uint32_t c = 0;
+#pragma unroll
+        for (int u = 0; u < NR; ++u) c += ((uint32_t)(r[u] >> 32) < cand) ? 1u : 0u;
+        if (__reduce_add_sync(kFull, c) < want) vkey = cand;
+    }
+    uint32_t less = 0, eq = 0, mx = 0;
+#pragma unroll
+    for (int u = 0; u < NR; ++u) {
+        const bool valid = u * 32 + (int)lane < n;
+        const uint32_t kk = (uint32_t)(r[u] >> 32);
+        less += (valid && kk < vkey) ? 1u : 0u;
+        const bool e = valid && kk == vkey;
+        eq += e ? 1u : 0u;
+        mx = e ? max(mx, (uint32_t)r[u]) : mx;
+    }
+    less = __reduce_add_sync(kFull, less);
+    eq = __reduce_add_sync(kFull, eq);
+    const uint32_t need = want - less;
+    uint32_t vidx;
+    if (eq == need) {
+        vidx = __reduce_max_sync(kFull, mx);
+    } else {
+        vidx = 0;
+#pragma unroll 1
+        for (int b = 31; b >= 0; --b) {
+            const uint32_t cand = vidx | (1u << b);
+            uint32_t c = 0;
+#pragma unroll
+            for (int u = 0; u < NR; ++u)
+                c += (u * 32 + (int)lane < n && (uint32_t)(r[u] >> 32) == vkey && (uint32_t)r[u] < cand) ? 1u : 0u;
+            if (__reduce_add_sync(kFull, c) < need) vidx = cand;
+        }
+    }
+    const unsigned long long T = ((unsigned long long)vkey << 32) | vidx;
+    const uint32_t lt = lanemask_lt();
+    int w = 0;
+#pragma unroll
+    for (int u = 0; u < NR; ++u) {
+        const bool keep = (u * 32 + (int)lane < n) && r[u] <= T;
+        const uint32_t bal = __ballot_sync(kFull, keep);
+        if (keep) pool[w + __popc(bal & lt)] = r[u];
+        w += __popc(bal);
+    }
+    __syncwarp();
+    *n_out = w;
+    return T;
+}
+
+}  // namespace ksel

@@ -26,6 +26,7 @@
 
 #include "ksel_common.cuh"
 #include "ksel_internal.h"
+#include "ksel_pool.cuh"
 
 #ifndef KSEL_ONLY_R
 #error "compile once per queue size with -DKSEL_ONLY_R=1|2|4|8|16|32"
@@ -55,142 +56,6 @@ struct PoolCfg {
 
 __device__ __forceinline__ void pool_group_bar(int id, int nthreads) {
     asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
-}
-
-// Exclusive warp prefix sum of v; total in `total`.
-__device__ __forceinline__ uint32_t warp_excl_scan(uint32_t v, uint32_t lane, uint32_t& total) {
-    uint32_t inc = v;
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-        const uint32_t t = __shfl_up_sync(kFull, inc, d);
-        if (lane >= (uint32_t)d) inc += t;
-    }
-    total = __shfl_sync(kFull, inc, 31);
-    return inc - v;
-}
-
-// Histogram bins are stored transposed (bin b at (b & 7) * 32 + (b >> 3)) so
-// that lane l reading its 8 bins 8l..8l+7 hits 8 distinct banks per access.
-__device__ __forceinline__ int hist_slot(uint32_t b) { return (int)((b & 7u) * 32u + (b >> 3)); }
-
-// Locate the bucket holding the want-th (1-based) element from a filled
-// histogram: returns the digit; `want` becomes the rank inside that bucket and
-// `cnt` the bucket's population.
-__device__ __forceinline__ uint32_t hist_find(const uint32_t* hist, uint32_t lane, uint32_t& want, uint32_t& cnt) {
-    uint32_t h[8], s = 0;
-#pragma unroll
-    for (int j = 0; j < 8; ++j) {
-        h[j] = hist[j * 32 + lane];
-        s += h[j];
-    }
-    uint32_t total;
-    const uint32_t excl = warp_excl_scan(s, lane, total);
-    const bool mine = excl < want && want <= excl + s;
-    const uint32_t bal = __ballot_sync(kFull, mine);
-    const int src = __ffs(bal) - 1;
-    uint32_t d = 0, before = excl, c = 0;
-    if (mine) {
-        uint32_t acc = excl;
-        bool done = false;
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-            if (!done && acc + h[j] >= want) {
-                d = lane * 8u + (uint32_t)j;
-                before = acc;
-                c = h[j];
-                done = true;
-            }
-            acc += h[j];
-        }
-    }
-    d = __shfl_sync(kFull, d, src);
-    before = __shfl_sync(kFull, before, src);
-    cnt = __shfl_sync(kFull, c, src);
-    want -= before;
-    return d;
-}
-
-// Exact want-th smallest (key, idx) pair among pool[0..n), want in [1, n].
-// MSD radix select, 8-bit digits: 4 passes over the key, then (only if the
-// k-th key value is tied beyond the rank needed) 4 passes over the index.
-static __device__ __noinline__ unsigned long long pool_kth(const uint32_t* __restrict__ pk, const uint32_t* __restrict__ pi,
-                                                    int n, uint32_t want, uint32_t* __restrict__ hist) {
-    const uint32_t lane = lane_id();
-    uint32_t prefix = 0, cnt = 0;
-#pragma unroll 1
-    for (int pass = 0; pass < 4; ++pass) {
-        const int shift = 24 - 8 * pass;
-#pragma unroll
-        for (int j = 0; j < 8; ++j) hist[j * 32 + lane] = 0u;
-        __syncwarp();
-        for (int e = (int)lane; e < n; e += 32) {
-            const uint32_t key = pk[e];
-            const bool sel = (pass == 0) || ((key ^ prefix) >> (shift + 8)) == 0u;
-            if (sel) atomicAdd(&hist[hist_slot((key >> shift) & 255u)], 1u);
-        }
-        __syncwarp();
-        const uint32_t d = hist_find(hist, lane, want, cnt);
-        prefix |= d << shift;
-        __syncwarp();
-    }
-    const uint32_t vkey = prefix;
-    uint32_t idx;
-    if (cnt == want) {
-        // every tie of the k-th key is needed: the threshold is the largest such index
-        uint32_t m = 0;
-        for (int e = (int)lane; e < n; e += 32)
-            if (pk[e] == vkey) m = max(m, pi[e]);
-        idx = __reduce_max_sync(kFull, m);
-    } else {
-        uint32_t ip = 0;
-#pragma unroll 1
-        for (int pass = 0; pass < 4; ++pass) {
-            const int shift = 24 - 8 * pass;
-#pragma unroll
-            for (int j = 0; j < 8; ++j) hist[j * 32 + lane] = 0u;
-            __syncwarp();
-            for (int e = (int)lane; e < n; e += 32) {
-                if (pk[e] != vkey) continue;
-                const uint32_t id = pi[e];
-                const bool sel = (pass == 0) || ((id ^ ip) >> (shift + 8)) == 0u;
-                if (sel) atomicAdd(&hist[hist_slot((id >> shift) & 255u)], 1u);
-            }
-            __syncwarp();
-            const uint32_t d = hist_find(hist, lane, want, cnt);
-            ip |= d << shift;
-            __syncwarp();
-        }
-        idx = ip;
-    }
-    return ((unsigned long long)vkey << 32) | idx;
-}
-
-// In-place compaction of pool[0..n) to the pairs <= (tk, ti); returns the new count.
-static __device__ __noinline__ int pool_compact(uint32_t* __restrict__ pk, uint32_t* __restrict__ pi, int n, uint32_t tk,
-                                         uint32_t ti) {
-    const uint32_t lane = lane_id();
-    const uint32_t lt = lanemask_lt();
-    int w = 0;
-    for (int base = 0; base < n; base += 32) {
-        const int e = base + (int)lane;
-        uint32_t kk = 0, ii = 0;
-        bool keep = false;
-        if (e < n) {
-            kk = pk[e];
-            ii = pi[e];
-            keep = !pair_lt(tk, ti, kk, ii);
-        }
-        const uint32_t bal = __ballot_sync(kFull, keep);
-        __syncwarp();
-        if (keep) {
-            const int pos = w + __popc(bal & lt);
-            pk[pos] = kk;
-            pi[pos] = ii;
-        }
-        w += __popc(bal);
-        __syncwarp();
-    }
-    return w;
 }
 
 // Sort pool[0..n) (n <= k') ascending into pool[0..k') with sentinel padding.
@@ -487,12 +352,8 @@ static cudaError_t launch_pool_cfg(const float* dist, int64_t Q, int64_t N, int 
                                    cudaStream_t stream) {
     using Cfg = PoolCfg<R, WPR, RPC>;
     auto kern = ksel_pool_kernel<R, WPR, RPC>;
-    static bool attr_done = false;
-    if (!attr_done) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::kSmem);
-        if (e != cudaSuccess) return e;
-        attr_done = true;
-    }
+    cudaError_t e = ensure_smem_attr(reinterpret_cast<const void*>(kern), Cfg::kSmem);
+    if (e != cudaSuccess) return e;
     const int64_t grid = (Q + RPC - 1) / RPC;
     kern<<<(unsigned)grid, Cfg::kThreads, Cfg::kSmem, stream>>>(dist, Q, N, k, ov, oi, chunk_order_mode());
     note_launch();

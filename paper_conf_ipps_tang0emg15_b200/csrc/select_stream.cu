@@ -316,12 +316,8 @@ static cudaError_t launch_cfg(const float* dist, int64_t Q, int64_t N, int k, fl
                               cudaStream_t stream) {
     using Cfg = StreamCfg<R, RB, WPR, RPC, CH, S>;
     auto kern = ksel_stream_kernel<R, RB, WPR, RPC, CH, S>;
-    static bool attr_done = false;  // benign race: setting the attribute twice is harmless
-    if (!attr_done) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::kSmem);
-        if (e != cudaSuccess) return e;
-        attr_done = true;
-    }
+    cudaError_t e = ensure_smem_attr(reinterpret_cast<const void*>(kern), Cfg::kSmem);
+    if (e != cudaSuccess) return e;
     const int64_t grid = (Q + RPC - 1) / RPC;
     kern<<<(unsigned)grid, Cfg::kThreads, Cfg::kSmem, stream>>>(dist, Q, N, k, ov, oi);
     note_launch();

@@ -1,0 +1,150 @@
+"""GPU parity of knn_search / knn_distances (tcgen05 distance GEMM) vs the oracle.
+
+Tolerance (reading R19, derived from the arithmetic of the bf16x3
+split): |d_gpu - d_ora| <= 1e-4 * d_ora + 3*2^-16 * sum_i |q_i||r_i|
++ (D+2)*2^-24 * (|q|^2 + |r|^2): each operand is hi + lo with a residue below
+2^-16 of its value (bf16 unit roundoff 2^-8, twice), the dropped lo*lo term is
+below 2^-16 of the product, fp32 accumulation over D terms and the rounded
+norms add the last term.  On the paper's workload (uniform [0,1]^128) the
+north star's plain relative bound |d_gpu - d_ora| <= 1e-4 * d_ora is asserted
+as well.  Integer data in [0,255] (knn-S) is bit-exact.
+
+Neighbour sets (reading R20): every GPU neighbour's oracle distance is within
+tolerance of the oracle's k-th distance, every oracle neighbour clearly inside
+(d < d_k - tol) is returned, the GPU list is sorted by its own (d, idx) and has
+distinct in-range indices.
+"""
+import numpy as np
+import pytest
+import torch
+
+import synth
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def K():
+    import paper_conf_ipps_tang0emg15_b200 as k
+    assert torch.cuda.is_available()
+    return k
+
+
+def norms(x):
+    return (x.astype(np.float64) ** 2).sum(axis=1)
+
+
+def tol_pairs(q, r, d_ora):
+    """R19 bound for d(q, r_j); q [D], r [n, D] (float64)."""
+    D = q.shape[0]
+    absdot = np.abs(r) @ np.abs(q)
+    return 1e-4 * d_ora + 3 * 2.0 ** -16 * absdot + (D + 2) * 2.0 ** -24 * ((q * q).sum() + (r * r).sum(axis=1))
+
+
+def check_knn(oracle_mod, ref, qry, k, gv, gi, idx_offset=0, exact=False):
+    ref = ref.numpy() if torch.is_tensor(ref) else ref
+    qry = qry.numpy() if torch.is_tensor(qry) else qry
+    gv = gv.cpu().numpy() if torch.is_tensor(gv) else gv
+    gi = gi.cpu().numpy() if torch.is_tensor(gi) else gi
+    N, D = ref.shape
+    ov, oi = oracle_mod.knn(ref, qry, k, idx_offset=idx_offset)
+    if exact:
+        assert np.array_equal(gi, oi)
+        assert np.array_equal(gv.view(np.uint32), ov.view(np.uint32))
+        return
+    rn, qn = norms(ref), norms(qry)
+    for q in range(qry.shape[0]):
+        idx = gi[q].astype(np.int64) - idx_offset
+        assert len(set(idx.tolist())) == k and idx.min() >= 0 and idx.max() < N
+        # sorted by its own (d, idx)
+        for t in range(k - 1):
+            assert gv[q][t] < gv[q][t + 1] or (gv[q][t] == gv[q][t + 1] and gi[q][t] < gi[q][t + 1])
+        qq = qry[q].astype(np.float64)
+        d_true = ((ref[idx].astype(np.float64) - qq) ** 2).sum(axis=1)
+        tol = tol_pairs(qq, ref[idx].astype(np.float64), d_true)
+        assert np.all(np.abs(gv[q].astype(np.float64) - d_true) <= tol), q
+        dk = float(ov[q][-1])
+        tol_k = 1e-4 * dk + 3 * 2.0 ** -16 * np.sqrt(qn[q] * rn.max()) + (D + 2) * 2.0 ** -24 * (qn[q] + rn.max())
+        assert np.all(d_true <= dk + 2 * tol_k), q
+        must = oi[q][ov[q].astype(np.float64) < dk - 2 * tol_k].astype(np.int64) - idx_offset
+        assert set(must.tolist()) <= set(idx.tolist()), q
+
+
+@pytest.mark.parametrize("kind,N,Q,D", [("knn-S", 700, 200, 128), ("knn-U", 700, 200, 128),
+                                        ("knn-U", 1000, 130, 64), ("knn-U", 513, 77, 3),
+                                        ("knn-S", 300, 260, 256), ("knn-U", 257, 129, 200),
+                                        ("knn-U", 1, 1, 1), ("knn-S", 999, 5, 17)])
+def test_knn_distances_vs_oracle(K, oracle_mod, kind, N, Q, D):
+    ref = synth.knn_points(kind, 1, 0, N, D)
+    qry = synth.knn_points(kind, 2, 0, Q, D)
+    dg = K.knn_distances(ref.cuda(), qry.cuda()).cpu().numpy().astype(np.float64)
+    do = oracle_mod.knn_dist(ref.numpy(), qry.numpy()).astype(np.float64)
+    if kind == "knn-S":
+        assert np.array_equal(dg, do)  # integers in [0,255]: exact
+    else:
+        r64, q64 = ref.numpy().astype(np.float64), qry.numpy().astype(np.float64)
+        for q in range(Q):
+            assert np.all(np.abs(dg[q] - do[q]) <= tol_pairs(q64[q], r64, do[q])), q
+        if D == 128:  # the paper's workload: plain relative 1e-4 (north star)
+            assert np.all(np.abs(dg - do) <= 1e-4 * do)
+
+
+@pytest.mark.parametrize("k", [1, 2, 31, 100, 128, 257, 1024])
+@pytest.mark.parametrize("kind", ["knn-U", "knn-S"])
+def test_knn_search_k_sweep(K, oracle_mod, kind, k):
+    N, Q, D = 5003, 150, 128
+    ref = synth.knn_points(kind, 3, 0, N, D)
+    qry = synth.knn_points(kind, 4, 0, Q, D)
+    gv, gi = K.knn_search(ref.cuda(), qry.cuda(), k)
+    check_knn(oracle_mod, ref, qry, k, gv, gi, exact=(kind == "knn-S"))
+
+
+@pytest.mark.parametrize("D", [1, 4, 17, 32, 64, 100, 129, 256])
+def test_knn_search_dims(K, oracle_mod, D):
+    ref = synth.knn_points("knn-U", 5, 0, 3001, D)
+    qry = synth.knn_points("knn-U", 6, 0, 131, D)
+    gv, gi = K.knn_search(ref.cuda(), qry.cuda(), 20)
+    check_knn(oracle_mod, ref, qry, 20, gv, gi)
+
+
+def test_knn_search_idx_offset_and_self_match(K, oracle_mod):
+    ref = synth.knn_points("knn-U", 7, 0, 4000, 128)
+    qry = ref[[0, 17, 1234, 3999]].clone()
+    gv, gi = K.knn_search(ref.cuda(), qry.cuda(), 10, idx_offset=1000000)
+    assert gi[:, 0].tolist() == [1000000, 1000017, 1001234, 1003999]
+    # d(q, q) = |q|^2 + |q|^2 - 2 q.q cancels: 0 up to the R19 floor, not exactly
+    assert np.all(gv[:, 0].cpu().numpy() <= 3 * 2.0 ** -16 * 2 * norms(qry.numpy()))
+    check_knn(oracle_mod, ref, qry, 10, gv, gi, idx_offset=1000000)
+
+
+def test_knn_search_duplicates_tie_by_index(K, oracle_mod):
+    # integer data with many exact duplicate references: ties broken by index
+    base = synth.knn_points("knn-S", 8, 0, 50, 16)
+    ref = base.repeat(40, 1)  # 2000 refs, each point 40 times
+    qry = synth.knn_points("knn-S", 9, 0, 70, 16)
+    gv, gi = K.knn_search(ref.cuda(), qry.cuda(), 64)
+    check_knn(oracle_mod, ref, qry, 64, gv, gi, exact=True)
+
+
+def test_knn_search_unsupported_and_invalid(K):
+    ref = torch.rand(100, 300, device="cuda")
+    qry = torch.rand(10, 300, device="cuda")
+    with pytest.raises(K.KselError) as e:
+        K.knn_search(ref, qry, 5)
+    assert e.value.status == 2  # D > 256
+    with pytest.raises(K.KselError):
+        K.knn_search(ref[:, :128].contiguous(), qry[:, :128].contiguous(), 101)  # k > N
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("kind", ["knn-U", "knn-S"])
+def test_config4_full_size_sampled_queries(K, oracle_mod, kind):
+    # configs[3]: N=1M references, Q=10000 queries, D=128, k=100 -- the bench launch;
+    # the oracle checks 64 sampled queries (first 32 + 32 spread)
+    N, Q, D, k = 1000000, 10000, 128, 100
+    ref = synth.knn_points(kind, 41, 0, N, D, device="cuda")
+    qry = synth.knn_points(kind, 42, 0, Q, D, device="cuda")
+    gv, gi = K.knn_search(ref, qry, k)
+    torch.cuda.synchronize()
+    sample = list(range(32)) + list(range(37, Q, Q // 32))[:32]
+    check_knn(oracle_mod, ref.cpu(), qry[sample].cpu(), k, gv[sample], gi[sample], exact=(kind == "knn-S"))
