@@ -413,6 +413,32 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
             const unsigned long long cc0 = PROF ? clock64() : 0;
             tc_fence_after();
             const uint32_t taddr = tmem_base + ((uint32_t)(quad * 32) << 16) + (uint32_t)(b * KNN_BN);
+            if (!DUMP && !PIPE_ONLY && lt == 0 && g.k <= KNN_BN && (int64_t)t * KNN_BN + KNN_BN <= g.N &&
+                __any_sync(kFull, qvalid && (uint32_t)(T >> 32) == kSentKey)) {
+                // Starting bound without a fill phase: the exact k-th smallest distance of
+                // this first (full) tile, by bisection on the bits of the clamped value
+                // (non-negative floats order like their bit patterns), re-reading the
+                // accumulator from TMEM each step.  At least k pairs of the row are <= it,
+                // so (that key, any index) is a valid bound.
+                uint32_t vb = 0;
+#pragma unroll 1
+                for (int bit = 30; bit >= 0; --bit) {
+                    const uint32_t cand = vb | (1u << bit);
+                    uint32_t cnt = 0;
+#pragma unroll 1
+                    for (int c = 0; c < KNN_BN / 32; ++c) {
+                        uint32_t v[32];
+                        tmem_ld32(taddr + (uint32_t)(c * 32), v);
+#pragma unroll
+                        for (int j = 0; j < 32; ++j) {
+                            const float x = __uint_as_float(v[j]);
+                            cnt += (__float_as_uint(x < 0.f ? 0.f : x) < cand) ? 1u : 0u;
+                        }
+                    }
+                    if (cnt < (uint32_t)g.k) vb = cand;
+                }
+                if (qvalid) adopt(((unsigned long long)key_of(__uint_as_float(vb)) << 32) | 0x7ffffffeu);
+            }
 #pragma unroll 1
             for (int c = 0; c < KNN_BN / 32; ++c) {
                 uint32_t v[32];
@@ -444,17 +470,16 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
                                        fminf(fminf(gmin[4], gmin[5]), fminf(gmin[6], gmin[7])));
                 if (!__any_sync(kFull, qvalid && (!fast || mn <= tv))) continue;
                 const unsigned long long cr0 = PROF ? clock64() : 0;
-                // rare path: stage this lane's 32 values, then visit only its candidate
-                // groups and, inside them, only its candidate elements.  The pair test
-                // against T is left to narrowing: an element with d == tv and a larger
-                // index is a harmless extra pool entry.
+                // rare path.  The pair test against T is left to narrowing: an element with
+                // d == tv and a larger index is a harmless extra pool entry.
                 uint32_t gm = 0;
 #pragma unroll
-                for (int u = 0; u < 8; ++u) {
-                    stage_f4(dst + (uint32_t)(u * 16), make_float4(d[4 * u], d[4 * u + 1], d[4 * u + 2], d[4 * u + 3]));
-                    gm |= (uint32_t)(!fast || gmin[u] <= tv) << u;
-                }
+                for (int u = 0; u < 8; ++u) gm |= (uint32_t)(!fast || gmin[u] <= tv) << u;
                 if (!qvalid) gm = 0;
+                // stage the lane's 32 values and visit only its own candidate groups
+#pragma unroll
+                for (int u = 0; u < 8; ++u)
+                    stage_f4(dst + (uint32_t)(u * 16), make_float4(d[4 * u], d[4 * u + 1], d[4 * u + 2], d[4 * u + 3]));
                 while (gm) {
                     const int u = __ffs(gm) - 1;
                     gm &= gm - 1u;
