@@ -44,7 +44,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--config", choices=sorted(CONFIGS), default="c3")
+    ap.add_argument("--config", choices=["c1", "c2", "c3", "c4", "c5"], default="c3")
     ap.add_argument("--k", type=int, default=None)
     ap.add_argument("--dist", default=None)
     ap.add_argument("--scaling", choices=["weak", "strong"], default="weak")
@@ -151,7 +151,45 @@ def oracle_rows_per_s(dist: str, seed: int, N: int, k: int, rows: list, threads:
     return len(rows) / dt, dt
 
 
+def run_reference_knn(args, rank, world):
+    """--impl reference for the kNN configs: the oracle (double-precision triple
+    loop + sort) on a bounded sample of queries per step."""
+    if rank != 0:
+        return
+    import oracle
+    import synth
+    N, Q, D, k, kind, mode = KNN_CONFIGS[args.config]
+    k = args.k or k
+    threads = cpu_count()
+    nref = N // world if mode == "row-sharded" else N
+    ref = synth.knn_points(kind, 41, 0, nref, D).numpy()
+    oracle.build()
+    nq = max(4, threads)
+    times = []
+    for s in range(args.warmup + args.steps):
+        qry = synth.knn_points(kind, 42, (s * nq) % Q, nq, D).numpy()
+        t0 = time.perf_counter()
+        oracle.knn(ref, qry, k, nthreads=threads)
+        if s >= args.warmup:
+            times.append(time.perf_counter() - t0)
+    total = sum(times)
+    value = nq * args.steps / total
+    line = {
+        "impl": "reference", "metric": "queries/sec (fused tcgen05 distance + k-selection)", "value": value,
+        "unit": "queries/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": 1e3 * total / args.steps, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "f64", "data": "synthetic",
+        "config": {"workload": "knn_search N=%d Q=%d D=%d k=%d %s (oracle on host cores)" % (nref, Q, D, k, kind)},
+        "cpu_baseline": {"value": value, "unit": "queries/s", "cores": threads, "kind": "oracle",
+                         "sample": "%d queries vs %d references per step" % (nq, nref)},
+        "e2e": {"value": value, "unit": "queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
 def run_reference(args, rank, world):
+    if args.config in KNN_CONFIGS:
+        return run_reference_knn(args, rank, world)
     Qr, N, k, dist = CONFIGS[args.config]
     k = args.k or k
     dist = args.dist or dist
@@ -184,42 +222,11 @@ def run_reference(args, rank, world):
     print(json.dumps(line), flush=True)
 
 
-def main():
-    args = parse()
-    rank = int(os.environ.get("RANK", "0"))
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
-
-    if args.impl == "reference":
-        run_reference(args, rank, world)
-        return
-
+def timed_loop(args, step, world, rank, local_rank, dev, K, tdist):
+    """Warm-up, a ~1 s clock soak, then EXACTLY args.steps timed steps between
+    barriers + device syncs, CUDA events on the launching stream, max over ranks.
+    Also returns the live CUDA-event time of the dominant kernel per launch."""
     import torch
-    import torch.distributed as tdist
-
-    torch.cuda.set_device(local_rank)
-    dev = torch.device("cuda", local_rank)
-    if world > 1:
-        tdist.init_process_group("nccl", device_id=dev)
-
-    import paper_conf_ipps_tang0emg15_b200 as K
-    import synth
-
-    Qr, N, k, dist = CONFIGS[args.config]
-    k = args.k or k
-    dist = args.dist or dist
-    Qglob = Qr * world
-    if args.scaling == "strong":
-        Qglob = Qr
-        Qr = Qglob // world
-    row0 = rank * Qr
-    seed = synth.seed_for(3, dist)
-
-    # ---- inputs resident in HBM (generation is not timed) ----------------------
-    x = synth.rows(dist, seed, row0, Qr, N, device=dev)
-    out_v = torch.empty((Qr, k), dtype=torch.float32, device=dev)
-    out_i = torch.empty((Qr, k), dtype=torch.int32, device=dev)
-    torch.cuda.synchronize()
 
     def barrier():
         if world > 1:
@@ -227,48 +234,67 @@ def main():
 
     stream = torch.cuda.current_stream(dev)
     for _ in range(args.warmup):
-        K.ksel_select(x, k, out_v, out_i)
+        step()
     torch.cuda.synchronize()
-
-    # clocks: sample during a ~1 s soak of the same step and the timed region
     sampler = ClockSampler(local_rank) if rank == 0 else None
     if sampler:
         sampler.start()
     t_soak = time.time()
     while time.time() - t_soak < 1.0:
-        K.ksel_select(x, k, out_v, out_i)
+        step()
         torch.cuda.synchronize()
-
     barrier()
     torch.cuda.synchronize()
+    K.timing_collect()  # drop anything recorded so far
+    K.timing_enable(True)
     l0 = K.launch_count()
     ev0 = torch.cuda.Event(enable_timing=True)
     ev1 = torch.cuda.Event(enable_timing=True)
     ev0.record(stream)
     for _ in range(args.steps):
-        K.ksel_select(x, k, out_v, out_i)
+        step()
     ev1.record(stream)
     torch.cuda.synchronize()
     barrier()
+    K.timing_enable(False)
+    kern_ms, kern_n = K.timing_collect()
     launches = K.launch_count() - l0
     ms = ev0.elapsed_time(ev1)
     clocks = sampler.stop() if sampler else None
-
     t = torch.tensor([ms], dtype=torch.float64, device=dev)
     if world > 1:
         tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
-    ms_max = float(t.item())
+    return float(t.item()), ms, kern_ms / max(1, kern_n), kern_n, launches, clocks
+
+
+def bench_select(args, rank, world, local_rank, dev, K, tdist):
+    import torch
+
+    import synth
+
+    Qr, N, k, dist = CONFIGS[args.config]
+    k = args.k or k
+    dist = args.dist or dist
+    if args.scaling == "strong":
+        Qr = Qr // world
+    row0 = rank * Qr
+    seed = synth.seed_for(3, dist)
+    # ---- inputs resident in HBM (generation is not timed) ----------------------
+    x = synth.rows(dist, seed, row0, Qr, N, device=dev)
+    out_v = torch.empty((Qr, k), dtype=torch.float32, device=dev)
+    out_i = torch.empty((Qr, k), dtype=torch.int32, device=dev)
+    torch.cuda.synchronize()
+
+    ms_max, ms_local, kern_ms, kern_n, launches, clocks = timed_loop(
+        args, lambda: K.ksel_select(x, k, out_v, out_i), world, rank, local_rank, dev, K, tdist)
     ms_step = ms_max / args.steps
     rows_total = Qr * world
     value = rows_total / (ms_step / 1e3)
-
-    # roofline of the dominant (only) kernel: one launch per step on this stream
+    # roofline of the dominant (only) kernel, timed live on the launching stream
     peak, peak_src = load_peaks()
     alg_bytes = Qr * (4.0 * N + 8.0 * k)
-    achieved = alg_bytes / (ms / args.steps / 1e3) / 1e9
+    achieved = alg_bytes / (kern_ms / 1e3) / 1e9
     workload = "ksel_select Q=%d N=%d k=%d %s" % (Qr, N, k, dist)
-    traffic = load_traffic(workload)
-
     line = None
     if rank == 0:
         line = {
@@ -281,14 +307,14 @@ def main():
                        "l2": "inputs (%.1f GiB/rank) far larger than L2; no flush" % (Qr * N * 4 / 2**30)},
             "hbm_gbs": achieved,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
-                         "kernel": "ksel_pool_kernel",
+                         "frac": achieved / peak, "traffic": load_traffic(workload), "peak_source": peak_src,
+                         "kernel": "ksel_pool_kernel", "kernel_ms": kern_ms, "kernel_launches_timed": kern_n,
                          "bytes_per_launch": alg_bytes, "bytes_formula": "Q*(4N+8k)"},
             "gpu_launches": launches,
             "clocks": clocks,
         }
 
-    # ---- end-to-end through the public host API (rank 0 .. all ranks) -------------
+    # ---- end-to-end through the public host API --------------------------------------
     if not args.no_e2e:
         er = min(args.e2e_rows, Qr)
         hx = torch.empty((er, N), dtype=torch.float32, pin_memory=True)
@@ -297,7 +323,8 @@ def main():
         hi = torch.empty((er, k), dtype=torch.int32, pin_memory=True)
         ws = torch.empty(K.ksel_select_host_workspace(N, k), dtype=torch.uint8, device=dev)
         K.ksel_select_host(hx, k, hv, hi, workspace=ws, device=dev)
-        barrier()
+        if world > 1:
+            tdist.barrier()
         t0 = time.perf_counter()
         for _ in range(args.e2e_steps):
             K.ksel_select_host(hx, k, hv, hi, workspace=ws, device=dev)
@@ -320,7 +347,147 @@ def main():
         rps, dt = oracle_rows_per_s(dist, seed, N, k, [row0 + r for r in sample], threads, device=dev)
         line["cpu_baseline"] = {"value": rps, "unit": "rows/s", "cores": threads, "kind": "oracle",
                                 "sample": "%d rows of the same workload (%.1f s)" % (len(sample), dt)}
+    return line
 
+
+KNN_CONFIGS = {
+    # name: (N total, Q, D, k, point kind, mode)
+    "c4": (1000000, 10000, 128, 100, "knn-U", "replica"),
+    "c5": (8000000, 10000, 128, 1024, "knn-U", "row-sharded"),
+}
+
+
+def bench_knn(args, rank, world, local_rank, dev, K, tdist):
+    import torch
+
+    import synth
+    from paper_conf_ipps_tang0emg15_b200 import dist as kd
+
+    N, Q, D, k, kind, mode = KNN_CONFIGS[args.config]
+    k = args.k or k
+    kind = args.dist or kind
+    if mode == "row-sharded":
+        r0, r1 = kd.shard_range(N, world, rank)
+    else:
+        r0, r1 = 0, N
+    Nl = r1 - r0
+    ref = synth.knn_points(kind, 41, r0, Nl, D, device=dev)
+    qry = synth.knn_points(kind, 42, 0, Q, D, device=dev)
+    ws = torch.empty(K.knn_search_workspace(Nl, Q, D, k), dtype=torch.uint8, device=dev)
+    ov = torch.empty((Q, k), dtype=torch.float32, device=dev)
+    oi = torch.empty((Q, k), dtype=torch.int32, device=dev)
+    torch.cuda.synchronize()
+
+    if mode == "row-sharded" and world > 1:
+        def local_knn(rs, qq, kk, off):
+            return K.knn_search(rs, qq, kk, idx_offset=off, out_dist=ov, out_idx=oi, workspace=ws)
+
+        def step():
+            return kd.knn_search_sharded(ref, qry, k, N, local_knn=local_knn)
+    else:
+        def step():
+            return K.knn_search(ref, qry, k, idx_offset=r0, out_dist=ov, out_idx=oi, workspace=ws)
+
+    ms_max, ms_local, kern_ms, kern_n, launches, clocks = timed_loop(args, step, world, rank, local_rank, dev, K, tdist)
+    ms_step = ms_max / args.steps
+    q_total = Q if mode == "row-sharded" else Q * world
+    value = q_total / (ms_step / 1e3)
+    peaks_bf16, src = 1637.7, "measured (MEASURED_PEAKS.json bf16_tflops, burst)"
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            peaks_bf16 = float(json.load(f)["bf16_tflops"])
+    except Exception:
+        src = "fallback (B200_PROFILING.md 1.59 PFLOP/s)"
+        peaks_bf16 = 1590.0
+    flops = 2.0 * Q * Nl * D  # algorithmic single-pass dot products of this rank's launch
+    achieved = flops / (kern_ms / 1e3) / 1e12
+    workload = "knn_search N=%d Q=%d D=%d k=%d %s (%s)" % (N, Q, D, k, kind, mode)
+    line = None
+    if rank == 0:
+        line = {
+            "metric": "queries/sec (fused tcgen05 distance + k-selection)", "value": value, "unit": "queries/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step,
+            "higher_is_better": True, "scaling": "strong" if mode == "row-sharded" else "weak",
+            "vs_baseline": None, "dtype": "bf16x3->f32", "data": "synthetic",
+            "config": {"workload": workload, "N": N, "N_per_rank": Nl, "Q": Q, "D": D, "k": k, "points": kind,
+                       "parallelism": ("reference rows sharded x%d + NCCL all-gather + ksel_merge" % world
+                                       if mode == "row-sharded" else "replicas x%d" % world),
+                       "l2": "reference image %.2f GB per rank (> L2)" % (Nl * D * 4 / 1e9)},
+            "roofline": {"bound": "tensor", "achieved": achieved, "peak": peaks_bf16, "unit": "TFLOP/s",
+                         "frac": achieved / peaks_bf16, "traffic": None, "peak_source": src,
+                         "kernel": "knn_fused_kernel", "kernel_ms": kern_ms,
+                         "flops_per_launch": flops, "flops_formula": "2*Q*N_rank*D (algorithmic, 1 pass; "
+                                                                     "executed: 3 bf16 passes + norm block)"},
+            "gpu_launches": launches,
+            "clocks": clocks,
+        }
+    if not args.no_e2e:
+        # end to end: pinned host inputs copied in every step, results copied back
+        href = torch.empty((Nl, D), dtype=torch.float32, pin_memory=True)
+        href.copy_(ref)
+        hq = torch.empty((Q, D), dtype=torch.float32, pin_memory=True)
+        hq.copy_(qry)
+        hv = torch.empty((Q, k), dtype=torch.float32, pin_memory=True)
+        hi = torch.empty((Q, k), dtype=torch.int32, pin_memory=True)
+
+        def e2e_step():
+            ref.copy_(href, non_blocking=True)
+            qry.copy_(hq, non_blocking=True)
+            v, i = K.knn_search(ref, qry, k, idx_offset=r0, out_dist=ov, out_idx=oi, workspace=ws)
+            hv.copy_(v, non_blocking=True)
+            hi.copy_(i, non_blocking=True)
+            torch.cuda.synchronize()
+
+        e2e_step()
+        t0 = time.perf_counter()
+        for _ in range(args.e2e_steps):
+            e2e_step()
+        dt = torch.tensor([(time.perf_counter() - t0) / args.e2e_steps], dtype=torch.float64, device=dev)
+        if world > 1:
+            tdist.all_reduce(dt, op=tdist.ReduceOp.MAX)
+        if rank == 0:
+            line["e2e"] = {"value": Q * world / float(dt.item()), "unit": "queries/s",
+                           "h2d_bytes_per_step": (Nl + Q) * D * 4, "d2h_bytes_per_step": Q * k * 8,
+                           "api": "knn_search (pinned host inputs copied in each step)"}
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        import oracle
+        threads = cpu_count()
+        nq = max(8, 2 * threads)
+        hr = ref.cpu().numpy()
+        hq = qry[:nq].cpu().numpy()
+        oracle.build()
+        t0 = time.perf_counter()
+        oracle.knn(hr, hq, k, nthreads=threads)
+        dt = time.perf_counter() - t0
+        line["cpu_baseline"] = {"value": nq / dt, "unit": "queries/s", "cores": threads, "kind": "oracle",
+                                "sample": "%d queries vs all %d references (%.1f s)" % (nq, Nl, dt)}
+    return line
+
+
+def main():
+    args = parse()
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+
+    import torch
+    import torch.distributed as tdist
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    if world > 1:
+        tdist.init_process_group("nccl", device_id=dev)
+
+    import paper_conf_ipps_tang0emg15_b200 as K
+
+    if args.config in KNN_CONFIGS:
+        line = bench_knn(args, rank, world, local_rank, dev, K, tdist)
+    else:
+        line = bench_select(args, rank, world, local_rank, dev, K, tdist)
     if rank == 0:
         print(json.dumps(line), flush=True)
     if world > 1:

@@ -136,6 +136,15 @@ KSEL_API size_t knn_distances_workspace(int64_t N, int64_t Q, int D);
 KSEL_API int knn_distances(const float* ref, const float* query, int64_t N, int64_t Q, int D, float* out,
                            void* d_work, size_t work_bytes, void* stream);
 
+/* Live per-kernel timing (measurement support for bench.py): while enabled,
+ * every entry point records a pair of CUDA events on its stream around its
+ * DOMINANT kernel (ksel_select: the selection kernel; knn_search: the fused
+ * distance+selection kernel).  ksel_timing_collect synchronises those events,
+ * returns the summed milliseconds and the number of launches timed, and
+ * clears the record.  Off by default (no events, no overhead). */
+KSEL_API int ksel_timing_enable(int on);
+KSEL_API int ksel_timing_collect(double* total_ms, int64_t* launches);
+
 /* Human-readable text for a ksel_status (static storage, never NULL). */
 KSEL_API const char* ksel_strerror(int status);
 

@@ -42,6 +42,10 @@ _lib.knn_distances_workspace.argtypes = [_i64, _i64, _i32]
 _lib.knn_distances_workspace.restype = _sz
 _lib.knn_distances.argtypes = [_p, _p, _i64, _i64, _i32, _p, _p, _sz, _p]
 _lib.knn_distances.restype = ctypes.c_int
+_lib.ksel_timing_enable.argtypes = [_i32]
+_lib.ksel_timing_enable.restype = ctypes.c_int
+_lib.ksel_timing_collect.argtypes = [ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_int64)]
+_lib.ksel_timing_collect.restype = ctypes.c_int
 _lib.ksel_strerror.argtypes = [_i32]
 _lib.ksel_strerror.restype = ctypes.c_char_p
 _lib.ksel_launch_count.restype = _i64
@@ -51,7 +55,7 @@ for _f in (_lib.ksel_select, _lib.ksel_select_config, _lib.ksel_select_host, _li
 KSEL_MAX_K = 1024
 ALGO_AUTO, ALGO_QUEUE, ALGO_POOL = 0, 1, 2
 EXPORTS = ("ksel_select", "ksel_select_config", "ksel_select_host_workspace", "ksel_select_host", "ksel_merge",
-           "knn_search_workspace", "knn_search", "knn_distances_workspace", "knn_distances", "ksel_strerror",
+           "knn_search_workspace", "knn_search", "knn_distances_workspace", "knn_distances", "ksel_timing_enable", "ksel_timing_collect", "ksel_strerror",
            "ksel_version", "ksel_launch_count")
 
 
@@ -72,6 +76,18 @@ def version() -> int:
 def launch_count() -> int:
     """Kernels enqueued by libksel since load (all entry points)."""
     return _lib.ksel_launch_count()
+
+
+def timing_enable(on: bool = True) -> None:
+    """Record CUDA events around the dominant kernel of every call (bench.py)."""
+    _lib.ksel_timing_enable(1 if on else 0)
+
+
+def timing_collect():
+    """(total milliseconds, launches) of the dominant kernels timed since the last collect."""
+    ms, n = ctypes.c_double(0.0), ctypes.c_int64(0)
+    _check("ksel_timing_collect", _lib.ksel_timing_collect(ctypes.byref(ms), ctypes.byref(n)))
+    return ms.value, n.value
 
 
 def _check(fn, status):

@@ -39,6 +39,31 @@ cudaError_t ensure_smem_attr(const void* func, int bytes) {
     return e;
 }
 
+// ---- dominant-kernel timing ------------------------------------------------
+static std::mutex g_tm_mu;
+static bool g_tm_on = false;
+struct TimedLaunch {
+    cudaEvent_t a, b;
+};
+static TimedLaunch g_tm[4096];
+static int g_tm_n = 0;
+
+int timing_begin(cudaStream_t stream) {
+    std::lock_guard<std::mutex> lock(g_tm_mu);
+    if (!g_tm_on || g_tm_n >= 4096) return -1;
+    TimedLaunch& t = g_tm[g_tm_n];
+    if (cudaEventCreate(&t.a) != cudaSuccess) return -1;
+    if (cudaEventCreate(&t.b) != cudaSuccess) { cudaEventDestroy(t.a); return -1; }
+    cudaEventRecord(t.a, stream);
+    return g_tm_n++;
+}
+
+void timing_end(int slot, cudaStream_t stream) {
+    if (slot < 0) return;
+    std::lock_guard<std::mutex> lock(g_tm_mu);
+    cudaEventRecord(g_tm[slot].b, stream);
+}
+
 int chunk_order_mode() {
     static const int mode = [] {
         const char* e = std::getenv("KSEL_ORDER");
@@ -94,6 +119,32 @@ int ksel_version(void) { return 100; }  // 0.1.0
 
 int64_t ksel_launch_count(void) { return g_launches.load(std::memory_order_relaxed); }
 
+int ksel_timing_enable(int on) {
+    std::lock_guard<std::mutex> lock(g_tm_mu);
+    g_tm_on = on != 0;
+    return KSEL_OK;
+}
+
+int ksel_timing_collect(double* total_ms, int64_t* launches) {
+    if (!total_ms || !launches) return KSEL_ERR_INVALID_ARG;
+    std::lock_guard<std::mutex> lock(g_tm_mu);
+    double tot = 0.0;
+    int st = KSEL_OK;
+    for (int i = 0; i < g_tm_n; ++i) {
+        float ms = 0.f;
+        if (cudaEventSynchronize(g_tm[i].b) != cudaSuccess ||
+            cudaEventElapsedTime(&ms, g_tm[i].a, g_tm[i].b) != cudaSuccess)
+            st = KSEL_ERR_CUDA;
+        tot += ms;
+        cudaEventDestroy(g_tm[i].a);
+        cudaEventDestroy(g_tm[i].b);
+    }
+    *total_ms = tot;
+    *launches = g_tm_n;
+    g_tm_n = 0;
+    return st;
+}
+
 const char* ksel_strerror(int status) {
     switch (status) {
         case KSEL_OK: return "success";
@@ -121,9 +172,11 @@ int ksel_select_config(const float* dist, int64_t Q, int64_t N, int k, float* ou
     if (st) return st;
     const int wpr = warps_per_row ? warps_per_row : stream_warps_per_row(Q, N, di.sms);
     if (algo == KSEL_ALGO_AUTO) algo = KSEL_ALGO_POOL;
+    const int slot = timing_begin((cudaStream_t)stream);
     cudaError_t e = (algo == KSEL_ALGO_QUEUE)
                         ? launch_select_stream(dist, Q, N, k, out_val, out_idx, wpr, (cudaStream_t)stream)
                         : launch_select_pool(dist, Q, N, k, out_val, out_idx, wpr, (cudaStream_t)stream);
+    timing_end(slot, (cudaStream_t)stream);
     return e == cudaSuccess ? KSEL_OK : KSEL_ERR_CUDA;
 }
 

@@ -658,12 +658,14 @@ static cudaError_t knn_run(const float* ref, const float* query, const KnnGeom& 
         e = cudaGetLastError();
         if (e != cudaSuccess) return e;
     }
+    const int slot = dump ? -1 : timing_begin(stream);
     kern<<<(unsigned)(g.QT * g.S), KNN_THREADS, smem, stream>>>(
         g, reinterpret_cast<const uint8_t*>(ref_img), reinterpret_cast<const uint8_t*>(q_img),
         reinterpret_cast<unsigned long long*>(work + w.pool),
         reinterpret_cast<float*>(work + w.cval), reinterpret_cast<int32_t*>(work + w.cidx),
         reinterpret_cast<unsigned long long*>(work + w.qthr), dump);
     note_launch();
+    timing_end(slot, stream);
     e = cudaGetLastError();
     if (e != cudaSuccess || (dump && mode_env != 3)) return e;
     return launch_merge(reinterpret_cast<const float*>(work + w.cval), reinterpret_cast<const int32_t*>(work + w.cidx),

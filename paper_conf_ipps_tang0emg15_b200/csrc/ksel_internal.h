@@ -25,6 +25,11 @@ int current_device_info(DevInfo* out);
 // Raise a kernel's dynamic shared memory limit once per (function, device).
 cudaError_t ensure_smem_attr(const void* func, int bytes);
 
+// Dominant-kernel timing (ksel_timing_enable): bracket a launch on `stream`.
+// timing_begin returns an opaque slot (or -1 when timing is off).
+int timing_begin(cudaStream_t stream);
+void timing_end(int slot, cudaStream_t stream);
+
 // Count one enqueued kernel (reported through ksel_launch_count()).
 void note_launch();
 
