@@ -414,7 +414,7 @@ def bench_knn(args, rank, world, local_rank, dev, K, tdist):
                                        if mode == "row-sharded" else "replicas x%d" % world),
                        "l2": "reference image %.2f GB per rank (> L2)" % (Nl * D * 4 / 1e9)},
             "roofline": {"bound": "tensor", "achieved": achieved, "peak": peaks_bf16, "unit": "TFLOP/s",
-                         "frac": achieved / peaks_bf16, "traffic": None, "peak_source": src,
+                         "frac": achieved / peaks_bf16, "traffic": load_traffic(workload), "peak_source": src,
                          "kernel": "knn_fused_kernel", "kernel_ms": kern_ms,
                          "flops_per_launch": flops, "flops_formula": "2*Q*N_rank*D (algorithmic, 1 pass; "
                                                                      "executed: 3 bf16 passes + norm block)"},

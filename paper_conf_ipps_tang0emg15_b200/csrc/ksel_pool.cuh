@@ -168,8 +168,8 @@ __device__ __noinline__ unsigned long long pool_narrow_regs(uint32_t* __restrict
 #pragma unroll
     for (int u = 0; u < NR; ++u) {
         const int x = u * 32 + (int)lane;
-        rk[u] = (x < n) ? __ldcg(pk + x) : 0xffffffffu;
-        ri[u] = (x < n) ? __ldcg(pi + x) : 0xffffffffu;
+        rk[u] = (x < n) ? pk[x] : 0xffffffffu;  // generic loads: shared- or global-memory pools
+        ri[u] = (x < n) ? pi[x] : 0xffffffffu;
     }
     // want-th smallest key: the largest v with #{key < v} < want
     uint32_t vkey = 0;

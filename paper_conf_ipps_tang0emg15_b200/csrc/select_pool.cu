@@ -39,7 +39,7 @@ struct PoolCfg {
     static constexpr int kQueue = 32 * R;  // k'
     static constexpr int kPool = (2 * kQueue > kQueue + 512) ? 2 * kQueue : kQueue + 512;
     static constexpr int CH = 512;         // floats per staged chunk (2 KB bulk copy)
-    static constexpr int S = 4;            // ring stages per warp
+    static constexpr int S = 3;            // ring stages per warp
     static constexpr int G = 4;            // float4 per lane per sub-step (512 elements per warp)
     static constexpr int NS = 4 * G;       // element slots per lane per sub-step
     static constexpr int kWarps = WPR * RPC;
@@ -207,9 +207,17 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC>::kThreads)
     };
     // pool full: exact k-th of everything seen so far becomes the threshold
     auto narrow = [&]() {
-        const unsigned long long t = pool_kth(pk, pi, n, (uint32_t)k, hist);
+        unsigned long long t;
+        if constexpr (Cfg::kPool <= 32 * 24) {
+            // small pools: register-resident bisection (no histogram atomics)
+            int nn;
+            t = pool_narrow_regs<Cfg::kPool / 32>(pk, pi, n, (uint32_t)k, &nn);
+            n = nn;
+        } else {
+            t = pool_kth(pk, pi, n, (uint32_t)k, hist);
+            n = pool_compact(pk, pi, n, (uint32_t)(t >> 32), (uint32_t)t);
+        }
         const uint32_t kk = (uint32_t)(t >> 32), ki = (uint32_t)t;
-        n = pool_compact(pk, pi, n, kk, ki);
         tighten(kk, ki);
         if (WPR > 1 && lane == 0) atomicMin(grp_thr, t);
     };
@@ -274,6 +282,48 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC>::kThreads)
         }
         n += __popc(bal);
         __syncwarp();
+    }
+
+    // ---- starting bound: the k-th smallest key of the first S staged chunks -----------
+    // (up to S*CH = 2048 values already in flight; bisection over their keys with
+    // warp-wide counts).  At least k elements of the row are <= it, so
+    // (key, largest index) bounds the k-th pair -- the stream then admits a few
+    // times k candidates instead of everything until the pool first fills.
+    if (nmine >= S && k <= S * CH / 2) {
+        uint32_t keys[S * CH / 128 * 4];
+        uint32_t nreal = 0;
+#pragma unroll
+        for (int li = 0; li < S; ++li) {
+            mbar_wait(&mbar[li], 0u);
+            const uint32_t len = chunk_len(cid[li]);
+            const float4* src4 = reinterpret_cast<const float4*>(ring + li * CH);
+#pragma unroll
+            for (int u = 0; u < CH / 128; ++u) {
+                const uint32_t e4 = (uint32_t)u * 32u + lane;
+                const bool ok = e4 * 4u < len;
+                const float4 v = ok ? src4[e4] : make_float4(0.f, 0.f, 0.f, 0.f);
+                const int base = (li * (CH / 128) + u) * 4;
+                keys[base + 0] = ok ? key_of(v.x) : 0xffffffffu;
+                keys[base + 1] = ok ? key_of(v.y) : 0xffffffffu;
+                keys[base + 2] = ok ? key_of(v.z) : 0xffffffffu;
+                keys[base + 3] = ok ? key_of(v.w) : 0xffffffffu;
+                nreal += ok ? 4u : 0u;
+            }
+        }
+        nreal = __reduce_add_sync(kFull, nreal);
+        if (nreal >= (uint32_t)k) {
+            uint32_t vkey = 0;
+#pragma unroll 1
+            for (int bit = 31; bit >= 0; --bit) {
+                const uint32_t cand = vkey | (1u << bit);
+                uint32_t c = 0;
+#pragma unroll
+                for (int j = 0; j < S * CH / 128 * 4; ++j) c += (keys[j] < cand) ? 1u : 0u;
+                if (__reduce_add_sync(kFull, c) < (uint32_t)k) vkey = cand;
+            }
+            tighten(vkey, 0x7ffffffeu);
+            if (WPR > 1 && lane == 0) atomicMin(grp_thr, ((unsigned long long)vkey << 32) | 0x7ffffffeu);
+        }
     }
 
     // ---- streaming body ------------------------------------------------------------------
@@ -378,7 +428,7 @@ cudaError_t launch_pool_r(const float* dist, int64_t Q, int64_t N, int k, float*
                           cudaStream_t stream) {
     switch (wpr) {
         case 1: return launch_pool_fit<R, 1, 1>(dist, Q, N, k, ov, oi, stream);
-        case 2: return launch_pool_fit<R, 2, 2>(dist, Q, N, k, ov, oi, stream);
+        case 2: return launch_pool_fit<R, 2, 1>(dist, Q, N, k, ov, oi, stream);
         case 4: return launch_pool_fit<R, 4, 1>(dist, Q, N, k, ov, oi, stream);
         default: return launch_pool_fit<R, 8, 1>(dist, Q, N, k, ov, oi, stream);
     }
