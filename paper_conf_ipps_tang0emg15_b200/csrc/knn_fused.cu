@@ -50,6 +50,7 @@ constexpr int KNN_STAGE_BYTES = 2 * KNN_KS * KNN_BN * 2;  // hi + lo bf16 = 32 K
 constexpr int KNN_NORM_B_BYTES = 16 * KNN_BN * 2;         // norm block of a reference tile (hi only)
 constexpr int KNN_NORM_A_BYTES = 16 * KNN_BM * 2;         // norm block of a query tile
 constexpr int KNN_THREADS = 192;                         // 6 warps
+constexpr int KNN_CW = 64;                                // accumulator columns per epilogue step
 constexpr int KNN_MAX_D = 256;
 constexpr int kNarrowRegs = 40;  // register-resident narrowing: pools of <= 1280 pairs
 constexpr unsigned long long kSentPair = ((unsigned long long)kSentKey << 32) | kSentIdx;
@@ -204,6 +205,14 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
     asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
 
+__device__ __forceinline__ void tmem_ld64(uint32_t taddr, uint32_t (&v)[64]) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x64.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, %15, %16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31, %32, %33, %34, %35, %36, %37, %38, %39, %40, %41, %42, %43, %44, %45, %46, %47, %48, %49, %50, %51, %52, %53, %54, %55, %56, %57, %58, %59, %60, %61, %62, %63}, [%64];"
+        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]), "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15]), "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]), "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]), "=r"(v[30]), "=r"(v[31]), "=r"(v[32]), "=r"(v[33]), "=r"(v[34]), "=r"(v[35]), "=r"(v[36]), "=r"(v[37]), "=r"(v[38]), "=r"(v[39]), "=r"(v[40]), "=r"(v[41]), "=r"(v[42]), "=r"(v[43]), "=r"(v[44]), "=r"(v[45]), "=r"(v[46]), "=r"(v[47]), "=r"(v[48]), "=r"(v[49]), "=r"(v[50]), "=r"(v[51]), "=r"(v[52]), "=r"(v[53]), "=r"(v[54]), "=r"(v[55]), "=r"(v[56]), "=r"(v[57]), "=r"(v[58]), "=r"(v[59]), "=r"(v[60]), "=r"(v[61]), "=r"(v[62]), "=r"(v[63])
+        : "r"(taddr));
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+
 __device__ __forceinline__ void stage_f4(uint32_t saddr, float4 v) {
     asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(saddr), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w)
                  : "memory");
@@ -219,8 +228,8 @@ __device__ __forceinline__ float4 lds_f4(uint32_t saddr) {
 // ---------------------------------------------------------------------------
 struct KnnSmem {
     static constexpr int kHistBytes = 4 * 256 * 4;
-    static constexpr int kStageRow = 36;  // floats per lane row (16-B aligned, conflict-free STS.128 phases)
-    // per epilogue warp: the rare-path staging rows (32 x 36 floats) OR, between
+    static constexpr int kStageRow = KNN_CW + 4;  // floats per lane row (16-B aligned, conflict-free STS.128 phases)
+    // per epilogue warp: the rare-path staging rows (32 x kStageRow floats) OR, between
     // chunks, one query's pool while it is narrowed (kNarrowCap pairs)
     static constexpr int kNarrowCap = 1152;
     static constexpr int kWarpScratch = (kNarrowCap * 8 > 32 * kStageRow * 4) ? kNarrowCap * 8 : 32 * kStageRow * 4;
@@ -440,18 +449,19 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
                 if (qvalid) adopt(((unsigned long long)key_of(__uint_as_float(vb)) << 32) | 0x7ffffffeu);
             }
 #pragma unroll 1
-            for (int c = 0; c < KNN_BN / 32; ++c) {
-                uint32_t v[32];
-                tmem_ld32(taddr + (uint32_t)(c * 32), v);
+            for (int c = 0; c < KNN_BN / KNN_CW; ++c) {
+                uint32_t v[KNN_CW];
+                tmem_ld64(taddr + (uint32_t)(c * KNN_CW), v);
                 if (PIPE_ONLY) {
-                    if (v[0] == 0x7fc00001u && v[31] == 0x7fc00001u) n++;  // keep the load alive
+                    if (v[0] == 0x7fc00001u && v[KNN_CW - 1] == 0x7fc00001u) n++;  // keep the load alive
                     continue;
                 }
-                const int64_t col0 = (int64_t)t * KNN_BN + c * 32;
+                const int64_t col0 = (int64_t)t * KNN_BN + c * KNN_CW;
                 // the accumulator is d = |q|^2 + |r|^2 - 2 q.r (clamped at 0 only where it is kept)
-                float d[32], gmin[8];
+                constexpr int NGR = KNN_CW / 4;  // 4-column groups
+                float d[KNN_CW], gmin[NGR];
 #pragma unroll
-                for (int j = 0; j < 32; j += 4) {
+                for (int j = 0; j < KNN_CW; j += 4) {
                     d[j + 0] = __uint_as_float(v[j + 0]);
                     d[j + 1] = __uint_as_float(v[j + 1]);
                     d[j + 2] = __uint_as_float(v[j + 2]);
@@ -460,41 +470,40 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
                 }
                 if (DUMP) {
                     if (qvalid)
-                        for (int j = 0; j < 32; ++j)
+                        for (int j = 0; j < KNN_CW; ++j)
                             if (col0 + j < g.N) dump[q * g.N + col0 + j] = (d[j] < 0.f) ? 0.f : d[j];
                     continue;
                 }
                 // thresholds are >= 0, so negative (pre-clamp) values pass as they should;
                 // the vote is warp-uniform: every lane takes part whatever its mode
-                const float mn = fminf(fminf(fminf(gmin[0], gmin[1]), fminf(gmin[2], gmin[3])),
-                                       fminf(fminf(gmin[4], gmin[5]), fminf(gmin[6], gmin[7])));
+                float mn = gmin[0];
+#pragma unroll
+                for (int u = 1; u < NGR; ++u) mn = fminf(mn, gmin[u]);
                 if (!__any_sync(kFull, qvalid && (!fast || mn <= tv))) continue;
                 const unsigned long long cr0 = PROF ? clock64() : 0;
                 // rare path.  The pair test against T is left to narrowing: an element with
                 // d == tv and a larger index is a harmless extra pool entry.
                 uint32_t gm = 0;
 #pragma unroll
-                for (int u = 0; u < 8; ++u) gm |= (uint32_t)(!fast || gmin[u] <= tv) << u;
+                for (int u = 0; u < NGR; ++u) gm |= (uint32_t)(!fast || gmin[u] <= tv) << u;
                 if (!qvalid) gm = 0;
-                // stage the lane's 32 values and visit only its own candidate groups
+                // stage the lane's values and visit only its own candidate groups
 #pragma unroll
-                for (int u = 0; u < 8; ++u)
+                for (int u = 0; u < NGR; ++u)
                     stage_f4(dst + (uint32_t)(u * 16), make_float4(d[4 * u], d[4 * u + 1], d[4 * u + 2], d[4 * u + 3]));
                 while (gm) {
                     const int u = __ffs(gm) - 1;
                     gm &= gm - 1u;
                     const float4 d4 = lds_f4(dst + (uint32_t)(u * 16));
-                    const float dd[4] = {d4.x, d4.y, d4.z, d4.w};
                     const int64_t cu = col0 + 4 * u;
-                    uint32_t em = 0;
+                    // up to 4 candidates, appended branch-free (predicated)
+                    const float dd[4] = {d4.x, d4.y, d4.z, d4.w};
 #pragma unroll
-                    for (int i = 0; i < 4; ++i) em |= (uint32_t)((cu + i < g.N) && (!fast || dd[i] <= tv)) << i;
-                    while (em) {
-                        const int i = __ffs(em) - 1;
-                        em &= em - 1u;
-                        const float x = (i == 0) ? dd[0] : (i == 1) ? dd[1] : (i == 2) ? dd[2] : dd[3];
-                        const float dc = (x < 0.f) ? 0.f : x;  // clamp, NaN propagates
-                        pool[n++] = ((unsigned long long)key_of(dc) << 32) | (uint32_t)(cu + i);
+                    for (int i = 0; i < 4; ++i) {
+                        if ((cu + i < g.N) && (!fast || dd[i] <= tv)) {
+                            const float dc = (dd[i] < 0.f) ? 0.f : dd[i];  // clamp, NaN propagates
+                            pool[n++] = ((unsigned long long)key_of(dc) << 32) | (uint32_t)(cu + i);
+                        }
                     }
                 }
                 if (PROF) { prof_rare += clock64() - cr0; prof_nrare++; }
