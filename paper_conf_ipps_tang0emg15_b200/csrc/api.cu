@@ -65,9 +65,14 @@ void timing_end(int slot, cudaStream_t stream) {
 }
 
 int chunk_order_mode() {
+    // bits 0-1: chunk visit order (KSEL_ORDER, default 2); bit 2: loose admission
+    // experiment (KSEL_LOOSE=1).  Experiments only; the defaults are the product.
     static const int mode = [] {
         const char* e = std::getenv("KSEL_ORDER");
-        return (e && (e[0] == '0' || e[0] == '1' || e[0] == '2')) ? e[0] - '0' : 2;
+        int m = (e && (e[0] == '0' || e[0] == '1' || e[0] == '2')) ? e[0] - '0' : 2;
+        const char* l = std::getenv("KSEL_LOOSE");
+        if (l && l[0] == '1') m |= 4;
+        return m;
     }();
     return mode;
 }
@@ -170,12 +175,16 @@ int ksel_select_config(const float* dist, int64_t Q, int64_t N, int k, float* ou
     DevInfo di;
     st = current_device_info(&di);
     if (st) return st;
-    const int wpr = warps_per_row ? warps_per_row : stream_warps_per_row(Q, N, di.sms);
     if (algo == KSEL_ALGO_AUTO) algo = KSEL_ALGO_POOL;
     const int slot = timing_begin((cudaStream_t)stream);
-    cudaError_t e = (algo == KSEL_ALGO_QUEUE)
-                        ? launch_select_stream(dist, Q, N, k, out_val, out_idx, wpr, (cudaStream_t)stream)
-                        : launch_select_pool(dist, Q, N, k, out_val, out_idx, wpr, (cudaStream_t)stream);
+    cudaError_t e;
+    if (algo == KSEL_ALGO_QUEUE) {
+        const int wpr = warps_per_row ? warps_per_row : stream_warps_per_row(Q, N, di.sms);
+        e = launch_select_stream(dist, Q, N, k, out_val, out_idx, wpr, (cudaStream_t)stream);
+    } else {
+        const int shape = pool_launch_shape(Q, N, k, di.sms, warps_per_row);
+        e = launch_select_pool(dist, Q, N, k, out_val, out_idx, shape, (cudaStream_t)stream);
+    }
     timing_end(slot, (cudaStream_t)stream);
     return e == cudaSuccess ? KSEL_OK : KSEL_ERR_CUDA;
 }
@@ -239,7 +248,7 @@ int ksel_select_host(const float* h_dist, int64_t Q, int64_t N, int k, float* h_
     if (st) return st;
     const cudaStream_t cs = (cudaStream_t)stream;
     const int64_t rows = rps < Q ? rps : Q;
-    const int wpr = stream_warps_per_row(rows, N, di.sms);
+    const int wpr = pool_launch_shape(rows, N, k, di.sms, 0);
 
     const size_t dist_b = al256((size_t)rps * (size_t)N * 4u), val_b = al256((size_t)rps * (size_t)k * 4u);
     const size_t slot_b = host_slot_bytes(rps, N, k);

@@ -19,6 +19,22 @@ int stream_warps_per_row(int64_t Q, int64_t N, int num_sms) {
     return wpr;
 }
 
+int pool_launch_shape(int64_t Q, int64_t N, int k, int num_sms, int forced_wpr) {
+    // Warps per row: spread short/few rows over more warps, but keep >= 128 k'
+    // elements per warp (each warp's pool has to find its own k-th) and >= 8 chunks.
+    const int kp = k <= 32 ? 32 : (k <= 64 ? 64 : (k <= 128 ? 128 : (k <= 256 ? 256 : (k <= 512 ? 512 : 1024))));
+    int wpr = forced_wpr;
+    if (wpr == 0) {
+        wpr = 1;
+        const int64_t seg_min = (int64_t)128 * kp > 4096 ? (int64_t)128 * kp : 4096;
+        while (wpr < 8 && Q * wpr < (int64_t)num_sms * 12 && N / (wpr * 2) >= seg_min) wpr *= 2;
+    }
+    // Deep (6-stage) ring when every warp can be resident at ~19 KB of shared
+    // memory each: more bytes in flight per warp when few warps share an SM.
+    const bool deep = Q * wpr <= (int64_t)num_sms * 11;
+    return deep ? -wpr : wpr;
+}
+
 #define KSEL_DISPATCH_R(FN, R_, ...)                  \
     switch (R_) {                                     \
         case 1: return FN<1>(__VA_ARGS__);            \

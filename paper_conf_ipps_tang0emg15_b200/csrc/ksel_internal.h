@@ -35,6 +35,8 @@ void note_launch();
 
 // Streaming selection (select_stream.cu).
 int stream_warps_per_row(int64_t Q, int64_t N, int num_sms);
+// Pool-kernel launch shape: warps per row, negative = deep (6-stage) ring.
+int pool_launch_shape(int64_t Q, int64_t N, int k, int num_sms, int forced_wpr);
 cudaError_t launch_select_stream(const float* dist, int64_t Q, int64_t N, int k, float* out_val,
                                  int32_t* out_idx, int wpr, cudaStream_t stream);
 

@@ -72,7 +72,8 @@ __device__ __forceinline__ uint32_t hist_find(const uint32_t* hist, uint32_t lan
 // MSD radix select, 8-bit digits: 4 passes over the key, then (only if the
 // k-th key value is tied beyond the rank needed) 4 passes over the index.
 __device__ __noinline__ static unsigned long long pool_kth(const uint32_t* __restrict__ pk, const uint32_t* __restrict__ pi,
-                                                    int n, uint32_t want, uint32_t* __restrict__ hist) {
+                                                    int n, uint32_t want, uint32_t* __restrict__ hist,
+                                                    uint32_t* ties_out = nullptr) {
     const uint32_t lane = lane_id();
     uint32_t prefix = 0, cnt = 0;
 #pragma unroll 1
@@ -93,6 +94,7 @@ __device__ __noinline__ static unsigned long long pool_kth(const uint32_t* __res
         __syncwarp();
     }
     const uint32_t vkey = prefix;
+    if (ties_out) *ties_out = cnt;  // pool entries whose key equals the k-th key
     uint32_t idx;
     if (cnt == want) {
         // every tie of the k-th key is needed: the threshold is the largest such index
@@ -162,7 +164,8 @@ __device__ __noinline__ static int pool_compact(uint32_t* __restrict__ pk, uint3
 // <= that pair (exactly `want` of them).  Returns the pair; *n_out = want.
 template <int NR>
 __device__ __noinline__ unsigned long long pool_narrow_regs(uint32_t* __restrict__ pk, uint32_t* __restrict__ pi,
-                                                            int n, uint32_t want, int* n_out) {
+                                                            int n, uint32_t want, int* n_out,
+                                                            uint32_t* ties_out = nullptr) {
     const uint32_t lane = lane_id();
     uint32_t rk[NR], ri[NR];
 #pragma unroll
@@ -192,6 +195,7 @@ __device__ __noinline__ unsigned long long pool_narrow_regs(uint32_t* __restrict
     }
     less = __reduce_add_sync(kFull, less);
     eq = __reduce_add_sync(kFull, eq);
+    if (ties_out) *ties_out = eq;
     const uint32_t need = want - less;  // ties of vkey to keep, in index order
     uint32_t vidx;
     if (eq == need) {

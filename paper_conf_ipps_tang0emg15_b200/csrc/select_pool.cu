@@ -34,12 +34,13 @@
 
 namespace ksel {
 
-template <int R, int WPR, int RPC>
+template <int R, int WPR, int RPC, int SD = 3>
 struct PoolCfg {
     static constexpr int kQueue = 32 * R;  // k'
     static constexpr int kPool = (2 * kQueue > kQueue + 512) ? 2 * kQueue : kQueue + 512;
     static constexpr int CH = 512;         // floats per staged chunk (2 KB bulk copy)
-    static constexpr int S = 3;            // ring stages per warp
+    static constexpr int NB = (2048 / CH < SD) ? 2048 / CH : SD;  // chunks feeding the starting bound
+    static constexpr int S = SD;           // ring stages per warp (3, or 6 when few warps run per SM)
     static constexpr int G = 4;            // float4 per lane per sub-step (512 elements per warp)
     static constexpr int NS = 4 * G;       // element slots per lane per sub-step
     static constexpr int kWarps = WPR * RPC;
@@ -101,11 +102,11 @@ __device__ __noinline__ void pool_merge_sorted(uint32_t* __restrict__ qk, uint32
     __syncwarp();
 }
 
-template <int R, int WPR, int RPC>
-__global__ void __launch_bounds__(PoolCfg<R, WPR, RPC>::kThreads)
+template <int R, int WPR, int RPC, int SD>
+__global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads)
     ksel_pool_kernel(const float* __restrict__ dist, int64_t Q, int64_t N, int k, float* __restrict__ out_val,
                      int32_t* __restrict__ out_idx, int order_mode) {
-    using Cfg = PoolCfg<R, WPR, RPC>;
+    using Cfg = PoolCfg<R, WPR, RPC, SD>;
     constexpr int CH = Cfg::CH, S = Cfg::S, G = Cfg::G, NS = Cfg::NS;
     extern __shared__ __align__(128) uint8_t smem[];
 
@@ -147,17 +148,17 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC>::kThreads)
     // (incrementally, no divisions); the chunk id travels with the stage.
     const uint32_t nm = (uint32_t)nmine;
     uint32_t np = (nm >= 64u) ? 16u : nm / 4u;
-    if (order_mode == 0) np = 0;
+    if ((order_mode & 3) == 0) np = 0;
     const uint32_t step = np ? nm / np : 1u;
     uint32_t pstride = 1;
-    if (order_mode == 2 && nm > 2u && lane == 0) {
+    if ((order_mode & 3) == 2 && nm > 2u && lane == 0) {
         pstride = ((uint32_t)((double)nm * 0.6180339887498949)) | 1u;
         auto gcd = [](uint32_t a, uint32_t b) { while (b) { const uint32_t t = a % b; a = b; b = t; } return a; };
         while (gcd(pstride, nm) != 1u) pstride += 2;
     }
     uint32_t it_i = 0, it_blk = 0, it_off = 1, it_tail = np * step, it_p = 0;
     auto next_chunk = [&]() -> uint32_t {  // lane 0 only; chunk index relative to c_begin
-        if (order_mode == 2) {
+        if ((order_mode & 3) == 2) {
             const uint32_t c = it_p;
             it_p += pstride;
             if (it_p >= nm) it_p -= nm;
@@ -206,17 +207,24 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC>::kThreads)
         tv = __uint_as_float(bits_of_key(Tk));
     };
     // pool full: exact k-th of everything seen so far becomes the threshold
+    // Admission is loose (value <= bound value: one compare per element) until a
+    // narrowing finds the k-th key tied across many pool entries; from then on this
+    // warp uses the exact lexicographic test, which keeps tied rows (few distinct
+    // values) from filling the pool with equal keys.
+    bool exact_ties = (order_mode & 4) != 0;  // KSEL_LOOSE=1 experiment: exact from the start
     auto narrow = [&]() {
         unsigned long long t;
+        uint32_t ties = 0;
         if constexpr (Cfg::kPool <= 32 * 24) {
             // small pools: register-resident bisection (no histogram atomics)
             int nn;
-            t = pool_narrow_regs<Cfg::kPool / 32>(pk, pi, n, (uint32_t)k, &nn);
+            t = pool_narrow_regs<Cfg::kPool / 32>(pk, pi, n, (uint32_t)k, &nn, &ties);
             n = nn;
         } else {
-            t = pool_kth(pk, pi, n, (uint32_t)k, hist);
+            t = pool_kth(pk, pi, n, (uint32_t)k, hist, &ties);
             n = pool_compact(pk, pi, n, (uint32_t)(t >> 32), (uint32_t)t);
         }
+        if (ties > 16u) exact_ties = true;
         const uint32_t kk = (uint32_t)(t >> 32), ki = (uint32_t)t;
         tighten(kk, ki);
         if (WPR > 1 && lane == 0) atomicMin(grp_thr, t);
@@ -229,33 +237,34 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC>::kThreads)
     auto exact = [&](const float* srcf, uint32_t g, uint32_t len, uint32_t col0, const float(&x)[NS]) {
         uint32_t m = 0;
         if (fast) {
-            // invalid slots of a partial chunk hold +Inf and never pass
+            // exact lexicographic admission, branch-free: value below the bound's, or
+            // equal to it (same key; -0.0 == +0.0) with a smaller index.  Invalid slots of
+            // a partial chunk hold +Inf and never pass.
+            if (!exact_ties) {  // loose admission (x <= tv); ties are left to narrowing
 #pragma unroll
-            for (int j = 0; j < NS; ++j) m |= (uint32_t)(x[j] <= tv) << j;
+                for (int j = 0; j < NS; ++j) m |= (uint32_t)(x[j] <= tv) << j;
+            } else {
+                const uint32_t cbase = col0 + (g * 32u + lane) * 4u;
+#pragma unroll
+                for (int j = 0; j < NS; ++j) {
+                    const uint32_t col = cbase + (uint32_t)((j >> 2) * 128 + (j & 3));
+                    m |= (uint32_t)(x[j] < tv || (x[j] == tv && col < Ti)) << j;
+                }
+            }
         } else {
 #pragma unroll
             for (int u = 0; u < G; ++u)
                 if (((g + (uint32_t)u) * 32u + lane) * 4u < len) m |= 0xfu << (4 * u);
         }
         auto elem = [&](int j) { return ((g + (uint32_t)(j >> 2)) * 32u + lane) * 4u + (uint32_t)(j & 3); };
-        auto refine = [&](uint32_t mm) {
-            uint32_t adm = 0;
-            for (uint32_t t = mm; t; t &= t - 1u) {
-                const int j = __ffs(t) - 1;
-                const uint32_t e = elem(j);
-                if (pair_lt(key_of(srcf[e]), col0 + e, Tk, Ti)) adm |= 1u << j;
-            }
-            return adm;
-        };
-        uint32_t adm = refine(m);
+        // The pool has room for a full sub-step after narrowing (P >= k' + 512); the
+        // pairs flagged before a narrowing inside this sub-step are appended without a
+        // re-test (harmless extra entries, dropped by the next narrowing).
+        const uint32_t adm = m;
         uint32_t total;
-        uint32_t excl = warp_excl_scan(__popc(adm), lane, total);
+        const uint32_t excl = warp_excl_scan(__popc(adm), lane, total);
         if (total == 0) return;
-        if (n + (int)total > Cfg::kPool) {
-            narrow();
-            adm = refine(adm);
-            excl = warp_excl_scan(__popc(adm), lane, total);
-        }
+        if (n + (int)total > Cfg::kPool) narrow();
         int pos = n + (int)excl;
         for (uint32_t t = adm; t; t &= t - 1u) {
             const uint32_t e = elem(__ffs(t) - 1);
@@ -289,11 +298,12 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC>::kThreads)
     // warp-wide counts).  At least k elements of the row are <= it, so
     // (key, largest index) bounds the k-th pair -- the stream then admits a few
     // times k candidates instead of everything until the pool first fills.
-    if (nmine >= S && k <= S * CH / 2) {
-        uint32_t keys[S * CH / 128 * 4];
+    constexpr int NB = Cfg::NB;
+    if (nmine >= NB && k <= NB * CH / 2) {
+        uint32_t keys[NB * CH / 128 * 4];
         uint32_t nreal = 0;
 #pragma unroll
-        for (int li = 0; li < S; ++li) {
+        for (int li = 0; li < NB; ++li) {
             mbar_wait(&mbar[li], 0u);
             const uint32_t len = chunk_len(cid[li]);
             const float4* src4 = reinterpret_cast<const float4*>(ring + li * CH);
@@ -318,7 +328,7 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC>::kThreads)
                 const uint32_t cand = vkey | (1u << bit);
                 uint32_t c = 0;
 #pragma unroll
-                for (int j = 0; j < S * CH / 128 * 4; ++j) c += (keys[j] < cand) ? 1u : 0u;
+                for (int j = 0; j < NB * CH / 128 * 4; ++j) c += (keys[j] < cand) ? 1u : 0u;
                 if (__reduce_add_sync(kFull, c) < (uint32_t)k) vkey = cand;
             }
             tighten(vkey, 0x7ffffffeu);
@@ -397,11 +407,11 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC>::kThreads)
     }
 }
 
-template <int R, int WPR, int RPC>
+template <int R, int WPR, int RPC, int SD>
 static cudaError_t launch_pool_cfg(const float* dist, int64_t Q, int64_t N, int k, float* ov, int32_t* oi,
                                    cudaStream_t stream) {
-    using Cfg = PoolCfg<R, WPR, RPC>;
-    auto kern = ksel_pool_kernel<R, WPR, RPC>;
+    using Cfg = PoolCfg<R, WPR, RPC, SD>;
+    auto kern = ksel_pool_kernel<R, WPR, RPC, SD>;
     cudaError_t e = ensure_smem_attr(reinterpret_cast<const void*>(kern), Cfg::kSmem);
     if (e != cudaSuccess) return e;
     const int64_t grid = (Q + RPC - 1) / RPC;
@@ -412,25 +422,34 @@ static cudaError_t launch_pool_cfg(const float* dist, int64_t Q, int64_t N, int 
 
 // Largest configuration <= (WPR, RPC) whose shared memory fits one SM (227 KB):
 // large queues with many warps per row fall back to fewer warps per CTA.
-template <int R, int WPR, int RPC>
+template <int R, int WPR, int RPC, int SD>
 static cudaError_t launch_pool_fit(const float* dist, int64_t Q, int64_t N, int k, float* ov, int32_t* oi,
                                    cudaStream_t stream) {
-    if constexpr (PoolCfg<R, WPR, RPC>::kSmem > kMaxSmemPerBlock) {
-        if constexpr (RPC > 1) return launch_pool_fit<R, WPR, RPC / 2>(dist, Q, N, k, ov, oi, stream);
-        else return launch_pool_fit<R, WPR / 2, 1>(dist, Q, N, k, ov, oi, stream);
+    if constexpr (PoolCfg<R, WPR, RPC, SD>::kSmem > kMaxSmemPerBlock) {
+        if constexpr (RPC > 1) return launch_pool_fit<R, WPR, RPC / 2, SD>(dist, Q, N, k, ov, oi, stream);
+        else return launch_pool_fit<R, WPR / 2, 1, SD>(dist, Q, N, k, ov, oi, stream);
     } else {
-        return launch_pool_cfg<R, WPR, RPC>(dist, Q, N, k, ov, oi, stream);
+        return launch_pool_cfg<R, WPR, RPC, SD>(dist, Q, N, k, ov, oi, stream);
     }
 }
 
+// wpr < 0 selects the deep ring (6 stages) with |wpr| warps per row.
 template <int R>
 cudaError_t launch_pool_r(const float* dist, int64_t Q, int64_t N, int k, float* ov, int32_t* oi, int wpr,
                           cudaStream_t stream) {
+    if (wpr < 0) {
+        switch (-wpr) {
+            case 1: return launch_pool_fit<R, 1, 1, 6>(dist, Q, N, k, ov, oi, stream);
+            case 2: return launch_pool_fit<R, 2, 1, 6>(dist, Q, N, k, ov, oi, stream);
+            case 4: return launch_pool_fit<R, 4, 1, 6>(dist, Q, N, k, ov, oi, stream);
+            default: return launch_pool_fit<R, 8, 1, 6>(dist, Q, N, k, ov, oi, stream);
+        }
+    }
     switch (wpr) {
-        case 1: return launch_pool_fit<R, 1, 1>(dist, Q, N, k, ov, oi, stream);
-        case 2: return launch_pool_fit<R, 2, 1>(dist, Q, N, k, ov, oi, stream);
-        case 4: return launch_pool_fit<R, 4, 1>(dist, Q, N, k, ov, oi, stream);
-        default: return launch_pool_fit<R, 8, 1>(dist, Q, N, k, ov, oi, stream);
+        case 1: return launch_pool_fit<R, 1, 1, 3>(dist, Q, N, k, ov, oi, stream);
+        case 2: return launch_pool_fit<R, 2, 1, 3>(dist, Q, N, k, ov, oi, stream);
+        case 4: return launch_pool_fit<R, 4, 1, 3>(dist, Q, N, k, ov, oi, stream);
+        default: return launch_pool_fit<R, 8, 1, 3>(dist, Q, N, k, ov, oi, stream);
     }
 }
 
