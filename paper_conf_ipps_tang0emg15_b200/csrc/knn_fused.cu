@@ -395,7 +395,9 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
                 unsigned long long* jp = (unsigned long long*)__shfl_sync(kFull, (unsigned long long)pool, j);
                 const int jn = __shfl_sync(kFull, n, j);
                 int nn;
-                const unsigned long long t = pool_narrow64<kNarrowRegs>(jp, jn, (uint32_t)target, &nn);
+                const unsigned long long t = (jn <= 32 * kNarrowRegs)
+                                                 ? pool_narrow64<kNarrowRegs>(jp, jn, (uint32_t)target, &nn)
+                                                 : pool_select64(jp, jn, (uint32_t)target, hist, &nn);
                 if ((int)lane == j) {
                     n = nn;
                     adopt(t);
@@ -568,7 +570,9 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     g.k = k;
     const int kk = k < 32 ? 32 : k;
     // room for >= 1 tile of candidates after narrowing to k; register narrowing holds 1152
-    int P = (kk + KNN_BN > 1152) ? kk + KNN_BN : 1152;  // <= 32 * kNarrowRegs for k' <= 1024
+    // register narrowing (<= 1280 pairs) for k' <= 128; larger queues get a pool with
+    // room for 8 tiles of candidates between narrowings (radix select, pool_select64)
+    int P = (kk <= 128) ? 1152 : kk + 8 * KNN_BN;
     g.P = (P + 31) / 32 * 32;
     // ring depth: as many 32 KB stages as fit next to the resident query tile
     const int fixed = 1024 + (g.Dp * 512 + KNN_NORM_A_BYTES) + KnnSmem::kHistBytes + KnnSmem::kDStageBytes + 512;
@@ -586,7 +590,7 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
         const double waves = ctas / num_sms;
         const double cost = (double)((int64_t)((ctas + num_sms - 1) / num_sms)) / waves  // tail efficiency
                             + (waves < 2.0 ? (2.0 - waves) : 0.0)                        // too few waves
-                            + 0.01 * s;                                                  // merge/pool overhead
+                            + 0.01 * s * (kk > 128 ? kk / 128.0 : 1.0);                   // merge/pool/cold starts
         if (cost < best_cost) { best_cost = cost; best = s; }
     }
     g.S = best;

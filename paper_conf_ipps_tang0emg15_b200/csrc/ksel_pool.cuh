@@ -306,4 +306,92 @@ __device__ __noinline__ unsigned long long pool_narrow64(unsigned long long* __r
     return T;
 }
 
+// Radix select for large packed-pair pools (key << 32 | idx, any memory): the
+// want-th smallest pair by MSD 8-bit digits of the key, starting below the
+// common prefix of the pool's smallest and largest key (distances share their
+// top bits), then of the index for ties; shared-memory histogram `hist` (256 u32,
+// transposed layout).  The pool is then compacted in place to the pairs <= it.
+__device__ __noinline__ static unsigned long long pool_select64(unsigned long long* __restrict__ pool, int n,
+                                                               uint32_t want, uint32_t* __restrict__ hist,
+                                                               int* n_out) {
+    const uint32_t lane = lane_id();
+    uint32_t kmin = 0xffffffffu, kmax = 0u;
+    for (int e = (int)lane; e < n; e += 32) {
+        const uint32_t kk = (uint32_t)(__ldcg(pool + e) >> 32);
+        kmin = min(kmin, kk);
+        kmax = max(kmax, kk);
+    }
+    kmin = __reduce_min_sync(kFull, kmin);
+    kmax = __reduce_max_sync(kFull, kmax);
+    int hi = (kmin == kmax) ? -1 : 31 - __clz(kmin ^ kmax);
+    uint32_t prefix = (hi < 0) ? kmin : (kmin & ~((2u << hi) - 1u));
+    uint32_t cnt = (uint32_t)n;  // entries matching the resolved prefix (all, initially)
+    // key digits
+    while (hi >= 0) {
+        const int lo = hi >= 7 ? hi - 7 : 0;
+        const uint32_t dmask = (2u << (hi - lo)) - 1u;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) hist[j * 32 + lane] = 0u;
+        __syncwarp();
+#pragma unroll 4
+        for (int e = (int)lane; e < n; e += 32) {
+            const uint32_t kk = (uint32_t)(__ldcg(pool + e) >> 32);
+            const bool sel = (hi == 31) || ((kk ^ prefix) >> (hi + 1)) == 0u;
+            if (sel) atomicAdd(&hist[hist_slot((kk >> lo) & dmask)], 1u);
+        }
+        __syncwarp();
+        const uint32_t d = hist_find(hist, lane, want, cnt);
+        prefix |= d << lo;
+        __syncwarp();
+        hi = lo - 1;
+    }
+    const uint32_t vkey = prefix;
+    uint32_t vidx;
+    if (cnt == want) {
+        uint32_t m = 0;
+        for (int e = (int)lane; e < n; e += 32) {
+            const unsigned long long v = __ldcg(pool + e);
+            if ((uint32_t)(v >> 32) == vkey) m = max(m, (uint32_t)v);
+        }
+        vidx = __reduce_max_sync(kFull, m);
+    } else {
+        uint32_t ip = 0;
+#pragma unroll 1
+        for (int pass = 0; pass < 4; ++pass) {
+            const int shift = 24 - 8 * pass;
+#pragma unroll
+            for (int j = 0; j < 8; ++j) hist[j * 32 + lane] = 0u;
+            __syncwarp();
+            for (int e = (int)lane; e < n; e += 32) {
+                const unsigned long long v = __ldcg(pool + e);
+                if ((uint32_t)(v >> 32) != vkey) continue;
+                const uint32_t id = (uint32_t)v;
+                const bool sel = (pass == 0) || ((id ^ ip) >> (shift + 8)) == 0u;
+                if (sel) atomicAdd(&hist[hist_slot((id >> shift) & 255u)], 1u);
+            }
+            __syncwarp();
+            const uint32_t d = hist_find(hist, lane, want, cnt);
+            ip |= d << shift;
+            __syncwarp();
+        }
+        vidx = ip;
+    }
+    const unsigned long long T = ((unsigned long long)vkey << 32) | vidx;
+    // in-place compaction (reads of a 32-wide slab precede its writes)
+    const uint32_t lt = lanemask_lt();
+    int w = 0;
+    for (int base = 0; base < n; base += 32) {
+        const int e = base + (int)lane;
+        const unsigned long long v = (e < n) ? __ldcg(pool + e) : ~0ull;
+        const bool keep = e < n && v <= T;
+        const uint32_t bal = __ballot_sync(kFull, keep);
+        __syncwarp();
+        if (keep) pool[w + __popc(bal & lt)] = v;
+        w += __popc(bal);
+    }
+    __syncwarp();
+    *n_out = w;
+    return T;
+}
+
 }  // namespace ksel

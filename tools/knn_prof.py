@@ -24,7 +24,7 @@ best, best_cost = 1, 1e30
 for s_ in range(1, min(NT, 64) + 1):
     ctas = QT * s_
     waves = ctas / 148.0
-    cost = ((ctas + 147) // 148) / waves + (2.0 - waves if waves < 2.0 else 0.0) + 0.01 * s_
+    cost = ((ctas + 147) // 148) / waves + (2.0 - waves if waves < 2.0 else 0.0) + 0.01 * s_ * (max(k, 32) / 128.0 if max(k, 32) > 128 else 1.0)
     if cost < best_cost:
         best, best_cost = s_, cost
 S = best
