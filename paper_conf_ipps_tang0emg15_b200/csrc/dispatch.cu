@@ -60,4 +60,10 @@ cudaError_t launch_merge(const float* cv, const int32_t* ci, int64_t Q, int S, i
     KSEL_DISPATCH_R(launch_merge_r, queue_regs(k), cv, ci, Q, S, kin, k, ov, oi, stream)
 }
 
+cudaError_t launch_merge_pools(const unsigned long long* pools, int64_t P, const int32_t* cnt, int S, int64_t Q,
+                               const unsigned long long* thr, int k, int64_t idx_offset, float* ov, int32_t* oi,
+                               cudaStream_t stream) {
+    KSEL_DISPATCH_R(launch_merge_pools_r, queue_regs(k), pools, P, cnt, S, Q, thr, k, idx_offset, ov, oi, stream)
+}
+
 }  // namespace ksel

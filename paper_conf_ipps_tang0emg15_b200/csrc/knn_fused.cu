@@ -23,12 +23,16 @@
 //     warp 0 = producer, warp 1 = TMEM allocator + single-thread MMA issuer,
 //     warps 2-5 = epilogue (one thread per query: the paper's thread-per-query
 //     layout, L243), double-buffered 2 x 256-column accumulators.
-//   * epilogue: tcgen05.ld 32 columns at a time, d = fma(-2, acc, |q|^2+|r|^2),
-//     clamp at 0, and the same pool/threshold selection as select_pool.cu: a
-//     per-query candidate pool (global memory), exact (key, idx) admission test,
-//     warp-cooperative radix narrowing (pool_kth) when a pool fills.
-//   * each CTA leaves the exact top-k of its reference range per query; the
-//     splits are combined by ksel_merge (divide-and-merge, L243).
+//   * epilogue: tcgen05.ld 64 columns at a time (the accumulator already is the
+//     distance), an fp32 min/vote pre-filter against the running bound, a rare
+//     path that appends packed (key << 32 | index) pairs to a per-query pool in
+//     global memory, warp-cooperative narrowing (register bisection, radix
+//     select for large pools) when a pool fills; the k-th pair of every
+//     narrowing is published per query (atomicMin) so all splits share bounds.
+//   * each CTA leaves its per-query pools (a superset of its reference range's
+//     share of the top-k); launch_merge_pools (merge.cu) gathers the pairs below
+//     the final shared bound and selects and sorts the exact top-k -- the
+//     divide-and-merge of L243.
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
@@ -63,6 +67,8 @@ struct KnnGeom {
     int NS;              // ring stages
     int64_t idx_offset;
     int ntiles, tstride; // this launch visits reference tiles i * tstride, i < ntiles (split over S)
+    int sample_tiles;    // cold CTAs (blockIdx < sample_ctas) first histogram this many tiles
+    int sample_ctas;
     __host__ __device__ size_t tile_bytes() const { return (size_t)KS * KNN_STAGE_BYTES + KNN_NORM_B_BYTES; }
     __host__ __device__ int a_bytes() const { return Dp * 512 + KNN_NORM_A_BYTES; }
 };
@@ -74,90 +80,91 @@ struct KnnGeom {
 // groups 128 B apart (SBO); 8-element K chunks ROWS*16 B apart (LBO).
 //   ref image : [tile][stage][hi,lo][4 chunks][256 rows][8]   (32 KB per stage)
 //   query img : [tile][hi,lo][Dp/8 chunks][128 rows][8]
-__device__ __forceinline__ void split8(const float* src, int nvalid, uint4& hi, uint4& lo, float scale = 1.f) {
-    uint32_t h[4], l[4];
-#pragma unroll
-    for (int p = 0; p < 4; ++p) {
-        const float x0 = (2 * p < nvalid) ? scale * src[2 * p] : 0.f;  // scale is -2 or 1: exact
-        const float x1 = (2 * p + 1 < nvalid) ? scale * src[2 * p + 1] : 0.f;
-        const __nv_bfloat16 h0 = __float2bfloat16_rn(x0), h1 = __float2bfloat16_rn(x1);
-        const __nv_bfloat16 l0 = __float2bfloat16_rn(x0 - __bfloat162float(h0));
-        const __nv_bfloat16 l1 = __float2bfloat16_rn(x1 - __bfloat162float(h1));
-        h[p] = (uint32_t)__bfloat16_as_ushort(h0) | ((uint32_t)__bfloat16_as_ushort(h1) << 16);
-        l[p] = (uint32_t)__bfloat16_as_ushort(l0) | ((uint32_t)__bfloat16_as_ushort(l1) << 16);
-    }
-    hi = make_uint4(h[0], h[1], h[2], h[3]);
-    lo = make_uint4(l[0], l[1], l[2], l[3]);
-}
 
-// grid (tiles, Dp/8), block 256 (ref) -- thread = row of the tile, one 8-dim chunk
-__global__ void knn_prep_ref_kernel(const float* __restrict__ ref, int64_t N, int D, int Dp, size_t tile_bytes,
-                                    uint4* __restrict__ img) {
-    const int64_t t = blockIdx.x;
-    const int c = blockIdx.y;
-    const int i = threadIdx.x;
-    const int64_t r = t * KNN_BN + i;
-    const int nvalid = (r < N) ? max(0, min(8, D - 8 * c)) : 0;
-    uint4 hi, lo;
-    split8(ref + r * (int64_t)D + 8 * c, nvalid, hi, lo);
-    const int KS = Dp / KNN_KS;
-    const int ks = c >> 2, kc = c & 3;
-    uint4* stage = img + (t * (int64_t)(tile_bytes / 16) + ks * (int64_t)(KNN_STAGE_BYTES / 16));
-    stage[(0 * 4 + kc) * KNN_BN + i] = hi;
-    stage[(1 * 4 + kc) * KNN_BN + i] = lo;
-}
-
-// grid (tiles, Dp/8), block 128 (query)
-__global__ void knn_prep_query_kernel(const float* __restrict__ qry, int64_t Q, int D, int Dp,
-                                      uint4* __restrict__ img) {
-    const int64_t t = blockIdx.x;
-    const int c = blockIdx.y;
-    const int i = threadIdx.x;
-    const int64_t q = t * KNN_BM + i;
-    const int nvalid = (q < Q) ? max(0, min(8, D - 8 * c)) : 0;
-    uint4 hi, lo;
-    split8(qry + q * (int64_t)D + 8 * c, nvalid, hi, lo, -2.f);  // A holds -2q
-    const int nch = Dp / 8;
-    uint4* tile = img + t * (int64_t)((Dp * 512 + KNN_NORM_A_BYTES) / 16);
-    tile[(0 * nch + c) * KNN_BM + i] = hi;
-    tile[(1 * nch + c) * KNN_BM + i] = lo;
-}
-
-// Norm block (the extra 16-wide K block of each operand tile).  Warp per row:
-// |x|^2 accumulated in double, split three ways in bf16 (x = n1 + n2 + n3 to
-// ~2^-24).  is_query: lanes [n1, n2, n3, 1, 1, 1, 0, 0]; reference:
-// [1, 1, 1, n1, n2, n3, 0, 0]; the second 8-element chunk is zero.  Rows past
-// the end get zeros (their results are never used).
+// bf16 pair of two floats (round to nearest even)
 __device__ __forceinline__ uint32_t bf2(float a, float b) {
     return (uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(a)) |
            ((uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(b)) << 16);
 }
-__global__ void knn_norm_block_kernel(const float* __restrict__ x, int64_t n, int64_t n_pad, int D, int rows_per_tile,
-                                      size_t tile_stride, size_t block_off, bool is_query, uint4* __restrict__ img) {
-    const int64_t row = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
-    const int lane = threadIdx.x & 31;
-    if (row >= n_pad) return;
+
+// One launch builds both operand images: blocks [0, NT) are reference tiles
+// (256 rows), blocks [NT, NT + QT) query tiles (128 rows, scaled by -2).  Each
+// block reads its rows once, 32 dims at a time, coalesced (a warp reads 32
+// consecutive floats of one row) into shared memory; thread i then owns row i:
+// accumulates |x|^2 in double and writes the hi/lo chunks of its row (16 B per
+// thread, consecutive threads -> consecutive 16 B).  Last, the norm block (the
+// extra 16-wide K block): |x|^2 split three ways in bf16 (x = n1 + n2 + n3 to
+// ~2^-24); queries [n1, n2, n3, 1, 1, 1, 0, 0], references [1, 1, 1, n1, n2, n3,
+// 0, 0], second 8-element chunk zero.  Rows past the end are all zeros.
+constexpr int KNN_PREP_THREADS = 256;
+
+__global__ void __launch_bounds__(KNN_PREP_THREADS)
+    knn_prep_kernel(const float* __restrict__ ref, const float* __restrict__ qry, KnnGeom g,
+                    uint4* __restrict__ ref_img, uint4* __restrict__ q_img) {
+    __shared__ float tile[KNN_BN][KNN_KS + 1];
+    const bool is_q = blockIdx.x >= (unsigned)g.NT;
+    const int64_t t = is_q ? (int64_t)blockIdx.x - g.NT : (int64_t)blockIdx.x;
+    const int rows = is_q ? KNN_BM : KNN_BN;
+    const int64_t n = is_q ? g.Q : g.N;
+    const float* x = is_q ? qry : ref;
+    const float scale = is_q ? -2.f : 1.f;  // exact
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int64_t row = t * rows + tid;
     double s = 0.0;
-    if (row < n)
-        for (int d = lane; d < D; d += 32) {
-            const double v = (double)x[row * (int64_t)D + d];
-            s += v * v;
+    for (int ks = 0; ks < g.KS; ++ks) {
+        const int d = ks * KNN_KS + lane;
+#pragma unroll 8
+        for (int r = warp; r < rows; r += KNN_PREP_THREADS / 32) {
+            const int64_t gr = t * rows + r;
+            tile[r][lane] = (gr < n && d < g.D) ? __ldcs(x + gr * (int64_t)g.D + d) : 0.f;
         }
+        __syncthreads();
+        if (tid < rows) {
+            uint4* dst;
+            int cstride;
+            if (is_q) {  // [hi,lo][Dp/8 chunks][128 rows][8]
+                dst = q_img + t * (int64_t)(g.a_bytes() / 16) + (int64_t)(ks * 4) * KNN_BM + tid;
+                cstride = KNN_BM;
+            } else {     // [stage][hi,lo][4 chunks][256 rows][8]
+                dst = ref_img + t * (int64_t)(g.tile_bytes() / 16) + (int64_t)ks * (KNN_STAGE_BYTES / 16) + tid;
+                cstride = KNN_BN;
+            }
+            const int64_t lo_off = is_q ? (int64_t)(g.Dp / 8) * KNN_BM : 4 * KNN_BN;
 #pragma unroll
-    for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(kFull, s, o);
-    if (lane == 0) {
+            for (int kc = 0; kc < 4; ++kc) {
+                uint32_t h[4], l[4];
+#pragma unroll
+                for (int p = 0; p < 4; ++p) {
+                    const float v0 = tile[tid][kc * 8 + 2 * p], v1 = tile[tid][kc * 8 + 2 * p + 1];
+                    s += (double)v0 * (double)v0;
+                    s += (double)v1 * (double)v1;
+                    const float x0 = scale * v0, x1 = scale * v1;
+                    const __nv_bfloat16 h0 = __float2bfloat16_rn(x0), h1 = __float2bfloat16_rn(x1);
+                    h[p] = (uint32_t)__bfloat16_as_ushort(h0) | ((uint32_t)__bfloat16_as_ushort(h1) << 16);
+                    l[p] = bf2(x0 - __bfloat162float(h0), x1 - __bfloat162float(h1));
+                }
+                dst[kc * cstride] = make_uint4(h[0], h[1], h[2], h[3]);
+                dst[lo_off + kc * cstride] = make_uint4(l[0], l[1], l[2], l[3]);
+            }
+        }
+        __syncthreads();
+    }
+    if (tid < rows) {
         const float n1 = __bfloat162float(__float2bfloat16_rn((float)s));
         const float n2 = __bfloat162float(__float2bfloat16_rn((float)(s - (double)n1)));
         const float n3 = __bfloat162float(__float2bfloat16_rn((float)(s - (double)n1 - (double)n2)));
-        const bool valid = row < n;
-        const float one = valid ? 1.f : 0.f;
+        const float one = (row < n) ? 1.f : 0.f;
+        uint4* blk;
         uint4 c0;
-        if (is_query) c0 = make_uint4(bf2(n1, n2), bf2(n3, one), bf2(one, one), 0u);
-        else c0 = make_uint4(bf2(one, one), bf2(one, n1), bf2(n2, n3), 0u);
-        const int64_t t = row / rows_per_tile, i = row % rows_per_tile;
-        uint4* blk = img + (t * (int64_t)tile_stride + (int64_t)block_off) / 16;
-        blk[i] = c0;
-        blk[rows_per_tile + i] = make_uint4(0u, 0u, 0u, 0u);
+        if (is_q) {
+            blk = q_img + (t * (int64_t)g.a_bytes() + (int64_t)g.Dp * 512) / 16;
+            c0 = make_uint4(bf2(n1, n2), bf2(n3, one), bf2(one, one), 0u);
+        } else {
+            blk = ref_img + (t * (int64_t)g.tile_bytes() + (int64_t)g.KS * KNN_STAGE_BYTES) / 16;
+            c0 = make_uint4(bf2(one, one), bf2(one, n1), bf2(n2, n3), 0u);
+        }
+        blk[tid] = c0;
+        blk[rows + tid] = make_uint4(0u, 0u, 0u, 0u);
     }
 }
 
@@ -213,6 +220,10 @@ __device__ __forceinline__ void tmem_ld64(uint32_t taddr, uint32_t (&v)[64]) {
     asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
 
+__device__ __forceinline__ void red_add_shared(uint32_t saddr, uint32_t v) {
+    asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(saddr), "r"(v) : "memory");
+}
+
 __device__ __forceinline__ void stage_f4(uint32_t saddr, float4 v) {
     asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(saddr), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w)
                  : "memory");
@@ -246,12 +257,13 @@ struct KnnSmem {
 template <int MODE>
 __global__ void __launch_bounds__(KNN_THREADS, 1)
     knn_fused_kernel(KnnGeom g, const uint8_t* __restrict__ ref_img, const uint8_t* __restrict__ q_img,
-                     unsigned long long* __restrict__ pool64, float* __restrict__ cand_val, int32_t* __restrict__ cand_idx,
+                     unsigned long long* __restrict__ pool64, int32_t* __restrict__ cnt_out,
                      unsigned long long* __restrict__ qthr, float* __restrict__ dump) {
     constexpr bool DUMP = (MODE == 1);
     constexpr bool PIPE_ONLY = (MODE == 2);
     constexpr bool PROF = (MODE == 3);  // selection + per-warp cycle counters (experiments)
     unsigned long long prof_narrow = 0, prof_wait = 0, prof_chunks = 0, prof_rare = 0, prof_nrare = 0, prof_nnarrow = 0;
+    const unsigned long long prof_t0 = PROF ? clock64() : 0;
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
     const int NS = g.NS;
@@ -273,6 +285,14 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
     const int split = blockIdx.x / g.QT;
     const int t0 = (int)((int64_t)g.ntiles * split / g.S);  // logical tile range of this CTA
     const int t1 = (int)((int64_t)g.ntiles * (split + 1) / g.S);
+    // Cold CTAs (the first wave: no split of their queries has published a bound
+    // yet) first stream their first Fs tiles through the pipeline for a distance
+    // histogram per query (starting bound, see the epilogue), then all t1 - t0.
+    const int Fs = (!DUMP && !PIPE_ONLY && (int)blockIdx.x < g.sample_ctas && g.k <= KNN_BN && g.tstride == 1 &&
+                    t1 - t0 >= 4 * g.sample_tiles && (int64_t)(t0 + g.sample_tiles) * KNN_BN <= g.N)
+                       ? g.sample_tiles
+                       : 0;
+    const int nsteps = Fs + (t1 - t0);
 
     if (warp == 0 && lane == 0) {
         for (int s = 0; s < NS; ++s) {
@@ -305,8 +325,8 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
             mbar_arrive_expect_tx(afull, abytes);
             bulk_g2s(sA, q_img + (size_t)qt * abytes, abytes, afull);
             uint32_t it = 0;
-            for (int ti = t0; ti < t1; ++ti) {
-                const int t = ti * g.tstride;
+            for (int lt = 0; lt < nsteps; ++lt) {
+                const int t = (lt < Fs ? t0 + lt : t0 + lt - Fs) * g.tstride;
                 for (int ks = 0; ks <= g.KS; ++ks, ++it) {
                     const int st = (int)(it % NS);
                     const uint32_t bytes = (ks < g.KS) ? KNN_STAGE_BYTES : KNN_NORM_B_BYTES;
@@ -327,7 +347,7 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
             mbar_wait(afull, 0);
             tc_fence_after();
             uint32_t it = 0;
-            for (int ti = t0, lt = 0; ti < t1; ++ti, ++lt) {
+            for (int lt = 0; lt < nsteps; ++lt) {
                 const int b = lt & 1;
                 mbar_wait(&acce[b], (((uint32_t)lt >> 1) & 1u) ^ 1u);
                 tc_fence_after();
@@ -395,7 +415,9 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
                 unsigned long long* jp = (unsigned long long*)__shfl_sync(kFull, (unsigned long long)pool, j);
                 const int jn = __shfl_sync(kFull, n, j);
                 int nn;
-                const unsigned long long t = (jn <= 32 * kNarrowRegs)
+                const unsigned long long t = (jn <= 256)   ? pool_narrow64<8>(jp, jn, (uint32_t)target, &nn)
+                                             : (jn <= 512) ? pool_narrow64<16>(jp, jn, (uint32_t)target, &nn)
+                                             : (jn <= 32 * kNarrowRegs)
                                                  ? pool_narrow64<kNarrowRegs>(jp, jn, (uint32_t)target, &nn)
                                                  : pool_select64(jp, jn, (uint32_t)target, hist, &nn);
                 if ((int)lane == j) {
@@ -408,8 +430,13 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
             __syncwarp();
         };
 
-        for (int ti = t0, lt = 0; ti < t1; ++ti, ++lt) {
-            const int t = ti * g.tstride;
+        // sample histogram of this lane's query: 64 buckets [lo, hi) in the warp scratch
+        uint32_t* shist = reinterpret_cast<uint32_t*>(wscratch) + lane;
+        const uint32_t shist_s = smem_u32(shist);
+        float s_lo = 0.f, s_hi = -1.f, s_inv = 0.f;
+        for (int lt = 0; lt < nsteps; ++lt) {
+            const bool sampling = lt < Fs;
+            const int t = (sampling ? t0 + lt : t0 + lt - Fs) * g.tstride;
             const int b = lt & 1;
             if (!DUMP && !PIPE_ONLY) {
                 // adopt the tightest bound any split of this query has published
@@ -425,7 +452,7 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
             tc_fence_after();
             const uint32_t taddr = tmem_base + ((uint32_t)(quad * 32) << 16) + (uint32_t)(b * KNN_BN);
             if (!DUMP && !PIPE_ONLY && lt == 0 && g.k <= KNN_BN && (int64_t)t * KNN_BN + KNN_BN <= g.N &&
-                __any_sync(kFull, qvalid && (uint32_t)(T >> 32) == kSentKey)) {
+                (Fs > 0 || __any_sync(kFull, qvalid && (uint32_t)(T >> 32) == kSentKey))) {
                 // Starting bound without a fill phase: the exact k-th smallest distance of
                 // this first (full) tile, by bisection on the bits of the clamped value
                 // (non-negative floats order like their bit patterns), re-reading the
@@ -449,6 +476,61 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
                     if (cnt < (uint32_t)g.k) vb = cand;
                 }
                 if (qvalid) adopt(((unsigned long long)key_of(__uint_as_float(vb)) << 32) | 0x7ffffffeu);
+                if (Fs > 0) {
+                    // histogram range: [max(0, tile minimum), k-th of the tile]
+                    float mn = __int_as_float(0x7f800000);
+#pragma unroll 1
+                    for (int c = 0; c < KNN_BN / KNN_CW; ++c) {
+                        uint32_t v[KNN_CW];
+                        tmem_ld64(taddr + (uint32_t)(c * KNN_CW), v);
+#pragma unroll
+                        for (int j = 0; j < KNN_CW; ++j) mn = fminf(mn, __uint_as_float(v[j]));
+                    }
+                    s_lo = fmaxf(mn, 0.f);
+                    s_hi = __uint_as_float(vb);
+                    // buckets must stay far wider than an ulp (the bound below keeps one
+                    // spare bucket for rounding); otherwise no histogram for this query
+                    if (!(s_hi < __int_as_float(0x7f800000)) || !(s_hi - s_lo > s_hi * 0x1p-10f)) s_hi = -1.f;
+                    s_inv = (s_hi > 0.f) ? 64.f / (s_hi - s_lo) : 0.f;
+#pragma unroll 8
+                    for (int j = 0; j < 64; ++j) shist[j * 32] = 0u;
+                }
+            }
+            if (sampling) {
+                // count this tile's distances <= hi per bucket (NaN fails the test)
+#pragma unroll 1
+                for (int c = 0; c < KNN_BN / KNN_CW; ++c) {
+                    uint32_t v[KNN_CW];
+                    tmem_ld64(taddr + (uint32_t)(c * KNN_CW), v);
+#pragma unroll
+                    for (int j = 0; j < KNN_CW; ++j) {
+                        const float d = __uint_as_float(v[j]);
+                        if (d <= s_hi) {
+                            const int bk = min(max((int)((d - s_lo) * s_inv), 0), 63);
+                            red_add_shared(shist_s + (uint32_t)(bk * 128), 1u);
+                        }
+                    }
+                }
+                if (lt == Fs - 1 && qvalid && s_hi > 0.f) {
+                    // >= k sampled distances lie in buckets <= j, i.e. below lo + (j + 1) w;
+                    // one spare bucket absorbs the rounding of the bucket index
+                    uint32_t cum = 0;
+                    int j = 0;
+                    for (; j < 64; ++j) {
+                        cum += shist[j * 32];
+                        if (cum >= (uint32_t)g.k) break;
+                    }
+                    if (j < 62) {
+                        const float bound = s_lo + (float)(j + 2) * ((s_hi - s_lo) * (1.f / 64.f));
+                        const unsigned long long tb = ((unsigned long long)key_of(bound) << 32) | 0x7ffffffeu;
+                        adopt(tb);
+                        atomicMin(&qthr[q], tb);
+                    }
+                }
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive_cta(&acce[b]);
+                continue;
             }
 #pragma unroll 1
             for (int c = 0; c < KNN_BN / KNN_CW; ++c) {
@@ -515,22 +597,23 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
             __syncwarp();
             if (lane == 0) mbar_arrive_cta(&acce[b]);
         }
-        if (PROF && lane == 0) {
-            unsigned long long* o = reinterpret_cast<unsigned long long*>(dump) + ((size_t)blockIdx.x * 4 + e) * 6;
-            o[0] = prof_narrow; o[1] = prof_wait; o[2] = prof_chunks; o[3] = prof_rare; o[4] = prof_nrare; o[5] = prof_nnarrow;
-        }
+        const unsigned long long prof_t1 = PROF ? clock64() : 0;
         if (!DUMP && !PIPE_ONLY) {
-            // exact top-k of this split for every query, unsorted (ksel_merge sorts)
+            // Narrow every pool to this split's exact top-k; its k-th pair is published
+            // (the bound the later splits and the merge start from).  The pool holds every
+            // pair of this split in the row's top-k (all pairs <= any bound; narrowing keeps
+            // the pool's k smallest); launch_merge_pools gathers the pools' pairs <= the
+            // final published bound and selects the exact top-k of the row.
             narrow_lanes(g.P - g.k, g.k);  // n > k  <=>  n + (P - k) > P
-            if (qvalid) {
-                float* cv = cand_val + ((size_t)split * g.Q + q) * g.k;
-                int32_t* ci = cand_idx + ((size_t)split * g.Q + q) * g.k;
-                for (int x = 0; x < g.k; ++x) {
-                    const bool real = x < n;
-                    const unsigned long long pr = real ? pool[x] : 0ull;
-                    cv[x] = __uint_as_float(real ? bits_of_key((uint32_t)(pr >> 32)) : 0x7fffffffu);
-                    ci[x] = real ? (int32_t)((int64_t)(uint32_t)pr + g.idx_offset) : (int32_t)kSentIdx;
-                }
+            if (qvalid) cnt_out[(size_t)split * g.Q + q] = n;
+        }
+        if (PROF) {
+            __syncwarp();
+            const unsigned long long prof_t2 = clock64();
+            if (lane == 0) {
+                unsigned long long* o = reinterpret_cast<unsigned long long*>(dump) + ((size_t)blockIdx.x * 4 + e) * 8;
+                o[0] = prof_narrow; o[1] = prof_wait; o[2] = prof_chunks; o[3] = prof_rare; o[4] = prof_nrare;
+                o[5] = prof_nnarrow; o[6] = prof_t2 - prof_t1; o[7] = prof_t2 - prof_t0;
             }
         }
     }
@@ -546,16 +629,8 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
 // ---------------------------------------------------------------------------
 static size_t al256(size_t x) { return (x + 255u) & ~(size_t)255u; }
 
-static bool knn_prologue_enabled() {  // experiments: KSEL_KNN_PROLOGUE=1
-    static const bool on = [] {
-        const char* e = std::getenv("KSEL_KNN_PROLOGUE");
-        return e && e[0] == '1';
-    }();
-    return on;
-}
-
 struct KnnWork {
-    size_t ref_img, q_img, pool, cval, cidx, qthr, prof, total;
+    size_t ref_img, q_img, pool, cnt, qthr, prof, total;
 };
 
 static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int64_t idx_offset) {
@@ -581,6 +656,13 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     g.idx_offset = idx_offset;
     g.ntiles = g.NT;
     g.tstride = 1;
+    // first-wave CTAs sample 16 tiles (4096 references) for their starting bound
+    static const int sample_env = [] {
+        const char* e = std::getenv("KSEL_KNN_SAMPLE");  // experiments: tiles sampled (0 = off)
+        return e ? std::atoi(e) : 16;
+    }();
+    g.sample_tiles = sample_env;
+    g.sample_ctas = g.sample_tiles > 0 ? num_sms : 0;
     // reference splits: enough CTAs for the SMs, waves as full as possible, <= 64 lists to merge
     int best = 1;
     double best_cost = 1e30;
@@ -603,10 +685,9 @@ static KnnWork knn_work_layout(const KnnGeom& g) {
     w.ref_img = off; off += al256((size_t)g.NT * g.tile_bytes());
     w.q_img = off;   off += al256((size_t)g.QT * g.a_bytes());
     w.pool = off;    off += al256((size_t)g.S * g.Q * g.P * 8);
-    w.cval = off;    off += al256((size_t)g.S * g.Q * g.k * 4);
-    w.cidx = off;    off += al256((size_t)g.S * g.Q * g.k * 4);
+    w.cnt = off;     off += al256((size_t)g.S * g.Q * 4);
     w.qthr = off;    off += al256((size_t)g.Q * 8);
-    w.prof = off;    off += al256((size_t)g.QT * g.S * 4 * 6 * 8);  // MODE 3 counters
+    w.prof = off;    off += al256((size_t)g.QT * g.S * 4 * 8 * 8);  // MODE 3 counters
     w.total = off;
     return w;
 }
@@ -622,18 +703,7 @@ static cudaError_t knn_run(const float* ref, const float* query, const KnnGeom& 
     uint4* ref_img = reinterpret_cast<uint4*>(work + w.ref_img);
     uint4* q_img = reinterpret_cast<uint4*>(work + w.q_img);
 
-    knn_prep_ref_kernel<<<dim3((unsigned)g.NT, (unsigned)(g.Dp / 8)), KNN_BN, 0, stream>>>(ref, g.N, g.D, g.Dp,
-                                                                                         g.tile_bytes(), ref_img);
-    note_launch();
-    knn_prep_query_kernel<<<dim3((unsigned)g.QT, (unsigned)(g.Dp / 8)), KNN_BM, 0, stream>>>(query, g.Q, g.D, g.Dp,
-                                                                                           q_img);
-    note_launch();
-    const int64_t rpad = (int64_t)g.NT * KNN_BN, qpad = (int64_t)g.QT * KNN_BM;
-    knn_norm_block_kernel<<<(unsigned)((rpad + 7) / 8), 256, 0, stream>>>(
-        ref, g.N, rpad, g.D, KNN_BN, g.tile_bytes(), (size_t)g.KS * KNN_STAGE_BYTES, false, ref_img);
-    note_launch();
-    knn_norm_block_kernel<<<(unsigned)((qpad + 7) / 8), 256, 0, stream>>>(
-        query, g.Q, qpad, g.D, KNN_BM, (size_t)g.a_bytes(), (size_t)g.Dp * 512, true, q_img);
+    knn_prep_kernel<<<(unsigned)(g.NT + g.QT), KNN_PREP_THREADS, 0, stream>>>(ref, query, g, ref_img, q_img);
     note_launch();
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
@@ -645,44 +715,25 @@ static cudaError_t knn_run(const float* ref, const float* query, const KnnGeom& 
         const char* e = std::getenv("KSEL_KNN_MODE");
         return (e && (e[0] == '2' || e[0] == '3')) ? e[0] - '0' : 0;
     }();
-    auto sel_kern = mode_env == 3 ? knn_fused_kernel<3> : knn_fused_kernel<0>;
     auto kern = dump ? knn_fused_kernel<1>
                      : (mode_env == 2 ? knn_fused_kernel<2> : (mode_env == 3 ? knn_fused_kernel<3> : knn_fused_kernel<0>));
     if (!dump && mode_env == 3) dump = reinterpret_cast<float*>(work + w.prof);
     e = ensure_smem_attr(reinterpret_cast<const void*>(kern), smem);
     if (e != cudaSuccess) return e;
-    if (!dump && g.NT >= 256 && knn_prologue_enabled()) {
-        // threshold prologue: exact top-k of every query over 64 reference tiles spread
-        // evenly across the set; each k-th pair is a valid bound for the whole row and is
-        // published in qthr, so the main pass starts filtering at rank ~k*NT/64 instead of
-        // admitting everything until its pools fill (outputs of this pass are discarded)
-        KnnGeom gp = g;
-        gp.ntiles = 64;
-        gp.tstride = g.NT / 64;
-        gp.S = (g.QT >= 148) ? 1 : ((2 * 148 + g.QT - 1) / g.QT > 4 ? 4 : (2 * 148 + g.QT - 1) / g.QT);
-        e = ensure_smem_attr(reinterpret_cast<const void*>(sel_kern), smem);
-        if (e != cudaSuccess) return e;
-        sel_kern<<<(unsigned)(gp.QT * gp.S), KNN_THREADS, smem, stream>>>(
-            gp, reinterpret_cast<const uint8_t*>(ref_img), reinterpret_cast<const uint8_t*>(q_img),
-            reinterpret_cast<unsigned long long*>(work + w.pool),
-            reinterpret_cast<float*>(work + w.cval), reinterpret_cast<int32_t*>(work + w.cidx),
-            reinterpret_cast<unsigned long long*>(work + w.qthr), mode_env == 3 ? dump : nullptr);
-        note_launch();
-        e = cudaGetLastError();
-        if (e != cudaSuccess) return e;
-    }
     const int slot = dump ? -1 : timing_begin(stream);
     kern<<<(unsigned)(g.QT * g.S), KNN_THREADS, smem, stream>>>(
         g, reinterpret_cast<const uint8_t*>(ref_img), reinterpret_cast<const uint8_t*>(q_img),
         reinterpret_cast<unsigned long long*>(work + w.pool),
-        reinterpret_cast<float*>(work + w.cval), reinterpret_cast<int32_t*>(work + w.cidx),
+        reinterpret_cast<int32_t*>(work + w.cnt),
         reinterpret_cast<unsigned long long*>(work + w.qthr), dump);
     note_launch();
     timing_end(slot, stream);
     e = cudaGetLastError();
     if (e != cudaSuccess || (dump && mode_env != 3)) return e;
-    return launch_merge(reinterpret_cast<const float*>(work + w.cval), reinterpret_cast<const int32_t*>(work + w.cidx),
-                        g.Q, g.S, g.k, g.k, out_dist, out_idx, stream);
+    return launch_merge_pools(reinterpret_cast<const unsigned long long*>(work + w.pool), g.P,
+                              reinterpret_cast<const int32_t*>(work + w.cnt), g.S, g.Q,
+                              reinterpret_cast<const unsigned long long*>(work + w.qthr), g.k, g.idx_offset, out_dist,
+                              out_idx, stream);
 }
 
 static int knn_check(const float* ref, const float* query, int64_t N, int64_t Q, int D, int k, int64_t idx_offset) {

@@ -155,6 +155,17 @@ __device__ __noinline__ static int pool_compact(uint32_t* __restrict__ pk, uint3
 }
 
 
+// #{u : rk[u] < cand} for this lane, with four independent partial sums (the
+// bisection steps below are latency-bound: a single add chain over NR compares
+// would dominate them).
+template <int NR>
+__device__ __forceinline__ uint32_t count_lt(const uint32_t (&rk)[NR], uint32_t cand) {
+    uint32_t c[4] = {0u, 0u, 0u, 0u};
+#pragma unroll
+    for (int u = 0; u < NR; ++u) c[u & 3] += (rk[u] < cand) ? 1u : 0u;
+    return (c[0] + c[1]) + (c[2] + c[3]);
+}
+
 // Register-resident narrowing of one pool of n <= 32*NR pairs (global or shared
 // memory): the pool is loaded once (NR pairs per lane), the want-th smallest
 // pair is found by bisection on the key bits with warp-wide counts
@@ -174,15 +185,25 @@ __device__ __noinline__ unsigned long long pool_narrow_regs(uint32_t* __restrict
         rk[u] = (x < n) ? pk[x] : 0xffffffffu;  // generic loads: shared- or global-memory pools
         ri[u] = (x < n) ? pi[x] : 0xffffffffu;
     }
-    // want-th smallest key: the largest v with #{key < v} < want
-    uint32_t vkey = 0;
-#pragma unroll 1
-    for (int b = 31; b >= 0; --b) {
-        const uint32_t cand = vkey | (1u << b);
-        uint32_t c = 0;
+    // want-th smallest key: the largest v with #{key < v} < want (pads are
+    // 0xffffffff: never below); bits above the highest bit where the smallest and
+    // largest key differ are those of the smallest
+    uint32_t kmin = 0xffffffffu, kmax = 0u;
 #pragma unroll
-        for (int u = 0; u < NR; ++u) c += (rk[u] < cand) ? 1u : 0u;  // pads are 0xffffffff: never below
-        if (__reduce_add_sync(kFull, c) < want) vkey = cand;
+    for (int u = 0; u < NR; ++u) {
+        if (u * 32 + (int)lane < n) {
+            kmin = min(kmin, rk[u]);
+            kmax = max(kmax, rk[u]);
+        }
+    }
+    kmin = __reduce_min_sync(kFull, kmin);
+    kmax = __reduce_max_sync(kFull, kmax);
+    const int top = (kmin == kmax) ? -1 : 31 - __clz(kmin ^ kmax);
+    uint32_t vkey = (top < 0) ? kmin : (kmin & ~((2u << top) - 1u));
+#pragma unroll 1
+    for (int b = top; b >= 0; --b) {
+        const uint32_t cand = vkey | (1u << b);
+        if (__reduce_add_sync(kFull, count_lt<NR>(rk, cand)) < want) vkey = cand;
     }
     uint32_t less = 0, eq = 0, mx = 0;
 #pragma unroll
@@ -233,8 +254,9 @@ __device__ __noinline__ unsigned long long pool_narrow_regs(uint32_t* __restrict
 
 // Same as pool_narrow_regs for a pool of packed pairs (key << 32 | idx) in one
 // u64 array; the key bisection starts below the common prefix of the pool's
-// smallest and largest key.
-template <int NR>
+// smallest and largest key.  GLOBAL: the pool is in global memory (L2 loads,
+// __ldcg: other lanes wrote it); otherwise generic loads (shared memory).
+template <int NR, bool GLOBAL = true>
 __device__ __noinline__ unsigned long long pool_narrow64(unsigned long long* __restrict__ pool, int n, uint32_t want,
                                                          int* n_out) {
     const uint32_t lane = lane_id();
@@ -243,7 +265,7 @@ __device__ __noinline__ unsigned long long pool_narrow64(unsigned long long* __r
 #pragma unroll
     for (int u = 0; u < NR; ++u) {
         const int x = u * 32 + (int)lane;
-        r[u] = (x < n) ? __ldcg(pool + x) : 0xffffffffffffffffull;
+        r[u] = (x < n) ? (GLOBAL ? __ldcg(pool + x) : pool[x]) : 0xffffffffffffffffull;
         if (x < n) {
             kmin = min(kmin, (uint32_t)(r[u] >> 32));
             kmax = max(kmax, (uint32_t)(r[u] >> 32));
@@ -255,13 +277,13 @@ __device__ __noinline__ unsigned long long pool_narrow64(unsigned long long* __r
     // highest bit where kmin and kmax differ are those of kmin
     const int top = (kmin == kmax) ? -1 : 31 - __clz(kmin ^ kmax);
     uint32_t vkey = (top < 0) ? kmin : (kmin & ~((2u << top) - 1u));
+    uint32_t hk[NR];  // the key halves (pads: 0xffffffff, never below)
+#pragma unroll
+    for (int u = 0; u < NR; ++u) hk[u] = (uint32_t)(r[u] >> 32);
 #pragma unroll 1
     for (int b = top; b >= 0; --b) {
         const uint32_t cand = vkey | (1u << b);
-        uint32_t c = 0;
-#pragma unroll
-        for (int u = 0; u < NR; ++u) c += ((uint32_t)(r[u] >> 32) < cand) ? 1u : 0u;
-        if (__reduce_add_sync(kFull, c) < want) vkey = cand;
+        if (__reduce_add_sync(kFull, count_lt<NR>(hk, cand)) < want) vkey = cand;
     }
     uint32_t less = 0, eq = 0, mx = 0;
 #pragma unroll

@@ -148,3 +148,34 @@ def test_config4_full_size_sampled_queries(K, oracle_mod, kind):
     torch.cuda.synchronize()
     sample = list(range(32)) + list(range(37, Q, Q // 32))[:32]
     check_knn(oracle_mod, ref.cpu(), qry[sample].cpu(), k, gv[sample], gi[sample], exact=(kind == "knn-S"))
+
+
+_SAMPLED_SCRIPT = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+import paper_conf_ipps_tang0emg15_b200 as K, synth
+kind, N, Q, k = sys.argv[3], int(sys.argv[4]), int(sys.argv[5]), int(sys.argv[6])
+ref = synth.knn_points(kind, 51, 0, N, 128, device="cuda")
+qry = synth.knn_points(kind, 52, 0, Q, 128, device="cuda")
+v, i = K.knn_search(ref, qry, k)
+np.save(sys.argv[2] + "/v.npy", v.cpu().numpy()); np.save(sys.argv[2] + "/i.npy", i.cpu().numpy())
+"""
+
+
+@pytest.mark.parametrize("kind,k", [("knn-U", 100), ("knn-U", 7), ("knn-S", 64), ("knn-U", 256)])
+def test_knn_search_sampled_start(oracle_mod, tmp_path, kind, k):
+    # first-wave CTAs histogram a sample of tiles for their starting bound; force it on a
+    # small problem (KSEL_KNN_SAMPLE=4 tiles) in a fresh process (the setting is read once)
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    N, Q = 50000, 7680  # 60 query tiles x ~12 splits of ~16 tiles
+    env = dict(os.environ, KSEL_KNN_SAMPLE="4")
+    subprocess.run([sys.executable, "-c", _SAMPLED_SCRIPT, root, str(tmp_path), kind, str(N), str(Q), str(k)],
+                   check=True, env=env, timeout=300)
+    gv, gi = np.load(tmp_path / "v.npy"), np.load(tmp_path / "i.npy")
+    ref = synth.knn_points(kind, 51, 0, N, 128)
+    qry = synth.knn_points(kind, 52, 0, Q, 128)
+    sample = list(range(32)) + list(range(40, Q, 29))
+    check_knn(oracle_mod, ref, qry[sample], k, gv[sample], gi[sample], exact=(kind == "knn-S"))
