@@ -33,6 +33,7 @@
 //     share of the top-k); launch_merge_pools (merge.cu) gathers the pairs below
 //     the final shared bound and selects and sorts the exact top-k -- the
 //     divide-and-merge of L243.
+#include <algorithm>
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
@@ -53,7 +54,11 @@ constexpr int KNN_KS = 32;                               // dims per pipeline st
 constexpr int KNN_STAGE_BYTES = 2 * KNN_KS * KNN_BN * 2;  // hi + lo bf16 = 32 KB
 constexpr int KNN_NORM_B_BYTES = 16 * KNN_BN * 2;         // norm block of a reference tile (hi only)
 constexpr int KNN_NORM_A_BYTES = 16 * KNN_BM * 2;         // norm block of a query tile
-constexpr int KNN_THREADS = 192;                         // 6 warps
+// epilogue warps EW: 4 (one per TMEM lane quadrant, all 256 columns of a tile) or
+// 8 (two per quadrant, 128 columns each); + producer + MMA issuer
+constexpr int KNN_MAX_EW = 8;
+__host__ __device__ constexpr int knn_threads(int ew) { return 64 + 32 * ew; }
+constexpr int KNN_SB = 32;                                // sampling histogram buckets
 constexpr int KNN_CW = 64;                                // accumulator columns per epilogue step
 constexpr int KNN_MAX_D = 256;
 constexpr int kNarrowRegs = 40;  // register-resident narrowing: pools of <= 1280 pairs
@@ -69,6 +74,8 @@ struct KnnGeom {
     int ntiles, tstride; // this launch visits reference tiles i * tstride, i < ntiles (split over S)
     int sample_tiles;    // cold CTAs (blockIdx < sample_ctas) first histogram this many tiles
     int sample_ctas;
+    int halves;          // column halves per tile (EW / 4): pools per split
+    int pcap;            // pool fill that triggers a narrowing before a tile (<= P)
     __host__ __device__ size_t tile_bytes() const { return (size_t)KS * KNN_STAGE_BYTES + KNN_NORM_B_BYTES; }
     __host__ __device__ int a_bytes() const { return Dp * 512 + KNN_NORM_A_BYTES; }
 };
@@ -220,31 +227,41 @@ __device__ __forceinline__ void tmem_ld64(uint32_t taddr, uint32_t (&v)[64]) {
     asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
 
-__device__ __forceinline__ void red_add_shared(uint32_t saddr, uint32_t v) {
-    asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(saddr), "r"(v) : "memory");
+// Split form of tmem_ld32: issue without waiting, and a wait that names the
+// destination registers (so no use of them can be scheduled above it).  Lets
+// the epilogue process one 32-column chunk while the next one is in flight.
+__device__ __forceinline__ void tmem_ld32_issue(uint32_t taddr, uint32_t (&v)[32]) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
+        "%15, %16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31}, [%32];"
+        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+          "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15]),
+          "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]),
+          "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
+        : "r"(taddr));
 }
-
-__device__ __forceinline__ void stage_f4(uint32_t saddr, float4 v) {
-    asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(saddr), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w)
+__device__ __forceinline__ void tmem_wait32(uint32_t (&v)[32]) {
+    asm volatile("tcgen05.wait::ld.sync.aligned;"
+                 : "+r"(v[0]), "+r"(v[1]), "+r"(v[2]), "+r"(v[3]), "+r"(v[4]), "+r"(v[5]), "+r"(v[6]), "+r"(v[7]),
+                   "+r"(v[8]), "+r"(v[9]), "+r"(v[10]), "+r"(v[11]), "+r"(v[12]), "+r"(v[13]), "+r"(v[14]),
+                   "+r"(v[15]), "+r"(v[16]), "+r"(v[17]), "+r"(v[18]), "+r"(v[19]), "+r"(v[20]), "+r"(v[21]),
+                   "+r"(v[22]), "+r"(v[23]), "+r"(v[24]), "+r"(v[25]), "+r"(v[26]), "+r"(v[27]), "+r"(v[28]),
+                   "+r"(v[29]), "+r"(v[30]), "+r"(v[31])
+                 :
                  : "memory");
 }
-__device__ __forceinline__ float4 lds_f4(uint32_t saddr) {
-    float4 v;
-    asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(saddr));
-    return v;
+
+__device__ __forceinline__ void red_add_shared(uint32_t saddr, uint32_t v) {
+    asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(saddr), "r"(v) : "memory");
 }
 
 // ---------------------------------------------------------------------------
 // the fused kernel
 // ---------------------------------------------------------------------------
 struct KnnSmem {
-    static constexpr int kHistBytes = 4 * 256 * 4;
-    static constexpr int kStageRow = KNN_CW + 4;  // floats per lane row (16-B aligned, conflict-free STS.128 phases)
-    // per epilogue warp: the rare-path staging rows (32 x kStageRow floats) OR, between
-    // chunks, one query's pool while it is narrowed (kNarrowCap pairs)
-    static constexpr int kNarrowCap = 1152;
-    static constexpr int kWarpScratch = (kNarrowCap * 8 > 32 * kStageRow * 4) ? kNarrowCap * 8 : 32 * kStageRow * 4;
-    static constexpr int kDStageBytes = 4 * kWarpScratch;
+    static constexpr int kHistBytes = KNN_MAX_EW * 256 * 4;        // radix histogram per warp (pool_select64)
+    static constexpr int kWarpScratch = KNN_SB * 32 * 4;      // per warp: sampling histogram, one per lane
+    static constexpr int kDStageBytes = KNN_MAX_EW * kWarpScratch;
     __host__ __device__ static int total(const KnnGeom& g) {
         return 1024 /*align slack*/ + g.a_bytes() + g.NS * KNN_STAGE_BYTES + kHistBytes + kDStageBytes +
                (2 * g.NS + 5) * 8 + 16;
@@ -254,15 +271,17 @@ struct KnnSmem {
 // MODE 0: selection (knn_search); 1: write every distance (knn_distances);
 // 2: pipeline only -- the epilogue reads the accumulators and drops them
 // (experiments: isolates the TMA + MMA + TMEM pipeline from the selection).
-template <int MODE>
-__global__ void __launch_bounds__(KNN_THREADS, 1)
+template <int MODE, int EW>
+__global__ void __launch_bounds__(knn_threads(EW), 1)
     knn_fused_kernel(KnnGeom g, const uint8_t* __restrict__ ref_img, const uint8_t* __restrict__ q_img,
                      unsigned long long* __restrict__ pool64, int32_t* __restrict__ cnt_out,
                      unsigned long long* __restrict__ qthr, float* __restrict__ dump) {
+    constexpr int HALVES = EW / 4;
+    constexpr int WCOLS = KNN_BN / HALVES;  // columns of each tile this epilogue warp scans
     constexpr bool DUMP = (MODE == 1);
     constexpr bool PIPE_ONLY = (MODE == 2);
     constexpr bool PROF = (MODE == 3);  // selection + per-warp cycle counters (experiments)
-    unsigned long long prof_narrow = 0, prof_wait = 0, prof_chunks = 0, prof_rare = 0, prof_nrare = 0, prof_nnarrow = 0;
+    unsigned long long prof_app = 0, prof_narrow = 0, prof_wait = 0, prof_chunks = 0, prof_rare = 0, prof_nrare = 0, prof_nnarrow = 0;
     const unsigned long long prof_t0 = PROF ? clock64() : 0;
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
@@ -301,7 +320,7 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
         }
         for (int b = 0; b < 2; ++b) {
             mbar_init(&accf[b], 1);
-            mbar_init(&acce[b], 4);
+            mbar_init(&acce[b], EW);
         }
         mbar_init(afull, 1);
         fence_mbar_init();
@@ -383,16 +402,18 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
         }
     } else {
         // ===== epilogue: one thread per query =====
-        const int e = warp - 2;                   // 0..3
+        const int e = warp - 2;                   // 0..EW-1
         const int quad = warp & 3;                // TMEM lane quadrant this warp may access
+        const int half = e >> 2;                  // columns [half * WCOLS, (half + 1) * WCOLS) of every tile
         const int row = quad * 32 + (int)lane;    // query row within the tile
         const int64_t q = (int64_t)qt * KNN_BM + row;
         const bool qvalid = q < g.Q;
         uint32_t* hist = hist_all + e * 256;
         uint8_t* wscratch = reinterpret_cast<uint8_t*>(dstage_all) + e * KnnSmem::kWarpScratch;
-        const uint32_t dst = smem_u32(wscratch + (int)lane * KnnSmem::kStageRow * 4);
         // this query's candidate pool: packed pairs (key << 32 | reference row)
-        unsigned long long* pool = pool64 + ((size_t)split * g.Q + (qvalid ? q : 0)) * g.P;
+        // (each (split, half) keeps its own pools: S * HALVES lists per query for the merge)
+        const size_t list = (size_t)split * HALVES + half;
+        unsigned long long* pool = pool64 + (list * g.Q + (qvalid ? q : 0)) * g.P;
         unsigned long long T = kSentPair;  // running bound on the k-th pair
         float tv = 0.f;
         bool fast = false;                 // T below +Inf: the fp32 compare d <= tv pre-filters
@@ -406,8 +427,8 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
             }
         };
         // warp-cooperative narrowing of every lane whose pool cannot take `room` more pairs
-        auto narrow_lanes = [&](int room, int target) {
-            uint32_t need = __ballot_sync(kFull, qvalid && n + room > g.P);
+        auto narrow_lanes = [&](int room, int target, int cap) {
+            uint32_t need = __ballot_sync(kFull, qvalid && n + room > cap);
             while (need) {
                 if (PROF) prof_nnarrow++;
                 const int j = __ffs(need) - 1;
@@ -434,15 +455,18 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
         uint32_t* shist = reinterpret_cast<uint32_t*>(wscratch) + lane;
         const uint32_t shist_s = smem_u32(shist);
         float s_lo = 0.f, s_hi = -1.f, s_inv = 0.f;
+        unsigned long long thr_next = (qvalid && !DUMP && !PIPE_ONLY) ? __ldcg(&qthr[q]) : kSentPair;
         for (int lt = 0; lt < nsteps; ++lt) {
             const bool sampling = lt < Fs;
             const int t = (sampling ? t0 + lt : t0 + lt - Fs) * g.tstride;
             const int b = lt & 1;
             if (!DUMP && !PIPE_ONLY) {
-                // adopt the tightest bound any split of this query has published
-                if (qvalid) adopt(__ldcg(&qthr[q]));
+                // adopt the tightest bound any split of this query had published when the
+                // previous tile started (the load's latency hides behind that tile)
+                adopt(thr_next);
+                if (qvalid) thr_next = __ldcg(&qthr[q]);
                 const unsigned long long c0 = PROF ? clock64() : 0;
-                narrow_lanes(KNN_BN, g.k);
+                narrow_lanes(WCOLS, g.k, g.pcap);
                 if (PROF) prof_narrow += clock64() - c0;
             }
             const unsigned long long cw0 = PROF ? clock64() : 0;
@@ -491,37 +515,37 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
                     // buckets must stay far wider than an ulp (the bound below keeps one
                     // spare bucket for rounding); otherwise no histogram for this query
                     if (!(s_hi < __int_as_float(0x7f800000)) || !(s_hi - s_lo > s_hi * 0x1p-10f)) s_hi = -1.f;
-                    s_inv = (s_hi > 0.f) ? 64.f / (s_hi - s_lo) : 0.f;
+                    s_inv = (s_hi > 0.f) ? (float)KNN_SB / (s_hi - s_lo) : 0.f;
 #pragma unroll 8
-                    for (int j = 0; j < 64; ++j) shist[j * 32] = 0u;
+                    for (int j = 0; j < KNN_SB; ++j) shist[j * 32] = 0u;
                 }
             }
             if (sampling) {
-                // count this tile's distances <= hi per bucket (NaN fails the test)
+                // count this warp's half-tile distances <= hi per bucket (NaN fails the test)
 #pragma unroll 1
-                for (int c = 0; c < KNN_BN / KNN_CW; ++c) {
+                for (int c = half * (WCOLS / KNN_CW); c < (half + 1) * (WCOLS / KNN_CW); ++c) {
                     uint32_t v[KNN_CW];
                     tmem_ld64(taddr + (uint32_t)(c * KNN_CW), v);
 #pragma unroll
                     for (int j = 0; j < KNN_CW; ++j) {
                         const float d = __uint_as_float(v[j]);
                         if (d <= s_hi) {
-                            const int bk = min(max((int)((d - s_lo) * s_inv), 0), 63);
+                            const int bk = min(max((int)((d - s_lo) * s_inv), 0), KNN_SB - 1);
                             red_add_shared(shist_s + (uint32_t)(bk * 128), 1u);
                         }
                     }
                 }
                 if (lt == Fs - 1 && qvalid && s_hi > 0.f) {
-                    // >= k sampled distances lie in buckets <= j, i.e. below lo + (j + 1) w;
+                    // >= k of this warp's sampled distances lie in buckets <= j, i.e. below lo + (j + 1) w;
                     // one spare bucket absorbs the rounding of the bucket index
                     uint32_t cum = 0;
                     int j = 0;
-                    for (; j < 64; ++j) {
+                    for (; j < KNN_SB; ++j) {
                         cum += shist[j * 32];
                         if (cum >= (uint32_t)g.k) break;
                     }
-                    if (j < 62) {
-                        const float bound = s_lo + (float)(j + 2) * ((s_hi - s_lo) * (1.f / 64.f));
+                    if (j < KNN_SB - 2) {
+                        const float bound = s_lo + (float)(j + 2) * ((s_hi - s_lo) * (1.f / KNN_SB));
                         const unsigned long long tb = ((unsigned long long)key_of(bound) << 32) | 0x7ffffffeu;
                         adopt(tb);
                         atomicMin(&qthr[q], tb);
@@ -532,8 +556,69 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
                 if (lane == 0) mbar_arrive_cta(&acce[b]);
                 continue;
             }
+            if constexpr (!DUMP && !PIPE_ONLY) {
+                // Selection scan of the tile: 32 columns per TMEM load, the next load in
+                // flight while the current chunk is filtered.  Per chunk: min of each
+                // 4-column group, one warp vote of the chunk minimum against each lane's
+                // bound; on a hit, one warp-uniform vote per group, and only groups some
+                // lane needs are visited (candidates appended, predicated, from registers).
+                const uint32_t colt = (uint32_t)t * KNN_BN;  // N < 2^31
+                const int nlim = (int)min((int64_t)KNN_BN, g.N - (int64_t)colt);  // valid columns of the tile
+                auto scan32 = [&](const uint32_t(&v)[32], int c0) {
+                    float gmn[8];
+#pragma unroll
+                    for (int j = 0; j < 8; ++j)
+                        gmn[j] = fminf(fminf(__uint_as_float(v[4 * j]), __uint_as_float(v[4 * j + 1])),
+                                       fminf(__uint_as_float(v[4 * j + 2]), __uint_as_float(v[4 * j + 3])));
+                    const float mn = fminf(fminf(fminf(gmn[0], gmn[1]), fminf(gmn[2], gmn[3])),
+                                           fminf(fminf(gmn[4], gmn[5]), fminf(gmn[6], gmn[7])));
+                    if (!__any_sync(kFull, qvalid && (!fast || mn <= tv))) return;
+                    const unsigned long long cr0 = PROF ? clock64() : 0;
+                    // rare path: each lane visits only its own candidate groups (a divergent
+                    // loop of max-over-lanes length); the group's 4 values are picked from the
+                    // registers by a 3-level select tree (registers cannot be indexed
+                    // dynamically).  An element with d == tv and a larger index than T's is a
+                    // harmless extra pool entry (narrowing applies the exact pair order).
+                    uint32_t gm = 0;
+#pragma unroll
+                    for (int u = 0; u < 8; ++u) gm |= (uint32_t)(!fast || gmn[u] <= tv) << u;
+                    if (!qvalid) gm = 0;
+                    while (gm) {
+                        const int u = __ffs(gm) - 1;
+                        gm &= gm - 1u;
+                        const bool b0 = u & 1, b1 = u & 2, b2 = u & 4;
+                        const int cu = c0 + 4 * u;
+#pragma unroll
+                        for (int i = 0; i < 4; ++i) {
+                            const uint32_t a0 = b0 ? v[4 + i] : v[i], a1 = b0 ? v[12 + i] : v[8 + i];
+                            const uint32_t a2 = b0 ? v[20 + i] : v[16 + i], a3 = b0 ? v[28 + i] : v[24 + i];
+                            const uint32_t c01 = b1 ? a1 : a0, c23 = b1 ? a3 : a2;
+                            const float x = __uint_as_float(b2 ? c23 : c01);
+                            if (cu + i < nlim && (!fast || x <= tv)) {
+                                const float dc = (x < 0.f) ? 0.f : x;  // clamp, NaN propagates
+                                pool[n++] = ((unsigned long long)key_of(dc) << 32) | (colt + (uint32_t)(cu + i));
+                                if (PROF) prof_app++;
+                            }
+                        }
+                    }
+                    if (PROF) { prof_rare += clock64() - cr0; prof_nrare++; }
+                };
+                uint32_t va[32], vb[32];
+                tmem_ld32_issue(taddr + (uint32_t)(half * WCOLS), va);
+                tmem_wait32(va);
+                const int cb = half * (WCOLS / 32), ce = cb + WCOLS / 32;
 #pragma unroll 1
-            for (int c = 0; c < KNN_BN / KNN_CW; ++c) {
+                for (int c = cb; c < ce; c += 2) {
+                    tmem_ld32_issue(taddr + (uint32_t)((c + 1) * 32), vb);
+                    scan32(va, c * 32);
+                    tmem_wait32(vb);
+                    if (c + 2 < ce) tmem_ld32_issue(taddr + (uint32_t)((c + 2) * 32), va);
+                    scan32(vb, (c + 1) * 32);
+                    if (c + 2 < ce) tmem_wait32(va);
+                }
+            }
+#pragma unroll 1
+            for (int c = half * (WCOLS / KNN_CW); c < ((DUMP || PIPE_ONLY) ? (half + 1) * (WCOLS / KNN_CW) : 0); ++c) {
                 uint32_t v[KNN_CW];
                 tmem_ld64(taddr + (uint32_t)(c * KNN_CW), v);
                 if (PIPE_ONLY) {
@@ -541,56 +626,13 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
                     continue;
                 }
                 const int64_t col0 = (int64_t)t * KNN_BN + c * KNN_CW;
-                // the accumulator is d = |q|^2 + |r|^2 - 2 q.r (clamped at 0 only where it is kept)
-                constexpr int NGR = KNN_CW / 4;  // 4-column groups
-                float d[KNN_CW], gmin[NGR];
+                // (knn_distances) the accumulator is d = |q|^2 + |r|^2 - 2 q.r; clamped at 0
+                float d[KNN_CW];
 #pragma unroll
-                for (int j = 0; j < KNN_CW; j += 4) {
-                    d[j + 0] = __uint_as_float(v[j + 0]);
-                    d[j + 1] = __uint_as_float(v[j + 1]);
-                    d[j + 2] = __uint_as_float(v[j + 2]);
-                    d[j + 3] = __uint_as_float(v[j + 3]);
-                    gmin[j >> 2] = fminf(fminf(d[j], d[j + 1]), fminf(d[j + 2], d[j + 3]));
-                }
-                if (DUMP) {
-                    if (qvalid)
-                        for (int j = 0; j < KNN_CW; ++j)
-                            if (col0 + j < g.N) dump[q * g.N + col0 + j] = (d[j] < 0.f) ? 0.f : d[j];
-                    continue;
-                }
-                // thresholds are >= 0, so negative (pre-clamp) values pass as they should;
-                // the vote is warp-uniform: every lane takes part whatever its mode
-                float mn = gmin[0];
-#pragma unroll
-                for (int u = 1; u < NGR; ++u) mn = fminf(mn, gmin[u]);
-                if (!__any_sync(kFull, qvalid && (!fast || mn <= tv))) continue;
-                const unsigned long long cr0 = PROF ? clock64() : 0;
-                // rare path.  The pair test against T is left to narrowing: an element with
-                // d == tv and a larger index is a harmless extra pool entry.
-                uint32_t gm = 0;
-#pragma unroll
-                for (int u = 0; u < NGR; ++u) gm |= (uint32_t)(!fast || gmin[u] <= tv) << u;
-                if (!qvalid) gm = 0;
-                // stage the lane's values and visit only its own candidate groups
-#pragma unroll
-                for (int u = 0; u < NGR; ++u)
-                    stage_f4(dst + (uint32_t)(u * 16), make_float4(d[4 * u], d[4 * u + 1], d[4 * u + 2], d[4 * u + 3]));
-                while (gm) {
-                    const int u = __ffs(gm) - 1;
-                    gm &= gm - 1u;
-                    const float4 d4 = lds_f4(dst + (uint32_t)(u * 16));
-                    const int64_t cu = col0 + 4 * u;
-                    // up to 4 candidates, appended branch-free (predicated)
-                    const float dd[4] = {d4.x, d4.y, d4.z, d4.w};
-#pragma unroll
-                    for (int i = 0; i < 4; ++i) {
-                        if ((cu + i < g.N) && (!fast || dd[i] <= tv)) {
-                            const float dc = (dd[i] < 0.f) ? 0.f : dd[i];  // clamp, NaN propagates
-                            pool[n++] = ((unsigned long long)key_of(dc) << 32) | (uint32_t)(cu + i);
-                        }
-                    }
-                }
-                if (PROF) { prof_rare += clock64() - cr0; prof_nrare++; }
+                for (int j = 0; j < KNN_CW; ++j) d[j] = __uint_as_float(v[j]);
+                if (qvalid)
+                    for (int j = 0; j < KNN_CW; ++j)
+                        if (col0 + j < g.N) dump[q * g.N + col0 + j] = (d[j] < 0.f) ? 0.f : d[j];
             }
             if (PROF) prof_chunks += clock64() - cc0;
             tc_fence_before();
@@ -604,16 +646,16 @@ __global__ void __launch_bounds__(KNN_THREADS, 1)
             // pair of this split in the row's top-k (all pairs <= any bound; narrowing keeps
             // the pool's k smallest); launch_merge_pools gathers the pools' pairs <= the
             // final published bound and selects the exact top-k of the row.
-            narrow_lanes(g.P - g.k, g.k);  // n > k  <=>  n + (P - k) > P
-            if (qvalid) cnt_out[(size_t)split * g.Q + q] = n;
+            narrow_lanes(g.P - g.k, g.k, g.P);  // n > k  <=>  n + (P - k) > P
+            if (qvalid) cnt_out[list * g.Q + q] = n;
         }
         if (PROF) {
             __syncwarp();
             const unsigned long long prof_t2 = clock64();
             if (lane == 0) {
-                unsigned long long* o = reinterpret_cast<unsigned long long*>(dump) + ((size_t)blockIdx.x * 4 + e) * 8;
+                unsigned long long* o = reinterpret_cast<unsigned long long*>(dump) + ((size_t)blockIdx.x * EW + e) * 16;
                 o[0] = prof_narrow; o[1] = prof_wait; o[2] = prof_chunks; o[3] = prof_rare; o[4] = prof_nrare;
-                o[5] = prof_nnarrow; o[6] = prof_t2 - prof_t1; o[7] = prof_t2 - prof_t0;
+                o[5] = prof_nnarrow; o[6] = prof_t2 - prof_t1; o[7] = prof_t2 - prof_t0; o[8] = prof_app;
             }
         }
     }
@@ -654,6 +696,19 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     g.NS = (kMaxSmemPerBlock - fixed) / KNN_STAGE_BYTES;
     if (g.NS > 6) g.NS = 6;
     g.idx_offset = idx_offset;
+    static const int ew_env = [] {
+        const char* e = std::getenv("KSEL_KNN_EW");  // experiments: 4 or 8 epilogue warps
+        return (e && std::atoi(e) == 8) ? 8 : 4;
+    }();
+    g.halves = ew_env / 4;
+    static const int cap_env = [] {
+        const char* e = std::getenv("KSEL_KNN_SOFTCAP");  // experiments: narrow early (pool fill cap)
+        return e ? std::atoi(e) : 0;
+    }();
+    // narrow before a pool reaches P when queues are small: the bound then tracks the
+    // k-th of what has been seen more closely in cold CTAs (measured: 512 for k <= 128)
+    const int cap = cap_env > 0 ? cap_env : (kk <= 128 ? 512 : g.P);
+    g.pcap = std::max(kk + 32 + KNN_BN / g.halves, std::min(g.P, cap));
     g.ntiles = g.NT;
     g.tstride = 1;
     // first-wave CTAs sample 16 tiles (4096 references) for their starting bound
@@ -684,10 +739,10 @@ static KnnWork knn_work_layout(const KnnGeom& g) {
     size_t off = 0;
     w.ref_img = off; off += al256((size_t)g.NT * g.tile_bytes());
     w.q_img = off;   off += al256((size_t)g.QT * g.a_bytes());
-    w.pool = off;    off += al256((size_t)g.S * g.Q * g.P * 8);
-    w.cnt = off;     off += al256((size_t)g.S * g.Q * 4);
+    w.pool = off;    off += al256((size_t)2 * g.S * g.Q * g.P * 8);  // 2 lists (column halves) per split
+    w.cnt = off;     off += al256((size_t)2 * g.S * g.Q * 4);
     w.qthr = off;    off += al256((size_t)g.Q * 8);
-    w.prof = off;    off += al256((size_t)g.QT * g.S * 4 * 8 * 8);  // MODE 3 counters
+    w.prof = off;    off += al256((size_t)g.QT * g.S * KNN_MAX_EW * 16 * 8);  // MODE 3 counters
     w.total = off;
     return w;
 }
@@ -715,13 +770,16 @@ static cudaError_t knn_run(const float* ref, const float* query, const KnnGeom& 
         const char* e = std::getenv("KSEL_KNN_MODE");
         return (e && (e[0] == '2' || e[0] == '3')) ? e[0] - '0' : 0;
     }();
-    auto kern = dump ? knn_fused_kernel<1>
-                     : (mode_env == 2 ? knn_fused_kernel<2> : (mode_env == 3 ? knn_fused_kernel<3> : knn_fused_kernel<0>));
+    const bool ew8 = g.halves == 2;
+    auto kern = dump ? (ew8 ? knn_fused_kernel<1, 8> : knn_fused_kernel<1, 4>)
+              : mode_env == 2 ? (ew8 ? knn_fused_kernel<2, 8> : knn_fused_kernel<2, 4>)
+              : mode_env == 3 ? (ew8 ? knn_fused_kernel<3, 8> : knn_fused_kernel<3, 4>)
+                              : (ew8 ? knn_fused_kernel<0, 8> : knn_fused_kernel<0, 4>);
     if (!dump && mode_env == 3) dump = reinterpret_cast<float*>(work + w.prof);
     e = ensure_smem_attr(reinterpret_cast<const void*>(kern), smem);
     if (e != cudaSuccess) return e;
     const int slot = dump ? -1 : timing_begin(stream);
-    kern<<<(unsigned)(g.QT * g.S), KNN_THREADS, smem, stream>>>(
+    kern<<<(unsigned)(g.QT * g.S), knn_threads(4 * g.halves), smem, stream>>>(
         g, reinterpret_cast<const uint8_t*>(ref_img), reinterpret_cast<const uint8_t*>(q_img),
         reinterpret_cast<unsigned long long*>(work + w.pool),
         reinterpret_cast<int32_t*>(work + w.cnt),
@@ -731,7 +789,7 @@ static cudaError_t knn_run(const float* ref, const float* query, const KnnGeom& 
     e = cudaGetLastError();
     if (e != cudaSuccess || (dump && mode_env != 3)) return e;
     return launch_merge_pools(reinterpret_cast<const unsigned long long*>(work + w.pool), g.P,
-                              reinterpret_cast<const int32_t*>(work + w.cnt), g.S, g.Q,
+                              reinterpret_cast<const int32_t*>(work + w.cnt), g.halves * g.S, g.Q,
                               reinterpret_cast<const unsigned long long*>(work + w.qthr), g.k, g.idx_offset, out_dist,
                               out_idx, stream);
 }

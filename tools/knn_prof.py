@@ -29,16 +29,17 @@ for s_ in range(1, min(NT, 64) + 1):
         best, best_cost = s_, cost
 S = best
 raw = ws.cpu().numpy()
-sz = QT * S * 4 * 8 * 8
+EW = 8 if os.environ.get('KSEL_KNN_EW') == '8' else 4
+sz = QT * S * 8 * 16 * 8
 szp = (sz + 255) // 256 * 256
-arr = raw[raw.size - szp: raw.size - szp + sz].view(np.uint64).reshape(QT * S, 4, 8)
+arr = raw[raw.size - szp: raw.size - szp + sz].view(np.uint64)[:QT * S * EW * 16].reshape(QT * S, EW, 16)[:, :, :9]
 print("S =", S)
-names = ["narrow", "wait_accf", "chunks", "rare", "n_rare", "n_narrow", "final", "total"]
-tot = arr.reshape(-1, 8).astype(np.float64)
+names = ["narrow", "wait_accf", "chunks", "rare", "n_rare", "n_narrow", "final", "total", "appends"]
+tot = arr.reshape(-1, 9).astype(np.float64)
 print("CTAs x warps:", tot.shape[0])
 for i, nm in enumerate(names):
     print("%-10s mean %.3g  max %.3g" % (nm, tot[:, i].mean(), tot[:, i].max()))
 split = np.arange(arr.shape[0]) // QT
 for s in range(split.max() + 1):
-    m = arr[split == s].reshape(-1, 8).astype(np.float64).mean(axis=0)
+    m = arr[split == s].reshape(-1, 9).astype(np.float64).mean(axis=0)
     print("split %d: " % s + "  ".join("%s %.3g" % (nm, v) for nm, v in zip(names, m)))
