@@ -364,11 +364,14 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads)
             }
             bool go = true;
             if (fast) {
-                // one compare per lane: the sub-step minimum (fminf skips NaN, which is never a candidate)
+                // one compare per lane: the sub-step minimum (fminf skips NaN, which is never a
+                // candidate).  Past the bound's index (col0 >= Ti) an element equal to the bound
+                // value cannot precede the bound pair, so the test is strict: rows with heavy
+                // ties then skip the sub-steps that only hold copies of the bound value.
                 float mn = x[0];
 #pragma unroll
                 for (int j = 1; j < NS; ++j) mn = fminf(mn, x[j]);
-                go = __any_sync(kFull, mn <= tv);
+                go = __any_sync(kFull, col0 >= Ti ? mn < tv : mn <= tv);
             }
             if (go) exact(srcf, (uint32_t)g, len, col0, x);
         }
