@@ -18,6 +18,8 @@ through ctypes.  Each function cites the passage it follows:
 * :func:`knn_dist` -- PAPER.md L13 (Euclidean distance phase); reading R9:
   squared L2 accumulated in double, one rounding to fp32.
 * :func:`knn`      -- knn_dist followed by select.
+* :func:`knn_graph` -- PAPER.md L635-L639 (k-NN graph construction, the target of
+  QMS [9]): per point, the k nearest other points (self excluded).
 
 Pins (tests/test_oracle_pins.py): brute-force rank counting, numpy stable
 argsort, the north-star invariants, the paper's worked examples
@@ -59,7 +61,9 @@ def _load():
         lib.oracle_merge.argtypes = [p, p, i64, i64, i64, i64, p, p]
         lib.oracle_knn_dist.argtypes = [p, p, i64, i64, i64, p, i32]
         lib.oracle_knn.argtypes = [p, p, i64, i64, i64, i64, i64, p, p, p, i32]
-        for f in (lib.oracle_select, lib.oracle_merge, lib.oracle_knn_dist, lib.oracle_knn):
+        lib.oracle_knn_graph.argtypes = [p, i64, i64, i64, p, p, p, i32]
+        for f in (lib.oracle_select, lib.oracle_merge, lib.oracle_knn_dist, lib.oracle_knn,
+                  lib.oracle_knn_graph):
             f.restype = ctypes.c_int
         _lib = lib
     return _lib
@@ -136,4 +140,20 @@ def knn(ref, query, k: int, idx_offset: int = 0, nthreads: int | None = None):
                             _ptr(ov), _ptr(oi), nthreads or default_threads())
     if rc:
         raise ValueError("oracle_knn failed (%d)" % rc)
+    return ov, oi
+
+
+def knn_graph(points, k: int, nthreads: int | None = None):
+    """(squared distances, indices) of the k nearest OTHER points of every point."""
+    x = np.ascontiguousarray(points, dtype=np.float32)
+    if x.ndim != 2:
+        raise ValueError("points must be N x D")
+    N, D = x.shape
+    scratch = np.empty((N, N), np.float32)
+    ov = np.empty((N, k), np.float32)
+    oi = np.empty((N, k), np.int32)
+    rc = _load().oracle_knn_graph(_ptr(x), N, D, k, _ptr(scratch), _ptr(ov), _ptr(oi),
+                                  nthreads or default_threads())
+    if rc:
+        raise ValueError("oracle_knn_graph failed (%d)" % rc)
     return ov, oi

@@ -220,3 +220,34 @@ int oracle_knn(const float* ref, const float* query, int64_t N, int64_t Q, int64
     for (int64_t t = 0; t < Q * k; ++t) out_idx[t] = (int32_t)(out_idx[t] + idx_offset);
     return 0;
 }
+
+/* oracle_knn_graph: the k-nearest-neighbour graph of one point set (the k-NNG
+ * construction QMS [9] targets): for every point
+ * i of points[N][D], the k smallest (d(i, j), j) over j != i -- distances as in
+ * oracle_knn_dist, order as in oracle_select.  Definition, written out: the
+ * pairs of row i without j == i, sorted, first k.  Requires 1 <= k <= N - 1.
+ * scratch_dist must hold N*N floats. */
+int oracle_knn_graph(const float* points, int64_t N, int64_t D, int64_t k, float* scratch_dist,
+                     float* out_dist, int32_t* out_idx, int nthreads) {
+    if (!points || !scratch_dist || !out_dist || !out_idx || N < 2 || k < 1 || k > N - 1) return 2;
+    int err = oracle_knn_dist(points, points, N, N, D, scratch_dist, nthreads);
+    if (err) return err;
+    pair_t* scratch = (pair_t*)malloc(sizeof(pair_t) * (size_t)N);
+    if (!scratch) return 1;
+    for (int64_t i = 0; i < N; ++i) {
+        int64_t n = 0;
+        for (int64_t j = 0; j < N; ++j) {
+            if (j == i) continue;
+            scratch[n].v = scratch_dist[i * N + j];
+            scratch[n].i = (int32_t)j;
+            ++n;
+        }
+        qsort(scratch, (size_t)n, sizeof(pair_t), pair_cmp);
+        for (int64_t t = 0; t < k; ++t) {
+            out_dist[i * k + t] = scratch[t].v;
+            out_idx[i * k + t] = scratch[t].i;
+        }
+    }
+    free(scratch);
+    return 0;
+}

@@ -292,3 +292,29 @@ def test_knn_self_match_first(oracle_mod):
     assert list(di[:, 0]) == [1017, 1250, 1499]
     assert list(dv[:, 0]) == [0.0, 0.0, 0.0]
     assert np.all(np.diff(dv, axis=1) >= 0)
+
+
+def test_knn_graph_brute_force_integers(oracle_mod):
+    """k-NN graph (QMS [9]): exact Python integer distances,
+    self excluded, ties (duplicate points) by lower index."""
+    rng = random.Random(11)
+    for trial in range(40):
+        N, D = rng.randint(2, 9), rng.randint(1, 4)
+        pts = [[rng.randint(0, 3) for _ in range(D)] for _ in range(N)]
+        k = rng.randint(1, N - 1)
+        ov, oi = oracle_mod.knn_graph(np.array(pts, np.float32), k)
+        for i in range(N):
+            pairs = sorted((sum((a - b) ** 2 for a, b in zip(pts[i], pts[j])), j) for j in range(N) if j != i)[:k]
+            assert oi[i].tolist() == [j for _, j in pairs], (trial, i)
+            assert ov[i].tolist() == [float(d) for d, _ in pairs], (trial, i)
+
+
+def test_knn_graph_equals_knn_without_self(oracle_mod):
+    x = synth.knn_points("knn-U", 21, 0, 60, 16).numpy()
+    ov, oi = oracle_mod.knn_graph(x, 7)
+    for i in (0, 17, 59):
+        rest = np.delete(x, i, axis=0)
+        rv, ri = oracle_mod.knn(rest, x[i:i + 1], 7)
+        ri = ri[0] + (ri[0] >= i)  # back to indices of x
+        assert np.array_equal(oi[i], ri) and np.array_equal(ov[i].view(np.uint32), rv[0].view(np.uint32))
+        assert i not in oi[i].tolist()
