@@ -127,6 +127,23 @@ KSEL_API int knn_search(const float* ref, const float* query, int64_t N, int64_t
                float* out_dist, int32_t* out_idx, int64_t idx_offset, void* d_work,
                size_t work_bytes, void* stream);
 
+/* knn_graph -- the k-nearest-neighbour graph of one point set (k-NNG
+ * construction, the workload of QMS [9]): for
+ * every point i of points[N][D], its k nearest OTHER points, i.e. the k
+ * lexicographically smallest (d(i, j), j) over j != i, ascending.  Computed as
+ * knn_search(points, points, k + 1) followed by removing i from row i (when i is
+ * not among the k + 1 -- more than k duplicates of i with lower indices -- the
+ * first k are the answer), so distances, ties and accuracy are those of
+ * knn_search.
+ *   points   device, N x D fp32 row-major (read only)
+ *   out_dist device, N x k fp32 (squared L2); out_idx device, N x k int32
+ *   d_work   device workspace of >= knn_graph_workspace(N, D, k) bytes
+ * Errors: KSEL_ERR_INVALID_ARG for N < 2, k < 1, k > N - 1, null pointers or a
+ * short workspace; KSEL_ERR_UNSUPPORTED for k + 1 > 1024 or D > 256. */
+KSEL_API size_t knn_graph_workspace(int64_t N, int D, int k);
+KSEL_API int knn_graph(const float* points, int64_t N, int D, int k, float* out_dist, int32_t* out_idx,
+                       void* d_work, size_t work_bytes, void* stream);
+
 /* knn_distances -- DIAGNOSTIC (not the hot path): the same tcgen05 distance
  * computation as knn_search, but every d(q, r) is written to out[Q][N] (device,
  * fp32) instead of being selected.  Lets tests pin the tensor-core distance

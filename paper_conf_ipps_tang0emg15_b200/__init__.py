@@ -11,6 +11,7 @@ Entry points (same names as the C ABI):
 * :func:`ksel_select_host` -- the same on host buffers (end-to-end path).
 * :func:`ksel_merge`       -- top-k of the union of S sorted candidate lists.
 * :func:`knn_search`       -- fused distance + selection brute-force k-NN.
+* :func:`knn_graph`        -- k-NN graph of one point set (self excluded).
 """
 from __future__ import annotations
 
@@ -38,6 +39,10 @@ _lib.ksel_merge.argtypes = [_p, _p, _i64, _i32, _i32, _i32, _p, _p, _p]
 _lib.knn_search_workspace.argtypes = [_i64, _i64, _i32, _i32]
 _lib.knn_search_workspace.restype = _sz
 _lib.knn_search.argtypes = [_p, _p, _i64, _i64, _i32, _i32, _p, _p, _i64, _p, _sz, _p]
+_lib.knn_graph_workspace.argtypes = [_i64, _i32, _i32]
+_lib.knn_graph_workspace.restype = _sz
+_lib.knn_graph.argtypes = [_p, _i64, _i32, _i32, _p, _p, _p, _sz, _p]
+_lib.knn_graph.restype = ctypes.c_int
 _lib.knn_distances_workspace.argtypes = [_i64, _i64, _i32]
 _lib.knn_distances_workspace.restype = _sz
 _lib.knn_distances.argtypes = [_p, _p, _i64, _i64, _i32, _p, _p, _sz, _p]
@@ -55,7 +60,7 @@ for _f in (_lib.ksel_select, _lib.ksel_select_config, _lib.ksel_select_host, _li
 KSEL_MAX_K = 1024
 ALGO_AUTO, ALGO_QUEUE, ALGO_POOL = 0, 1, 2
 EXPORTS = ("ksel_select", "ksel_select_config", "ksel_select_host_workspace", "ksel_select_host", "ksel_merge",
-           "knn_search_workspace", "knn_search", "knn_distances_workspace", "knn_distances", "ksel_timing_enable", "ksel_timing_collect", "ksel_strerror",
+           "knn_search_workspace", "knn_search", "knn_graph_workspace", "knn_graph", "knn_distances_workspace", "knn_distances", "ksel_timing_enable", "ksel_timing_collect", "ksel_strerror",
            "ksel_version", "ksel_launch_count")
 
 
@@ -203,6 +208,30 @@ def knn_search(ref: torch.Tensor, query: torch.Tensor, k: int, idx_offset: int =
         _check("knn_search", _lib.knn_search(ref.data_ptr(), query.data_ptr(), N, Q, D, k,
                                              out_dist.data_ptr(), out_idx.data_ptr(), idx_offset,
                                              wptr, wlen, _stream(ref.device)))
+    return out_dist, out_idx
+
+
+def knn_graph_workspace(N: int, D: int, k: int) -> int:
+    return int(_lib.knn_graph_workspace(N, D, k))
+
+
+def knn_graph(points: torch.Tensor, k: int, out_dist: torch.Tensor | None = None,
+              out_idx: torch.Tensor | None = None, workspace: torch.Tensor | None = None):
+    """k nearest OTHER points of every point (k-NN graph); points [N, D]."""
+    _dev_f32(points, "points", 2)
+    N, D = points.shape
+    if out_dist is None:
+        out_dist = torch.empty((N, k), dtype=torch.float32, device=points.device)
+    if out_idx is None:
+        out_idx = torch.empty((N, k), dtype=torch.int32, device=points.device)
+    need = knn_graph_workspace(N, D, k)
+    if workspace is None and need > 0:
+        workspace = torch.empty(need, dtype=torch.uint8, device=points.device)
+    wptr = workspace.data_ptr() if workspace is not None else 0
+    wlen = workspace.numel() if workspace is not None else 0
+    with torch.cuda.device(points.device):
+        _check("knn_graph", _lib.knn_graph(points.data_ptr(), N, D, k, out_dist.data_ptr(), out_idx.data_ptr(),
+                                           wptr, wlen, _stream(points.device)))
     return out_dist, out_idx
 
 

@@ -804,6 +804,30 @@ static int knn_check(const float* ref, const float* query, int64_t N, int64_t Q,
     return KSEL_OK;
 }
 
+// knn_graph: row i of knn_search(points, points, k + 1) without i.  One warp per
+// row: find i among the k + 1 indices (ballot), copy the others in order.
+__global__ void __launch_bounds__(256)
+    knn_drop_self_kernel(const float* __restrict__ tv, const int32_t* __restrict__ ti, int64_t N, int k,
+                         float* __restrict__ ov, int32_t* __restrict__ oi) {
+    const int64_t row = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
+    const uint32_t lane = lane_id();
+    if (row >= N) return;
+    const int k1 = k + 1;
+    const float* rv = tv + row * k1;
+    const int32_t* ri = ti + row * k1;
+    int pos = k1;  // position of the point itself (k1: absent)
+    for (int base = 0; base < k1; base += 32) {
+        const int e = base + (int)lane;
+        const uint32_t m = __ballot_sync(kFull, e < k1 && ri[e] == (int32_t)row);
+        if (m) { pos = base + __ffs(m) - 1; break; }
+    }
+    for (int e = (int)lane; e < k; e += 32) {
+        const int src = e < pos ? e : e + 1;
+        ov[row * k + e] = rv[src];
+        oi[row * k + e] = ri[src];
+    }
+}
+
 }  // namespace ksel
 
 using namespace ksel;
@@ -829,6 +853,36 @@ int knn_search(const float* ref, const float* query, int64_t N, int64_t Q, int D
     cudaError_t e = knn_run(ref, query, g, static_cast<uint8_t*>(d_work), out_dist, out_idx, nullptr,
                             (cudaStream_t)stream);
     return e == cudaSuccess ? KSEL_OK : KSEL_ERR_CUDA;
+}
+
+size_t knn_graph_workspace(int64_t N, int D, int k) {
+    if (N < 2 || k < 1 || k > N - 1 || k + 1 > KSEL_MAX_K) return 0;
+    const size_t base = knn_search_workspace(N, N, D, k + 1);
+    if (base == 0) return 0;
+    return al256(base) + 2 * al256((size_t)N * (k + 1) * 4);
+}
+
+int knn_graph(const float* points, int64_t N, int D, int k, float* out_dist, int32_t* out_idx, void* d_work,
+              size_t work_bytes, void* stream) {
+    if (!points || !out_dist || !out_idx || N < 2 || k < 1 || k > N - 1) return KSEL_ERR_INVALID_ARG;
+    int st = knn_check(points, points, N, N, D, k + 1, 0);
+    if (st) return st;
+    if (!d_work) return KSEL_ERR_INVALID_ARG;
+    DevInfo di;
+    st = current_device_info(&di);
+    if (st) return st;
+    const KnnGeom g = knn_geometry(N, N, D, k + 1, di.sms, 0);
+    const size_t base = al256(knn_work_layout(g).total);
+    const size_t tmp = al256((size_t)N * (k + 1) * 4);
+    if (work_bytes < base + 2 * tmp) return KSEL_ERR_INVALID_ARG;
+    uint8_t* w = static_cast<uint8_t*>(d_work);
+    float* tv = reinterpret_cast<float*>(w + base);
+    int32_t* ti = reinterpret_cast<int32_t*>(w + base + tmp);
+    cudaError_t e = knn_run(points, points, g, w, tv, ti, nullptr, (cudaStream_t)stream);
+    if (e != cudaSuccess) return KSEL_ERR_CUDA;
+    knn_drop_self_kernel<<<(unsigned)((N + 7) / 8), 256, 0, (cudaStream_t)stream>>>(tv, ti, N, k, out_dist, out_idx);
+    note_launch();
+    return cudaGetLastError() == cudaSuccess ? KSEL_OK : KSEL_ERR_CUDA;
 }
 
 size_t knn_distances_workspace(int64_t N, int64_t Q, int D) { return knn_search_workspace(N, Q, D, 1); }

@@ -322,17 +322,32 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads)
         }
         nreal = __reduce_add_sync(kFull, nreal);
         if (nreal >= (uint32_t)k) {
-            uint32_t vkey = 0;
+            // Bisection on the key bits below the common prefix of the smallest and
+            // largest real key, stopped at bit kLow: the k-th key then lies in
+            // [vkey, vkey + 2^kLow), so vkey | (2^kLow - 1) bounds it (>= k keys are
+            // <= it; looser by < 2^-15 relative for floats, for ~40% fewer steps).
+            constexpr int kLow = 8;
+            uint32_t kmin = 0xffffffffu, kmax = 0u;
+#pragma unroll
+            for (int j = 0; j < NB * CH / 128 * 4; ++j) {
+                kmin = min(kmin, keys[j]);  // (pads of a short chunk are 0xffffffff: only widen the range)
+                kmax = max(kmax, keys[j]);
+            }
+            kmin = __reduce_min_sync(kFull, kmin);
+            kmax = __reduce_max_sync(kFull, kmax);
+            const int top = (kmin == kmax) ? -1 : 31 - __clz(kmin ^ kmax);
+            uint32_t vkey = (top < 0) ? kmin : (kmin & ~((2u << top) - 1u));
 #pragma unroll 1
-            for (int bit = 31; bit >= 0; --bit) {
+            for (int bit = top; bit >= kLow; --bit) {
                 const uint32_t cand = vkey | (1u << bit);
                 uint32_t c = 0;
 #pragma unroll
                 for (int j = 0; j < NB * CH / 128 * 4; ++j) c += (keys[j] < cand) ? 1u : 0u;
                 if (__reduce_add_sync(kFull, c) < (uint32_t)k) vkey = cand;
             }
-            tighten(vkey, 0x7ffffffeu);
-            if (WPR > 1 && lane == 0) atomicMin(grp_thr, ((unsigned long long)vkey << 32) | 0x7ffffffeu);
+            const uint32_t bkey = (top >= kLow) ? (vkey | ((1u << kLow) - 1u)) : kmax;
+            tighten(bkey, 0x7ffffffeu);
+            if (WPR > 1 && lane == 0) atomicMin(grp_thr, ((unsigned long long)bkey << 32) | 0x7ffffffeu);
         }
     }
 

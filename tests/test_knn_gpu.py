@@ -41,13 +41,15 @@ def tol_pairs(q, r, d_ora):
     return 1e-4 * d_ora + 3 * 2.0 ** -16 * absdot + (D + 2) * 2.0 ** -24 * ((q * q).sum() + (r * r).sum(axis=1))
 
 
-def check_knn(oracle_mod, ref, qry, k, gv, gi, idx_offset=0, exact=False):
+def check_knn(oracle_mod, ref, qry, k, gv, gi, idx_offset=0, exact=False, oracle_out=None, rows=None):
+    """oracle_out: precomputed (ov, oi) (e.g. the k-NN graph oracle); rows: global row id of
+    each query for the k-NN graph (its own index must not appear)."""
     ref = ref.numpy() if torch.is_tensor(ref) else ref
     qry = qry.numpy() if torch.is_tensor(qry) else qry
     gv = gv.cpu().numpy() if torch.is_tensor(gv) else gv
     gi = gi.cpu().numpy() if torch.is_tensor(gi) else gi
     N, D = ref.shape
-    ov, oi = oracle_mod.knn(ref, qry, k, idx_offset=idx_offset)
+    ov, oi = oracle_out if oracle_out is not None else oracle_mod.knn(ref, qry, k, idx_offset=idx_offset)
     if exact:
         assert np.array_equal(gi, oi)
         assert np.array_equal(gv.view(np.uint32), ov.view(np.uint32))
@@ -56,6 +58,8 @@ def check_knn(oracle_mod, ref, qry, k, gv, gi, idx_offset=0, exact=False):
     for q in range(qry.shape[0]):
         idx = gi[q].astype(np.int64) - idx_offset
         assert len(set(idx.tolist())) == k and idx.min() >= 0 and idx.max() < N
+        if rows is not None:
+            assert rows[q] not in idx.tolist()
         # sorted by its own (d, idx)
         for t in range(k - 1):
             assert gv[q][t] < gv[q][t + 1] or (gv[q][t] == gv[q][t + 1] and gi[q][t] < gi[q][t + 1])
@@ -179,3 +183,66 @@ def test_knn_search_sampled_start(oracle_mod, tmp_path, kind, k):
     qry = synth.knn_points(kind, 52, 0, Q, 128)
     sample = list(range(32)) + list(range(40, Q, 29))
     check_knn(oracle_mod, ref, qry[sample], k, gv[sample], gi[sample], exact=(kind == "knn-S"))
+
+
+_EW8_SCRIPT = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+import paper_conf_ipps_tang0emg15_b200 as K, synth
+kind, N, Q, k = sys.argv[3], int(sys.argv[4]), int(sys.argv[5]), int(sys.argv[6])
+ref = synth.knn_points(kind, 61, 0, N, 128, device="cuda")
+qry = synth.knn_points(kind, 62, 0, Q, 128, device="cuda")
+v, i = K.knn_search(ref, qry, k)
+np.save(sys.argv[2] + "/v.npy", v.cpu().numpy()); np.save(sys.argv[2] + "/i.npy", i.cpu().numpy())
+"""
+
+
+@pytest.mark.parametrize("kind,k", [("knn-U", 100), ("knn-S", 32), ("knn-U", 512)])
+def test_knn_search_eight_epilogue_warps(oracle_mod, tmp_path, kind, k):
+    # the 8-epilogue-warp variant (two warps per TMEM lane quadrant, 128 columns each,
+    # 2 S pool lists per query) in a fresh process (KSEL_KNN_EW is read once)
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    N, Q = 40000, 2000
+    env = dict(os.environ, KSEL_KNN_EW="8")
+    subprocess.run([sys.executable, "-c", _EW8_SCRIPT, root, str(tmp_path), kind, str(N), str(Q), str(k)],
+                   check=True, env=env, timeout=300)
+    gv, gi = np.load(tmp_path / "v.npy"), np.load(tmp_path / "i.npy")
+    ref = synth.knn_points(kind, 61, 0, N, 128)
+    qry = synth.knn_points(kind, 62, 0, Q, 128)
+    sample = list(range(24)) + list(range(50, Q, 47))
+    check_knn(oracle_mod, ref, qry[sample], k, gv[sample], gi[sample], exact=(kind == "knn-S"))
+
+
+@pytest.mark.parametrize("kind,N,D,k", [("knn-S", 700, 128, 16), ("knn-U", 900, 64, 10), ("knn-U", 2, 5, 1),
+                                        ("knn-U", 333, 3, 332), ("knn-S", 1500, 96, 100)])
+def test_knn_graph_vs_oracle(K, oracle_mod, kind, N, D, k):
+    """k-NN graph (QMS [9]): knn_search(points, points, k+1)
+    minus the point itself, against the graph oracle."""
+    x = synth.knn_points(kind, 71, 0, N, D)
+    gv, gi = K.knn_graph(x.cuda(), k)
+    check_knn(oracle_mod, x, x, k, gv, gi, exact=(kind == "knn-S"),
+              oracle_out=oracle_mod.knn_graph(x.numpy(), k), rows=list(range(N)))
+
+
+def test_knn_graph_duplicates(K, oracle_mod):
+    # many exact duplicates: rows whose point has > k duplicates of lower index do not
+    # see themselves among the k + 1 and keep the first k; integer data -> bit-exact
+    base = synth.knn_points("knn-S", 72, 0, 40, 12)
+    x = base[torch.arange(400) % 40].contiguous()
+    gv, gi = K.knn_graph(x.cuda(), 6)
+    ov, oi = oracle_mod.knn_graph(x.numpy(), 6)
+    assert np.array_equal(gi.cpu().numpy(), oi)
+    assert np.array_equal(gv.cpu().numpy().view(np.uint32), ov.view(np.uint32))
+    assert not np.any(gi.cpu().numpy() == np.arange(400)[:, None])
+
+
+def test_knn_graph_invalid(K):
+    x = torch.rand(10, 8, device="cuda")
+    with pytest.raises(K.KselError):
+        K.knn_graph(x, 10)  # k > N - 1
+    with pytest.raises(K.KselError) as e:
+        K.knn_graph(torch.rand(2000, 8, device="cuda"), 1024)  # k + 1 > 1024
+    assert e.value.status == 2
