@@ -328,6 +328,26 @@ __device__ __noinline__ unsigned long long pool_narrow64(unsigned long long* __r
     return T;
 }
 
+// Visit pool[0..n) in batches of 8 loads per lane (8 L2 requests in flight
+// before any use: the passes below are latency-bound otherwise, since the
+// compiler cannot hoist a global load above a shared-memory atomic of the
+// previous element); f(v) on every valid entry.
+template <typename F>
+__device__ __forceinline__ void pool_scan64(const unsigned long long* __restrict__ pool, int n, uint32_t lane, F f) {
+#pragma unroll 1
+    for (int base = 0; base < n; base += 256) {
+        unsigned long long v[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            const int e = base + j * 32 + (int)lane;
+            v[j] = (e < n) ? __ldcg(pool + e) : 0ull;
+        }
+#pragma unroll
+        for (int j = 0; j < 8; ++j)
+            if (base + j * 32 + (int)lane < n) f(v[j]);
+    }
+}
+
 // Radix select for large packed-pair pools (key << 32 | idx, any memory): the
 // want-th smallest pair by MSD 8-bit digits of the key, starting below the
 // common prefix of the pool's smallest and largest key (distances share their
@@ -338,11 +358,11 @@ __device__ __noinline__ static unsigned long long pool_select64(unsigned long lo
                                                                int* n_out) {
     const uint32_t lane = lane_id();
     uint32_t kmin = 0xffffffffu, kmax = 0u;
-    for (int e = (int)lane; e < n; e += 32) {
-        const uint32_t kk = (uint32_t)(__ldcg(pool + e) >> 32);
+    pool_scan64(pool, n, lane, [&](unsigned long long v) {
+        const uint32_t kk = (uint32_t)(v >> 32);
         kmin = min(kmin, kk);
         kmax = max(kmax, kk);
-    }
+    });
     kmin = __reduce_min_sync(kFull, kmin);
     kmax = __reduce_max_sync(kFull, kmax);
     int hi = (kmin == kmax) ? -1 : 31 - __clz(kmin ^ kmax);
@@ -355,12 +375,11 @@ __device__ __noinline__ static unsigned long long pool_select64(unsigned long lo
 #pragma unroll
         for (int j = 0; j < 8; ++j) hist[j * 32 + lane] = 0u;
         __syncwarp();
-#pragma unroll 4
-        for (int e = (int)lane; e < n; e += 32) {
-            const uint32_t kk = (uint32_t)(__ldcg(pool + e) >> 32);
+        pool_scan64(pool, n, lane, [&](unsigned long long v) {
+            const uint32_t kk = (uint32_t)(v >> 32);
             const bool sel = (hi == 31) || ((kk ^ prefix) >> (hi + 1)) == 0u;
             if (sel) atomicAdd(&hist[hist_slot((kk >> lo) & dmask)], 1u);
-        }
+        });
         __syncwarp();
         const uint32_t d = hist_find(hist, lane, want, cnt);
         prefix |= d << lo;
@@ -371,10 +390,9 @@ __device__ __noinline__ static unsigned long long pool_select64(unsigned long lo
     uint32_t vidx;
     if (cnt == want) {
         uint32_t m = 0;
-        for (int e = (int)lane; e < n; e += 32) {
-            const unsigned long long v = __ldcg(pool + e);
+        pool_scan64(pool, n, lane, [&](unsigned long long v) {
             if ((uint32_t)(v >> 32) == vkey) m = max(m, (uint32_t)v);
-        }
+        });
         vidx = __reduce_max_sync(kFull, m);
     } else {
         uint32_t ip = 0;
@@ -384,13 +402,12 @@ __device__ __noinline__ static unsigned long long pool_select64(unsigned long lo
 #pragma unroll
             for (int j = 0; j < 8; ++j) hist[j * 32 + lane] = 0u;
             __syncwarp();
-            for (int e = (int)lane; e < n; e += 32) {
-                const unsigned long long v = __ldcg(pool + e);
-                if ((uint32_t)(v >> 32) != vkey) continue;
+            pool_scan64(pool, n, lane, [&](unsigned long long v) {
+                if ((uint32_t)(v >> 32) != vkey) return;
                 const uint32_t id = (uint32_t)v;
                 const bool sel = (pass == 0) || ((id ^ ip) >> (shift + 8)) == 0u;
                 if (sel) atomicAdd(&hist[hist_slot((id >> shift) & 255u)], 1u);
-            }
+            });
             __syncwarp();
             const uint32_t d = hist_find(hist, lane, want, cnt);
             ip |= d << shift;
@@ -399,17 +416,26 @@ __device__ __noinline__ static unsigned long long pool_select64(unsigned long lo
         vidx = ip;
     }
     const unsigned long long T = ((unsigned long long)vkey << 32) | vidx;
-    // in-place compaction (reads of a 32-wide slab precede its writes)
+    // in-place compaction, 8 slabs of 32 per batch: every read of a batch precedes its
+    // writes, and writes never pass the batch's first slab (w <= base)
     const uint32_t lt = lanemask_lt();
     int w = 0;
-    for (int base = 0; base < n; base += 32) {
-        const int e = base + (int)lane;
-        const unsigned long long v = (e < n) ? __ldcg(pool + e) : ~0ull;
-        const bool keep = e < n && v <= T;
-        const uint32_t bal = __ballot_sync(kFull, keep);
+#pragma unroll 1
+    for (int base = 0; base < n; base += 256) {
+        unsigned long long v[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            const int e = base + j * 32 + (int)lane;
+            v[j] = (e < n) ? __ldcg(pool + e) : ~0ull;
+        }
         __syncwarp();
-        if (keep) pool[w + __popc(bal & lt)] = v;
-        w += __popc(bal);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            const bool keep = base + j * 32 + (int)lane < n && v[j] <= T;
+            const uint32_t bal = __ballot_sync(kFull, keep);
+            if (keep) pool[w + __popc(bal & lt)] = v[j];
+            w += __popc(bal);
+        }
     }
     __syncwarp();
     *n_out = w;
