@@ -68,6 +68,22 @@ typedef enum {
 KSEL_API int ksel_select(const float* dist, int64_t Q, int64_t N, int k, float* out_val,
                 int32_t* out_idx, void* stream);
 
+/* ksel_select_ex -- ksel_select with a caller-provided device workspace, which
+ * lets few long rows use the whole GPU (split rows): when Q is below
+ * the SM count, every row is cut into S equal segments (S * Q <= #SMs, each
+ * >= max(32768, 64 k') elements), each segment's top-k is selected by its own
+ * CTA (row-global indices), and a second selection over each row's S*k
+ * candidates merges them -- the divide-and-merge of PAPER.md L243 (ref. [18]);
+ * ties there fall in index order, so the result is identical to ksel_select's.
+ *   d_work  device workspace of >= ksel_select_workspace(Q, N, k) bytes (the
+ *           segment lists), not overlapping the inputs/outputs; when that size
+ *           is 0 (enough rows) or d_work is NULL, this is ksel_select.
+ * Errors as ksel_select; a non-NULL workspace that is too small or overlaps ->
+ * KSEL_ERR_INVALID_ARG. */
+KSEL_API size_t ksel_select_workspace(int64_t Q, int64_t N, int k);
+KSEL_API int ksel_select_ex(const float* dist, int64_t Q, int64_t N, int k, float* out_val, int32_t* out_idx,
+                            void* d_work, size_t work_bytes, void* stream);
+
 /* ksel_select_config -- ksel_select with the kernel variant fixed (ablation /
  * tuning; same result bits for every variant):
  *   algo           KSEL_ALGO_AUTO (0), KSEL_ALGO_QUEUE (1): candidates merged into a

@@ -32,6 +32,10 @@ _lib = ctypes.CDLL(LIB_PATH)
 _p, _i64, _i32, _sz = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int, ctypes.c_size_t
 _lib.ksel_select.argtypes = [_p, _i64, _i64, _i32, _p, _p, _p]
 _lib.ksel_select_config.argtypes = [_p, _i64, _i64, _i32, _p, _p, _i32, _i32, _p]
+_lib.ksel_select_workspace.argtypes = [_i64, _i64, _i32]
+_lib.ksel_select_workspace.restype = _sz
+_lib.ksel_select_ex.argtypes = [_p, _i64, _i64, _i32, _p, _p, _p, _sz, _p]
+_lib.ksel_select_ex.restype = ctypes.c_int
 _lib.ksel_select_host_workspace.argtypes = [_i64, _i32]
 _lib.ksel_select_host_workspace.restype = _sz
 _lib.ksel_select_host.argtypes = [_p, _i64, _i64, _i32, _p, _p, _p, _sz, _p]
@@ -59,7 +63,7 @@ for _f in (_lib.ksel_select, _lib.ksel_select_config, _lib.ksel_select_host, _li
 
 KSEL_MAX_K = 1024
 ALGO_AUTO, ALGO_QUEUE, ALGO_POOL = 0, 1, 2
-EXPORTS = ("ksel_select", "ksel_select_config", "ksel_select_host_workspace", "ksel_select_host", "ksel_merge",
+EXPORTS = ("ksel_select", "ksel_select_workspace", "ksel_select_ex", "ksel_select_config", "ksel_select_host_workspace", "ksel_select_host", "ksel_merge",
            "knn_search_workspace", "knn_search", "knn_graph_workspace", "knn_graph", "knn_distances_workspace", "knn_distances", "ksel_timing_enable", "ksel_timing_collect", "ksel_strerror",
            "ksel_version", "ksel_launch_count")
 
@@ -111,13 +115,21 @@ def _stream(device) -> int:
     return torch.cuda.current_stream(device).cuda_stream
 
 
+def ksel_select_workspace(Q: int, N: int, k: int) -> int:
+    return int(_lib.ksel_select_workspace(Q, N, k))
+
+
 def ksel_select(dist: torch.Tensor, k: int, out_val: torch.Tensor | None = None,
-                out_idx: torch.Tensor | None = None, algo: int = ALGO_AUTO, warps_per_row: int = 0):
+                out_idx: torch.Tensor | None = None, algo: int = ALGO_AUTO, warps_per_row: int = 0,
+                workspace: torch.Tensor | None = None, split_rows: bool = True):
     """k smallest (value, index) pairs per row of ``dist`` [Q, N], ascending.
 
     Returns (values float32 [Q, k] with the input bits, indices int32 [Q, k]).
     Enqueued on the current stream; asynchronous.  ``algo``/``warps_per_row``
-    pin the kernel variant (ksel_select_config); defaults pick automatically."""
+    pin the kernel variant (ksel_select_config); defaults pick automatically.
+    With the defaults, few long rows go through ksel_select_ex (split rows) with
+    ``workspace`` (allocated here when None and needed); ``split_rows=False``
+    forces the one-CTA-per-row path."""
     _dev_f32(dist, "dist", 2)
     Q, N = dist.shape
     if out_val is None:
@@ -125,7 +137,13 @@ def ksel_select(dist: torch.Tensor, k: int, out_val: torch.Tensor | None = None,
     if out_idx is None:
         out_idx = torch.empty((Q, k), dtype=torch.int32, device=dist.device)
     with torch.cuda.device(dist.device):
-        if algo == ALGO_AUTO and warps_per_row == 0:
+        need = ksel_select_workspace(Q, N, k) if (algo == ALGO_AUTO and warps_per_row == 0 and split_rows) else 0
+        if need > 0:
+            if workspace is None:
+                workspace = torch.empty(need, dtype=torch.uint8, device=dist.device)
+            st = _lib.ksel_select_ex(dist.data_ptr(), Q, N, k, out_val.data_ptr(), out_idx.data_ptr(),
+                                     workspace.data_ptr(), workspace.numel(), _stream(dist.device))
+        elif algo == ALGO_AUTO and warps_per_row == 0:
             st = _lib.ksel_select(dist.data_ptr(), Q, N, k, out_val.data_ptr(), out_idx.data_ptr(),
                                   _stream(dist.device))
         else:

@@ -4,6 +4,7 @@
 // the host-buffer (end-to-end) pipeline.  No torch types, no allocation on the
 // device paths, no stream synchronisation except in ksel_select_host.
 #include <atomic>
+#include <algorithm>
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
@@ -98,6 +99,8 @@ int current_device_info(DevInfo* out) {
     if (out->major != 10) return KSEL_ERR_NO_DEVICE;  // built for sm_100a only
     return KSEL_OK;
 }
+
+static size_t al256(size_t x) { return (x + 255u) & ~(size_t)255u; }
 
 static bool overlaps(const void* a, size_t na, const void* b, size_t nb) {
     const uintptr_t x = reinterpret_cast<uintptr_t>(a), y = reinterpret_cast<uintptr_t>(b);
@@ -194,6 +197,101 @@ int ksel_select(const float* dist, int64_t Q, int64_t N, int k, float* out_val, 
     return ksel_select_config(dist, Q, N, k, out_val, out_idx, KSEL_ALGO_AUTO, 0, stream);
 }
 
+// ---------------------------------------------------------------------------
+// split rows: few rows cannot fill the GPU with row parallelism
+// (a row lives in one CTA of <= 8 warps), so each row is cut into S segments and
+// every segment selects its own top-k (the pool kernel on Q*S virtual rows,
+// row-global indices).  The S sorted lists of a row are contiguous ([Q][S][k]),
+// so the divide-and-merge (ref. [18]) is one more selection over
+// that row of S*k candidates: ties in it fall in position order, which is the
+// index order (segments and lists are index-ordered), so the top-k by (value,
+// position) is the top-k by (value, index); a gather maps positions to indices.
+// ---------------------------------------------------------------------------
+struct SplitPlan {
+    int S = 1;
+    int64_t seg_len = 0;
+};
+
+static SplitPlan split_plan(int64_t Q, int64_t N, int k, int sms) {
+    SplitPlan p;
+    if (Q >= sms) return p;  // a row per SM at least: the direct path streams at full rate
+    const int kp = k <= 32 ? 32 : k <= 64 ? 64 : k <= 128 ? 128 : k <= 256 ? 256 : k <= 512 ? 512 : 1024;
+    const int64_t min_seg = std::max<int64_t>(32768, 64 * (int64_t)kp);  // each segment >> its k
+    // one virtual row per SM at most: each CTA (<= 8 warps, deep ring) then runs in a
+    // single wave -- a second, partial wave would double the time
+    int64_t S = (int64_t)sms / Q;
+    S = std::min<int64_t>(S, N / min_seg);
+    if (S < 2) return p;
+    p.S = (int)S;
+    // equal segments (no alignment rounding: unaligned segment heads are handled in
+    // the kernel); the last one holds N - (S-1)*ceil(N/S) >= N/S - S + 1 >> k elements
+    p.seg_len = (N + S - 1) / S;
+    return p;
+}
+
+static size_t split_workspace(const SplitPlan& p, int64_t Q, int k) {
+    if (p.S < 2) return 0;
+    return 2 * al256((size_t)p.S * (size_t)Q * (size_t)k * 4u) + al256((size_t)Q * (size_t)k * 4u);
+}
+
+// out_idx[q][j] = lidx[q][pos[q][j]] (row q of lidx holds S*k indices)
+__global__ void split_gather_idx_kernel(const int32_t* __restrict__ lidx, const int32_t* __restrict__ pos,
+                                        int64_t Q, int64_t Sk, int k, int32_t* __restrict__ out_idx) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= Q * (int64_t)k) return;
+    const int64_t q = t / k;
+    out_idx[t] = lidx[q * Sk + pos[t]];
+}
+
+size_t ksel_select_workspace(int64_t Q, int64_t N, int k) {
+    if (Q < 1 || N < 1 || k < 1 || k > N || k > KSEL_MAX_K) return 0;
+    DevInfo di;
+    if (current_device_info(&di) != KSEL_OK) return 0;
+    return split_workspace(split_plan(Q, N, k, di.sms), Q, k);
+}
+
+int ksel_select_ex(const float* dist, int64_t Q, int64_t N, int k, float* out_val, int32_t* out_idx, void* d_work,
+                   size_t work_bytes, void* stream) {
+    int st = check_select_args(dist, Q, N, k, out_val, out_idx);
+    if (st) return st;
+    if (!d_work || work_bytes == 0) return ksel_select(dist, Q, N, k, out_val, out_idx, stream);
+    DevInfo di;
+    st = current_device_info(&di);
+    if (st) return st;
+    const SplitPlan p = split_plan(Q, N, k, di.sms);
+    const size_t need = split_workspace(p, Q, k);
+    if (need == 0) return ksel_select(dist, Q, N, k, out_val, out_idx, stream);
+    if (work_bytes < need) return KSEL_ERR_INVALID_ARG;
+    const size_t in_bytes = (size_t)Q * (size_t)N * 4u, out_bytes = (size_t)Q * (size_t)k * 4u;
+    if (overlaps(dist, in_bytes, out_val, out_bytes) || overlaps(dist, in_bytes, out_idx, out_bytes) ||
+        overlaps(out_val, out_bytes, out_idx, out_bytes) || overlaps(d_work, need, dist, in_bytes) ||
+        overlaps(d_work, need, out_val, out_bytes) || overlaps(d_work, need, out_idx, out_bytes))
+        return KSEL_ERR_INVALID_ARG;
+    uint8_t* w = static_cast<uint8_t*>(d_work);
+    const int64_t Sk = (int64_t)p.S * k;
+    const size_t lb = al256((size_t)Q * (size_t)Sk * 4u);
+    float* lv = reinterpret_cast<float*>(w);
+    int32_t* li = reinterpret_cast<int32_t*>(w + lb);
+    int32_t* pos = reinterpret_cast<int32_t*>(w + 2 * lb);
+    const cudaStream_t cs = (cudaStream_t)stream;
+    const int slot = timing_begin(cs);
+    SegMap seg;
+    seg.nseg = p.S;
+    seg.seg_len = p.seg_len;
+    const int64_t V = (int64_t)p.S * Q;  // virtual rows, [Q][S] order
+    cudaError_t e = launch_select_pool(dist, V, N, k, lv, li, pool_launch_shape(V, p.seg_len, k, di.sms, 0), cs, seg);
+    // second level: top-k of each row's S*k candidates, 8 warps per row (few, short rows)
+    if (e == cudaSuccess) e = launch_select_pool(lv, Q, Sk, k, out_val, pos, pool_launch_shape(Q, Sk, k, di.sms, 8), cs);
+    if (e == cudaSuccess) {
+        const int64_t n = Q * (int64_t)k;
+        split_gather_idx_kernel<<<(unsigned)((n + 255) / 256), 256, 0, cs>>>(li, pos, Q, Sk, k, out_idx);
+        note_launch();
+        e = cudaGetLastError();
+    }
+    timing_end(slot, cs);
+    return e == cudaSuccess ? KSEL_OK : KSEL_ERR_CUDA;
+}
+
 int ksel_merge(const float* cand_val, const int32_t* cand_idx, int64_t Q, int S, int kin, int k, float* out_val,
                int32_t* out_idx, void* stream) {
     if (!cand_val || !cand_idx || !out_val || !out_idx) return KSEL_ERR_INVALID_ARG;
@@ -216,7 +314,6 @@ int ksel_merge(const float* cand_val, const int32_t* cand_idx, int64_t Q, int S,
 // ---------------------------------------------------------------------------
 static const size_t kHostSlotTarget = 256ull << 20;  // bytes of input per pipeline slot
 
-static size_t al256(size_t x) { return (x + 255u) & ~(size_t)255u; }
 
 // bytes of one pipeline slot holding `rows` rows: [dist | out_val | out_idx], 256-B aligned parts
 static size_t host_slot_bytes(int64_t rows, int64_t N, int k) {

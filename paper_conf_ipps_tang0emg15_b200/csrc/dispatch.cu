@@ -51,8 +51,8 @@ cudaError_t launch_select_stream(const float* dist, int64_t Q, int64_t N, int k,
 }
 
 cudaError_t launch_select_pool(const float* dist, int64_t Q, int64_t N, int k, float* ov, int32_t* oi, int wpr,
-                               cudaStream_t stream) {
-    KSEL_DISPATCH_R(launch_pool_r, queue_regs(k), dist, Q, N, k, ov, oi, wpr, stream)
+                               cudaStream_t stream, SegMap seg) {
+    KSEL_DISPATCH_R(launch_pool_r, queue_regs(k), dist, Q, N, k, ov, oi, wpr, seg, stream)
 }
 
 cudaError_t launch_merge(const float* cv, const int32_t* ci, int64_t Q, int S, int kin, int k, float* ov,

@@ -731,6 +731,11 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
         if (cost < best_cost) { best_cost = cost; best = s; }
     }
     g.S = best;
+    static const int splits_env = [] {
+        const char* e = std::getenv("KSEL_KNN_SPLITS");  // experiments: force the split count
+        return e ? std::atoi(e) : 0;
+    }();
+    if (splits_env > 0) g.S = std::min(splits_env, smax);
     return g;
 }
 

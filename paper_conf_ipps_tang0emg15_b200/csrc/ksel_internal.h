@@ -40,9 +40,16 @@ int pool_launch_shape(int64_t Q, int64_t N, int k, int num_sms, int forced_wpr);
 cudaError_t launch_select_stream(const float* dist, int64_t Q, int64_t N, int k, float* out_val,
                                  int32_t* out_idx, int wpr, cudaStream_t stream);
 
-// Pool + radix-narrowing selection (select_pool.cu).
+// Split-row mapping of the pool kernel (seg_len == 0: one virtual row per row).
+struct SegMap {
+    int64_t nseg = 1;     // segments per row
+    int64_t seg_len = 0;  // columns per segment (the last one may be shorter)
+};
+
+// Pool + radix-narrowing selection (select_pool.cu).  With seg.seg_len > 0, Q counts
+// virtual rows (segments x real rows).
 cudaError_t launch_select_pool(const float* dist, int64_t Q, int64_t N, int k, float* out_val, int32_t* out_idx,
-                               int wpr, cudaStream_t stream);
+                               int wpr, cudaStream_t stream, SegMap seg = SegMap());
 
 // Merge of S sorted candidate lists (merge.cu).
 cudaError_t launch_merge(const float* cand_val, const int32_t* cand_idx, int64_t Q, int S, int kin,
@@ -59,7 +66,7 @@ cudaError_t launch_stream_r(const float* dist, int64_t Q, int64_t N, int k, floa
                             cudaStream_t stream);
 template <int R>
 cudaError_t launch_pool_r(const float* dist, int64_t Q, int64_t N, int k, float* ov, int32_t* oi, int wpr,
-                          cudaStream_t stream);
+                          SegMap seg, cudaStream_t stream);
 template <int R>
 cudaError_t launch_merge_r(const float* cv, const int32_t* ci, int64_t Q, int S, int kin, int k, float* ov,
                            int32_t* oi, cudaStream_t stream);

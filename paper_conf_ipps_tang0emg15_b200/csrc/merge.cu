@@ -42,6 +42,49 @@ __device__ __forceinline__ bool warr_is_sorted(const WArr<RL>& a, uint32_t lane)
     return !__any_sync(kFull, bad);
 }
 
+// Bits of the candidate (key, idx) of query q in the [S][Q][kin] lists: lanes take
+// lists, binary search for the lexicographic lower bound of (key, idx) in a sorted
+// list (8-10 dependent loads); a warp-wide linear scan if no list has it at the
+// searched position (unsorted input lists).  Warp-uniform result.
+static __device__ __noinline__ uint32_t regather_bits(const float* __restrict__ cv, const int32_t* __restrict__ ci, int64_t q,
+                                               int64_t Q, int S, int kin, uint32_t key, uint32_t idx,
+                                               uint32_t lane) {
+    for (int s0 = 0; s0 < S; s0 += 32) {
+        const int s = s0 + (int)lane;
+        bool hit = false;
+        uint32_t hb = 0;
+        if (s < S) {
+            const int64_t base = ((int64_t)s * Q + q) * kin;
+            int lo = 0, hi = kin;  // first position not below (key, idx)
+            while (lo < hi) {
+                const int mid = (lo + hi) >> 1;
+                if (pair_lt(key_of(cv[base + mid]), (uint32_t)ci[base + mid], key, idx)) lo = mid + 1;
+                else hi = mid;
+            }
+            if (lo < kin && (uint32_t)ci[base + lo] == idx && key_of(cv[base + lo]) == key) {
+                hit = true;
+                hb = __float_as_uint(cv[base + lo]);
+            }
+        }
+        const uint32_t m = __ballot_sync(kFull, hit);
+        if (m) return __shfl_sync(kFull, hb, __ffs(m) - 1);
+    }
+    const int64_t total = (int64_t)S * kin;
+    for (int64_t t0 = 0; t0 < total; t0 += 32) {
+        const int64_t t = t0 + lane;
+        bool hit = false;
+        uint32_t hb = 0;
+        if (t < total) {
+            const int64_t a = ((t / kin) * Q + q) * kin + t % kin;
+            hit = (uint32_t)ci[a] == idx && key_of(cv[a]) == key;
+            hb = __float_as_uint(cv[a]);
+        }
+        const uint32_t m = __ballot_sync(kFull, hit);
+        if (m) return __shfl_sync(kFull, hb, __ffs(m) - 1);
+    }
+    return bits_of_key(key);  // not reached: the pair came from the lists
+}
+
 template <int R, int RL>
 __global__ void __launch_bounds__(32 * kMergeWarps)
     ksel_merge_kernel(const float* __restrict__ cv, const int32_t* __restrict__ ci, int64_t Q, int S, int kin,
@@ -78,23 +121,20 @@ __global__ void __launch_bounds__(32 * kMergeWarps)
 #pragma unroll
     for (int r = 0; r < R; ++r) {
         const int e = r * 32 + (int)lane;
+        const uint32_t key = acc.k[r];
+        const uint32_t idx = acc.i[r];
+        uint32_t bits = bits_of_key(key);
+        // -0.0 / NaN payloads: the canonical key dropped the bits; find the candidate's
+        // own copy, warp-cooperatively, one such output at a time (rare)
+        uint32_t need = __ballot_sync(kFull, e < k && key_needs_regather(key));
+        while (need) {
+            const int j = __ffs(need) - 1;
+            need &= need - 1u;
+            const uint32_t b = regather_bits(cv, ci, q, Q, S, kin, __shfl_sync(kFull, key, j),
+                                             __shfl_sync(kFull, idx, j), lane);
+            if ((int)lane == j) bits = b;
+        }
         if (e < k) {
-            const uint32_t key = acc.k[r];
-            const uint32_t idx = acc.i[r];
-            uint32_t bits = bits_of_key(key);
-            if (key_needs_regather(key)) {  // -0.0 / NaN payload: find the candidate's own bits
-                for (int s = 0; s < S; ++s) {
-                    const int64_t base = ((int64_t)s * Q + q) * kin;
-                    bool found = false;
-                    for (int t = 0; t < kin; ++t)
-                        if ((uint32_t)ci[base + t] == idx && key_of(cv[base + t]) == key) {
-                            bits = __float_as_uint(cv[base + t]);
-                            found = true;
-                            break;
-                        }
-                    if (found) break;
-                }
-            }
             ov[e] = __uint_as_float(bits);
             oi[e] = (int32_t)idx;
         }

@@ -105,7 +105,7 @@ __device__ __noinline__ void pool_merge_sorted(uint32_t* __restrict__ qk, uint32
 template <int R, int WPR, int RPC, int SD>
 __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads)
     ksel_pool_kernel(const float* __restrict__ dist, int64_t Q, int64_t N, int k, float* __restrict__ out_val,
-                     int32_t* __restrict__ out_idx, int order_mode) {
+                     int32_t* __restrict__ out_idx, int order_mode, SegMap seg) {
     using Cfg = PoolCfg<R, WPR, RPC, SD>;
     constexpr int CH = Cfg::CH, S = Cfg::S, G = Cfg::G, NS = Cfg::NS;
     extern __shared__ __align__(128) uint8_t smem[];
@@ -127,8 +127,19 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads)
     uint32_t* cid = reinterpret_cast<uint32_t*>(mbar + S);  // chunk id of each stage
 
     // ---- row geometry -----------------------------------------------------------
-    const uint64_t g0 = (uint64_t)row * (uint64_t)N;
-    const uint64_t g1 = g0 + (uint64_t)N;
+    // Split rows (seg.seg_len > 0): virtual row v = q * seg.nseg + s is segment s
+    // of row q, columns [s * seg_len, min(N, (s + 1) * seg_len)); its top-k goes to output
+    // row v ([Q][S][k]: a row's S sorted lists are contiguous) with row-global indices.
+    int64_t qrow = row;
+    uint64_t coloff = 0, len = (uint64_t)N;
+    if (seg.seg_len > 0) {
+        qrow = row / seg.nseg;
+        const int64_t sg = row - qrow * seg.nseg;
+        coloff = (uint64_t)sg * (uint64_t)seg.seg_len;
+        len = min((uint64_t)seg.seg_len, (uint64_t)N - coloff);
+    }
+    const uint64_t g0 = (uint64_t)qrow * (uint64_t)N + coloff;
+    const uint64_t g1 = g0 + len;
     const uint64_t mis = ((reinterpret_cast<uintptr_t>(dist) >> 2) + g0) & 3u;
     uint64_t a0 = g0 + ((4u - mis) & 3u);
     if (a0 > g1) a0 = g1;
@@ -421,19 +432,19 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads)
         const uint32_t col = pi[e];
         const uint32_t bits = key_needs_regather(key) ? __float_as_uint(dist[g0 + col]) : bits_of_key(key);
         ov[e] = __uint_as_float(bits);
-        oi[e] = (int32_t)col;
+        oi[e] = (int32_t)(col + (uint32_t)coloff);
     }
 }
 
 template <int R, int WPR, int RPC, int SD>
 static cudaError_t launch_pool_cfg(const float* dist, int64_t Q, int64_t N, int k, float* ov, int32_t* oi,
-                                   cudaStream_t stream) {
+                                   SegMap seg, cudaStream_t stream) {
     using Cfg = PoolCfg<R, WPR, RPC, SD>;
     auto kern = ksel_pool_kernel<R, WPR, RPC, SD>;
     cudaError_t e = ensure_smem_attr(reinterpret_cast<const void*>(kern), Cfg::kSmem);
     if (e != cudaSuccess) return e;
     const int64_t grid = (Q + RPC - 1) / RPC;
-    kern<<<(unsigned)grid, Cfg::kThreads, Cfg::kSmem, stream>>>(dist, Q, N, k, ov, oi, chunk_order_mode());
+    kern<<<(unsigned)grid, Cfg::kThreads, Cfg::kSmem, stream>>>(dist, Q, N, k, ov, oi, chunk_order_mode(), seg);
     note_launch();
     return cudaGetLastError();
 }
@@ -442,37 +453,37 @@ static cudaError_t launch_pool_cfg(const float* dist, int64_t Q, int64_t N, int 
 // large queues with many warps per row fall back to fewer warps per CTA.
 template <int R, int WPR, int RPC, int SD>
 static cudaError_t launch_pool_fit(const float* dist, int64_t Q, int64_t N, int k, float* ov, int32_t* oi,
-                                   cudaStream_t stream) {
+                                   SegMap seg, cudaStream_t stream) {
     if constexpr (PoolCfg<R, WPR, RPC, SD>::kSmem > kMaxSmemPerBlock) {
-        if constexpr (RPC > 1) return launch_pool_fit<R, WPR, RPC / 2, SD>(dist, Q, N, k, ov, oi, stream);
-        else return launch_pool_fit<R, WPR / 2, 1, SD>(dist, Q, N, k, ov, oi, stream);
+        if constexpr (RPC > 1) return launch_pool_fit<R, WPR, RPC / 2, SD>(dist, Q, N, k, ov, oi, seg, stream);
+        else return launch_pool_fit<R, WPR / 2, 1, SD>(dist, Q, N, k, ov, oi, seg, stream);
     } else {
-        return launch_pool_cfg<R, WPR, RPC, SD>(dist, Q, N, k, ov, oi, stream);
+        return launch_pool_cfg<R, WPR, RPC, SD>(dist, Q, N, k, ov, oi, seg, stream);
     }
 }
 
 // wpr < 0 selects the deep ring (6 stages) with |wpr| warps per row.
 template <int R>
 cudaError_t launch_pool_r(const float* dist, int64_t Q, int64_t N, int k, float* ov, int32_t* oi, int wpr,
-                          cudaStream_t stream) {
+                          SegMap seg, cudaStream_t stream) {
     if (wpr < 0) {
         switch (-wpr) {
-            case 1: return launch_pool_fit<R, 1, 1, 6>(dist, Q, N, k, ov, oi, stream);
-            case 2: return launch_pool_fit<R, 2, 1, 6>(dist, Q, N, k, ov, oi, stream);
-            case 4: return launch_pool_fit<R, 4, 1, 6>(dist, Q, N, k, ov, oi, stream);
-            default: return launch_pool_fit<R, 8, 1, 6>(dist, Q, N, k, ov, oi, stream);
+            case 1: return launch_pool_fit<R, 1, 1, 6>(dist, Q, N, k, ov, oi, seg, stream);
+            case 2: return launch_pool_fit<R, 2, 1, 6>(dist, Q, N, k, ov, oi, seg, stream);
+            case 4: return launch_pool_fit<R, 4, 1, 6>(dist, Q, N, k, ov, oi, seg, stream);
+            default: return launch_pool_fit<R, 8, 1, 6>(dist, Q, N, k, ov, oi, seg, stream);
         }
     }
     switch (wpr) {
-        case 1: return launch_pool_fit<R, 1, 1, 3>(dist, Q, N, k, ov, oi, stream);
-        case 2: return launch_pool_fit<R, 2, 1, 3>(dist, Q, N, k, ov, oi, stream);
-        case 4: return launch_pool_fit<R, 4, 1, 3>(dist, Q, N, k, ov, oi, stream);
-        default: return launch_pool_fit<R, 8, 1, 3>(dist, Q, N, k, ov, oi, stream);
+        case 1: return launch_pool_fit<R, 1, 1, 3>(dist, Q, N, k, ov, oi, seg, stream);
+        case 2: return launch_pool_fit<R, 2, 1, 3>(dist, Q, N, k, ov, oi, seg, stream);
+        case 4: return launch_pool_fit<R, 4, 1, 3>(dist, Q, N, k, ov, oi, seg, stream);
+        default: return launch_pool_fit<R, 8, 1, 3>(dist, Q, N, k, ov, oi, seg, stream);
     }
 }
 
 // One object per queue size R (build.py compiles this file with -DKSEL_ONLY_R=R).
-template cudaError_t launch_pool_r<KSEL_ONLY_R>(const float*, int64_t, int64_t, int, float*, int32_t*, int,
+template cudaError_t launch_pool_r<KSEL_ONLY_R>(const float*, int64_t, int64_t, int, float*, int32_t*, int, SegMap,
                                                 cudaStream_t);
 
 }  // namespace ksel

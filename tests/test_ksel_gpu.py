@@ -138,6 +138,73 @@ def test_config3_full_size_sampled_rows(K, oracle_mod):
     assert_same(ev, ei, gv[sample].cpu().numpy(), gi[sample].cpu().numpy(), "C3 sample")
 
 
+@pytest.mark.slow
+@pytest.mark.parametrize("dist,k", [("T", 256), ("T", 1024), ("SD", 256), ("G", 1024), ("DG", 256), ("U", 1024)])
+def test_config3_rows_other_distributions(K, oracle_mod, dist, k):
+    # configs[2] row shape (N=2^20) with the kernel configuration the Q=16384 bench launch
+    # uses (one warp per row, 3-stage ring: any Q > 1776 rows), on 2048 rows; heavy ties
+    # exercise the strict pre-filter past the bound's index
+    Q, N = 2048, 1 << 20
+    seed = synth.seed_for(3, dist)
+    x = synth.rows(dist, seed, 0, Q, N, device="cuda")
+    gv, gi = K.ksel_select(x, k)
+    torch.cuda.synchronize()
+    sample = list(range(24)) + list(range(100, Q, 53))
+    del x
+    xs = synth.row_subset(dist, seed, sample, N)
+    ev, ei = oracle_mod.select(xs.numpy(), k)
+    assert_same(ev, ei, gv[sample].cpu().numpy(), gi[sample].cpu().numpy(), "C3-shape %s k=%d" % (dist, k))
+
+
+# ---- split rows (few long rows over the whole GPU) ----------------
+
+@pytest.mark.parametrize("Q,N", [(1, (1 << 18) + 13), (3, 1 << 20), (7, 3 * (1 << 19) + 1), (40, 1 << 18)])
+@pytest.mark.parametrize("dist", ["U", "SD", "T", "X"])
+def test_split_rows_vs_oracle(K, oracle_mod, Q, N, dist):
+    # Q below the SM count: ksel_select cuts rows into segments (one CTA each, row-global
+    # indices) and merges the S lists; ragged N makes unaligned segment heads and a short
+    # last segment
+    assert K.ksel_select_workspace(Q, N, 100) > 0
+    x_cpu = synth.rows(dist, 41, 0, Q, N)
+    x = x_cpu.cuda()
+    for k in (1, 100, 256, 1024):
+        gv, gi = K.ksel_select(x, k)
+        dv, di = K.ksel_select(x, k, split_rows=False)
+        torch.cuda.synchronize()
+        ev, ei = oracle_mod.select(x_cpu.numpy(), k)
+        assert_same(ev, ei, gv, gi, "split Q=%d N=%d %s k=%d" % (Q, N, dist, k))
+        assert_same(ev, ei, dv, di, "direct Q=%d N=%d %s k=%d" % (Q, N, dist, k))
+
+
+@pytest.mark.slow
+def test_split_rows_single_long_row(K, oracle_mod):
+    # one row of 2^24 over every SM (148 segments), then the second-level selection over
+    # 148*k candidates with ties mapped back to row indices
+    N = 1 << 24
+    for dist in ("G", "T"):
+        x = synth.rows(dist, 42, 0, 1, N, device="cuda")
+        assert K.ksel_select_workspace(1, N, 64) > 0
+        for k in (64, 1000):
+            gv, gi = K.ksel_select(x, k)
+            torch.cuda.synchronize()
+            ev, ei = oracle_mod.select(x.cpu().numpy(), k)
+            assert_same(ev, ei, gv, gi, "one row %s k=%d" % (dist, k))
+
+
+def test_split_rows_workspace_errors(K):
+    x = torch.rand(2, 1 << 20, device="cuda")
+    v = torch.empty(2, 10, device="cuda")
+    i = torch.empty(2, 10, dtype=torch.int32, device="cuda")
+    need = K.ksel_select_workspace(2, 1 << 20, 10)
+    assert need > 0
+    small = torch.empty(need - 256, dtype=torch.uint8, device="cuda")
+    st = K._lib.ksel_select_ex(x.data_ptr(), 2, 1 << 20, 10, v.data_ptr(), i.data_ptr(), small.data_ptr(),
+                               small.numel(), K._stream(x.device))
+    assert st == 1
+    # enough rows for every SM: no workspace, ksel_select_ex == ksel_select
+    assert K.ksel_select_workspace(4096, 1 << 16, 10) == 0
+
+
 # ---- ksel_merge -----------------------------------------------------------
 
 @pytest.mark.parametrize("S", [1, 2, 3, 8])

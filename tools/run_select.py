@@ -21,15 +21,18 @@ ap.add_argument("--dist", default="U")
 ap.add_argument("--reps", type=int, default=5)
 ap.add_argument("--algo", type=int, default=0)
 ap.add_argument("--wpr", type=int, default=0)
+ap.add_argument("--nosplit", action="store_true", help="force one CTA per row (no split rows)")
 a = ap.parse_args()
 x = synth.rows(a.dist, synth.seed_for(2, a.dist), 0, a.Q, a.N, device="cuda")
 v = torch.empty((a.Q, a.k), dtype=torch.float32, device="cuda")
 i = torch.empty((a.Q, a.k), dtype=torch.int32, device="cuda")
+need = K.ksel_select_workspace(a.Q, a.N, a.k)
+ws = torch.empty(max(need, 1), dtype=torch.uint8, device="cuda")
 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 for r in range(a.reps):
     torch.cuda.synchronize()
     e0.record()
-    K.ksel_select(x, a.k, v, i, algo=a.algo, warps_per_row=a.wpr)
+    K.ksel_select(x, a.k, v, i, algo=a.algo, warps_per_row=a.wpr, workspace=ws, split_rows=not a.nosplit)
     e1.record()
     torch.cuda.synchronize()
     ms = e0.elapsed_time(e1)
