@@ -349,7 +349,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                 for (int ks = 0; ks <= g.KS; ++ks, ++it) {
                     const int st = (int)(it % NS);
                     const uint32_t bytes = (ks < g.KS) ? KNN_STAGE_BYTES : KNN_NORM_B_BYTES;
-                    mbar_wait(&empty[st], ((it / NS) & 1u) ^ 1u);
+                    mbar_wait_sleep(&empty[st], ((it / NS) & 1u) ^ 1u);
                     mbar_arrive_expect_tx(&full[st], bytes);
                     bulk_g2s(sB + st * KNN_STAGE_BYTES, ref_img + (size_t)t * g.tile_bytes() + (size_t)ks * KNN_STAGE_BYTES,
                              bytes, &full[st]);
@@ -368,12 +368,12 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
             uint32_t it = 0;
             for (int lt = 0; lt < nsteps; ++lt) {
                 const int b = lt & 1;
-                mbar_wait(&acce[b], (((uint32_t)lt >> 1) & 1u) ^ 1u);
+                mbar_wait_sleep(&acce[b], (((uint32_t)lt >> 1) & 1u) ^ 1u);
                 tc_fence_after();
                 const uint32_t d_tmem = tmem_base + (uint32_t)(b * KNN_BN);
                 for (int ks = 0; ks <= g.KS; ++ks, ++it) {
                     const int st = (int)(it % NS);
-                    mbar_wait(&full[st], (it / NS) & 1u);
+                    mbar_wait_sleep(&full[st], (it / NS) & 1u);
                     tc_fence_after();
                     const uint32_t bs = smem_u32(sB + st * KNN_STAGE_BYTES);
                     if (ks == g.KS) {  // norm block: |q|^2 + |r|^2 into the same accumulator
