@@ -151,6 +151,23 @@ def oracle_rows_per_s(dist: str, seed: int, N: int, k: int, rows: list, threads:
     return len(rows) / dt, dt
 
 
+def select_config(Qr, N, k, dist, world):
+    """The ksel_select workload config (shared by both arms)."""
+    return {"workload": "ksel_select Q=%d N=%d k=%d %s" % (Qr, N, k, dist), "Q_per_rank": Qr,
+            "Q_total": Qr * world, "N": N, "k": k, "dist": dist,
+            "parallelism": "query-sharded x%d (no communication)" % world,
+            "l2": "inputs (%.1f GiB/rank) far larger than L2; no flush" % (Qr * N * 4 / 2**30)}
+
+
+def knn_config(N, Nl, Q, D, k, kind, mode, world):
+    """The knn_search workload config (shared by both arms)."""
+    return {"workload": "knn_search N=%d Q=%d D=%d k=%d %s (%s)" % (N, Q, D, k, kind, mode), "N": N,
+            "N_per_rank": Nl, "Q": Q, "D": D, "k": k, "points": kind,
+            "parallelism": ("reference rows sharded x%d + NCCL all-gather + ksel_merge" % world
+                            if mode == "row-sharded" else "replicas x%d" % world),
+            "l2": "reference image %.2f GB per rank (> L2)" % (Nl * D * 4 / 1e9)}
+
+
 def run_reference_knn(args, rank, world):
     """--impl reference for the kNN configs: the oracle (double-precision triple
     loop + sort) on a bounded sample of queries per step."""
@@ -177,9 +194,10 @@ def run_reference_knn(args, rank, world):
     line = {
         "impl": "reference", "metric": "queries/sec (fused tcgen05 distance + k-selection)", "value": value,
         "unit": "queries/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-        "ms_per_step": 1e3 * total / args.steps, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "ms_per_step": 1e3 * total / args.steps, "higher_is_better": True,
+        "scaling": "strong" if mode == "row-sharded" else "weak", "vs_baseline": None,
         "dtype": "f64", "data": "synthetic",
-        "config": {"workload": "knn_search N=%d Q=%d D=%d k=%d %s (oracle on host cores)" % (nref, Q, D, k, kind)},
+        "config": knn_config(N, nref, Q, D, k, kind, mode, world),
         "cpu_baseline": {"value": value, "unit": "queries/s", "cores": threads, "kind": "oracle",
                          "sample": "%d queries vs %d references per step" % (nq, nref)},
         "e2e": {"value": value, "unit": "queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -212,8 +230,7 @@ def run_reference(args, rank, world):
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * total / args.steps,
         "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None, "dtype": "f32",
         "data": "synthetic",
-        "config": {"workload": "ksel_select Q=%d/rank N=%d k=%d %s (oracle on host cores)" % (Qr, N, k, dist),
-                   "Q_per_rank": Qr, "N": N, "k": k, "dist": dist},
+        "config": select_config(Qr, N, k, dist, world),
         "cpu_baseline": {"value": value, "unit": "rows/s", "cores": threads, "kind": "oracle",
                          "sample": "%d rows of N=%d per step (stable sort by (value,index), truncate to k)"
                                    % (rows_per_step, N)},
@@ -294,7 +311,8 @@ def bench_select(args, rank, world, local_rank, dev, K, tdist):
     peak, peak_src = load_peaks()
     alg_bytes = Qr * (4.0 * N + 8.0 * k)
     achieved = alg_bytes / (kern_ms / 1e3) / 1e9
-    workload = "ksel_select Q=%d N=%d k=%d %s" % (Qr, N, k, dist)
+    cfg = select_config(Qr, N, k, dist, world)
+    workload = cfg["workload"]
     line = None
     if rank == 0:
         line = {
@@ -302,9 +320,7 @@ def bench_select(args, rank, world, local_rank, dev, K, tdist):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step,
             "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None,
             "dtype": "f32", "data": "synthetic",
-            "config": {"workload": workload, "Q_per_rank": Qr, "Q_total": rows_total, "N": N, "k": k,
-                       "dist": dist, "parallelism": "query-sharded x%d (no communication)" % world,
-                       "l2": "inputs (%.1f GiB/rank) far larger than L2; no flush" % (Qr * N * 4 / 2**30)},
+            "config": cfg,
             "hbm_gbs": achieved,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": load_traffic(workload), "peak_source": peak_src,
@@ -401,7 +417,8 @@ def bench_knn(args, rank, world, local_rank, dev, K, tdist):
         peaks_bf16 = 1590.0
     flops = 2.0 * Q * Nl * D  # algorithmic single-pass dot products of this rank's launch
     achieved = flops / (kern_ms / 1e3) / 1e12
-    workload = "knn_search N=%d Q=%d D=%d k=%d %s (%s)" % (N, Q, D, k, kind, mode)
+    cfg = knn_config(N, Nl, Q, D, k, kind, mode, world)
+    workload = cfg["workload"]
     line = None
     if rank == 0:
         line = {
@@ -409,10 +426,7 @@ def bench_knn(args, rank, world, local_rank, dev, K, tdist):
             "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step,
             "higher_is_better": True, "scaling": "strong" if mode == "row-sharded" else "weak",
             "vs_baseline": None, "dtype": "bf16x3->f32", "data": "synthetic",
-            "config": {"workload": workload, "N": N, "N_per_rank": Nl, "Q": Q, "D": D, "k": k, "points": kind,
-                       "parallelism": ("reference rows sharded x%d + NCCL all-gather + ksel_merge" % world
-                                       if mode == "row-sharded" else "replicas x%d" % world),
-                       "l2": "reference image %.2f GB per rank (> L2)" % (Nl * D * 4 / 1e9)},
+            "config": cfg,
             "roofline": {"bound": "tensor", "achieved": achieved, "peak": peaks_bf16, "unit": "TFLOP/s",
                          "frac": achieved / peaks_bf16, "traffic": load_traffic(workload), "peak_source": src,
                          "kernel": "knn_fused_kernel", "kernel_ms": kern_ms,
