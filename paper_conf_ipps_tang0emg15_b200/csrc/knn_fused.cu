@@ -76,6 +76,10 @@ struct KnnGeom {
     int sample_ctas;
     int halves;          // column halves per tile (EW / 4): pools per split
     int pcap;            // pool fill that triggers a narrowing before a tile (<= P)
+    int cs;              // cluster size: CTAs (consecutive query tiles, same reference range) that
+                         // share every reference stage through one multicast load
+    int QTp;             // query tiles padded to a multiple of cs (padding tiles select nothing)
+    int passes;          // 3 (hi.hi + hi.lo + lo.hi); 1 = hi.hi only (experiments: pipeline timing)
     __host__ __device__ size_t tile_bytes() const { return (size_t)KS * KNN_STAGE_BYTES + KNN_NORM_B_BYTES; }
     __host__ __device__ int a_bytes() const { return Dp * 512 + KNN_NORM_A_BYTES; }
 };
@@ -255,6 +259,33 @@ __device__ __forceinline__ void red_add_shared(uint32_t saddr, uint32_t v) {
     asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(saddr), "r"(v) : "memory");
 }
 
+// cluster helpers (reference-stage multicast across the CTAs of a cluster)
+__device__ __forceinline__ uint32_t cluster_rank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+// 1-D bulk copy global -> the same shared-memory offset in every CTA of `mask`;
+// each destination CTA's mbarrier at `bar`'s offset receives the complete_tx bytes
+__device__ __forceinline__ void bulk_g2s_mc(void* dst, const void* src, uint32_t bytes, uint64_t* bar, uint16_t mask) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster [%0], [%1], %2, [%3], "
+        "%4;" ::"r"(smem_u32(dst)),
+        "l"(src), "r"(bytes), "r"(smem_u32(bar)), "h"(mask)
+        : "memory");
+}
+// MMA completion -> arrive on the mbarrier at `bar`'s offset in every CTA of `mask`
+__device__ __forceinline__ void umma_commit_mc(uint64_t* bar, uint16_t mask) {
+    asm volatile(
+        "tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+            smem_u32(bar)),
+        "h"(mask)
+        : "memory");
+}
+
 // ---------------------------------------------------------------------------
 // the fused kernel
 // ---------------------------------------------------------------------------
@@ -270,7 +301,8 @@ struct KnnSmem {
 
 // MODE 0: selection (knn_search); 1: write every distance (knn_distances);
 // 2: pipeline only -- the epilogue reads the accumulators and drops them
-// (experiments: isolates the TMA + MMA + TMEM pipeline from the selection).
+// (experiments: isolates the TMA + MMA + TMEM pipeline from the selection);
+// 3: selection + per-warp cycle counters; 4: pipeline without any TMEM read.
 template <int MODE, int EW>
 __global__ void __launch_bounds__(knn_threads(EW), 1)
     knn_fused_kernel(KnnGeom g, const uint8_t* __restrict__ ref_img, const uint8_t* __restrict__ q_img,
@@ -279,7 +311,8 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
     constexpr int HALVES = EW / 4;
     constexpr int WCOLS = KNN_BN / HALVES;  // columns of each tile this epilogue warp scans
     constexpr bool DUMP = (MODE == 1);
-    constexpr bool PIPE_ONLY = (MODE == 2);
+    constexpr bool PIPE_ONLY = (MODE == 2 || MODE == 4);
+    constexpr bool NO_READ = (MODE == 4);  // pipeline only, accumulators never read (experiments)
     constexpr bool PROF = (MODE == 3);  // selection + per-warp cycle counters (experiments)
     unsigned long long prof_app = 0, prof_narrow = 0, prof_wait = 0, prof_chunks = 0, prof_rare = 0, prof_nrare = 0, prof_nnarrow = 0;
     const unsigned long long prof_t0 = PROF ? clock64() : 0;
@@ -300,8 +333,10 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
 
     const int warp = threadIdx.x >> 5;
     const uint32_t lane = lane_id();
-    const int qt = blockIdx.x % g.QT;
-    const int split = blockIdx.x / g.QT;
+    const int qt = blockIdx.x % g.QTp;  // >= QT: padding tile of a cluster (loads, MMAs, no queries)
+    const int split = blockIdx.x / g.QTp;
+    const uint32_t crank = g.cs > 1 ? cluster_rank() : 0u;
+    const uint16_t cmask = (uint16_t)((1u << g.cs) - 1u);
     const int t0 = (int)((int64_t)g.ntiles * split / g.S);  // logical tile range of this CTA
     const int t1 = (int)((int64_t)g.ntiles * (split + 1) / g.S);
     // Cold CTAs (the first wave: no split of their queries has published a bound
@@ -316,7 +351,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
     if (warp == 0 && lane == 0) {
         for (int s = 0; s < NS; ++s) {
             mbar_init(&full[s], 1);
-            mbar_init(&empty[s], 1);
+            mbar_init(&empty[s], g.cs);  // every CTA of the cluster must have consumed the stage
         }
         for (int b = 0; b < 2; ++b) {
             mbar_init(&accf[b], 1);
@@ -333,6 +368,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
     }
     tc_fence_before();
     __syncthreads();
+    if (g.cs > 1) cluster_sync_all();  // peers' barriers initialised before any multicast
     tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
 
@@ -342,7 +378,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
         if (lane == 0) {
             const uint32_t abytes = (uint32_t)g.a_bytes();
             mbar_arrive_expect_tx(afull, abytes);
-            bulk_g2s(sA, q_img + (size_t)qt * abytes, abytes, afull);
+            bulk_g2s(sA, q_img + (size_t)(qt < g.QT ? qt : 0) * abytes, abytes, afull);
             uint32_t it = 0;
             for (int lt = 0; lt < nsteps; ++lt) {
                 const int t = (lt < Fs ? t0 + lt : t0 + lt - Fs) * g.tstride;
@@ -351,8 +387,13 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                     const uint32_t bytes = (ks < g.KS) ? KNN_STAGE_BYTES : KNN_NORM_B_BYTES;
                     mbar_wait_sleep(&empty[st], ((it / NS) & 1u) ^ 1u);
                     mbar_arrive_expect_tx(&full[st], bytes);
-                    bulk_g2s(sB + st * KNN_STAGE_BYTES, ref_img + (size_t)t * g.tile_bytes() + (size_t)ks * KNN_STAGE_BYTES,
-                             bytes, &full[st]);
+                    const uint8_t* src = ref_img + (size_t)t * g.tile_bytes() + (size_t)ks * KNN_STAGE_BYTES;
+                    if (g.cs == 1) {
+                        bulk_g2s(sB + st * KNN_STAGE_BYTES, src, bytes, &full[st]);
+                    } else {  // this CTA's slice of the stage, into every CTA of the cluster
+                        const uint32_t sl = bytes / g.cs;
+                        bulk_g2s_mc(sB + st * KNN_STAGE_BYTES + crank * sl, src + crank * sl, sl, &full[st], cmask);
+                    }
                 }
             }
         }
@@ -380,7 +421,8 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                         const uint64_t an = umma_desc(anorm, KNN_BM * 16, 128);
                         const uint64_t bn = umma_desc(bs, KNN_BN * 16, 128);
                         umma_bf16(d_tmem, an, bn, idesc, 1u);
-                        umma_commit(&empty[st]);
+                        if (g.cs == 1) umma_commit(&empty[st]);
+                        else umma_commit_mc(&empty[st], cmask);
                         continue;
                     }
 #pragma unroll
@@ -392,10 +434,14 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                         const uint64_t bl =
                             umma_desc(bs + KNN_STAGE_BYTES / 2 + (uint32_t)(2 * j) * (KNN_BN * 16), KNN_BN * 16, 128);
                         umma_bf16(d_tmem, ah, bh, idesc, (ks | j) ? 1u : 0u);
-                        umma_bf16(d_tmem, ah, bl, idesc, 1u);
-                        umma_bf16(d_tmem, al, bh, idesc, 1u);
+                        if (g.passes == 3) {
+                            umma_bf16(d_tmem, ah, bl, idesc, 1u);
+                            umma_bf16(d_tmem, al, bh, idesc, 1u);
+                        }
                     }
-                    umma_commit(&empty[st]);  // frees the stage when these MMAs complete
+                    // frees the stage (in every CTA of the cluster) when these MMAs complete
+                    if (g.cs == 1) umma_commit(&empty[st]);
+                    else umma_commit_mc(&empty[st], cmask);
                 }
                 umma_commit(&accf[b]);  // accumulator b ready for the epilogue
             }
@@ -618,7 +664,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                 }
             }
 #pragma unroll 1
-            for (int c = half * (WCOLS / KNN_CW); c < ((DUMP || PIPE_ONLY) ? (half + 1) * (WCOLS / KNN_CW) : 0); ++c) {
+            for (int c = half * (WCOLS / KNN_CW); c < ((DUMP || (PIPE_ONLY && !NO_READ)) ? (half + 1) * (WCOLS / KNN_CW) : 0); ++c) {
                 uint32_t v[KNN_CW];
                 tmem_ld64(taddr + (uint32_t)(c * KNN_CW), v);
                 if (PIPE_ONLY) {
@@ -662,6 +708,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
 
     tc_fence_before();
     __syncthreads();
+    if (g.cs > 1) cluster_sync_all();  // no peer multicasts into / arrives on this CTA any more
     tc_fence_after();
     if (warp == 1) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(512) : "memory");
 }
@@ -684,6 +731,25 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     g.KS = g.Dp / KNN_KS;
     g.NT = (int)((N + KNN_BN - 1) / KNN_BN);
     g.QT = (int)((Q + KNN_BM - 1) / KNN_BM);
+    static const int cs_env = [] {
+        const char* e = std::getenv("KSEL_KNN_CLUSTER");  // experiments: cluster size 1, 2 or 4
+        const int v = e ? std::atoi(e) : 1;
+        return (v == 2 || v == 4) ? v : 1;
+    }();
+    // Every CTA streams its whole reference range through L2 -> shared memory (4 B per
+    // dim and reference per 128 queries): with one CTA per query tile that stream, not
+    // the tensor pipe, is the floor (measured: ~40 B/clk/SM, the chip's L2 -> SM rate).
+    // A cluster of cs query tiles loads each stage once (every CTA a 1/cs slice,
+    // multicast to all), cutting the L2 traffic per MMA by cs.  Measured on C4: no
+    // gain (cs = 1 / 2 / 4: 6.79 / 6.95 / 8.16 ms; pipeline-only 1-pass 4.08 / 4.36 /
+    // 5.14 ms), so L2 is not the floor and the default is cs = 1.
+    g.cs = (g.QT >= cs_env) ? cs_env : 1;
+    g.QTp = (g.QT + g.cs - 1) / g.cs * g.cs;
+    static const int passes_env = [] {
+        const char* e = std::getenv("KSEL_KNN_PASSES");  // experiments only: 1 breaks the accuracy bound
+        return (e && std::atoi(e) == 1) ? 1 : 3;
+    }();
+    g.passes = passes_env;
     g.k = k;
     const int kk = k < 32 ? 32 : k;
     // room for >= 1 tile of candidates after narrowing to k; register narrowing holds 1152
@@ -717,13 +783,13 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
         return e ? std::atoi(e) : 16;
     }();
     g.sample_tiles = sample_env;
-    g.sample_ctas = g.sample_tiles > 0 ? num_sms : 0;
+    g.sample_ctas = g.sample_tiles > 0 ? num_sms / g.cs * g.cs : 0;  // whole clusters
     // reference splits: enough CTAs for the SMs, waves as full as possible, <= 64 lists to merge
     int best = 1;
     double best_cost = 1e30;
     const int smax = (int)((g.NT < 64) ? g.NT : 64);
     for (int s = 1; s <= smax; ++s) {
-        const double ctas = (double)g.QT * s;
+        const double ctas = (double)g.QTp * s;
         const double waves = ctas / num_sms;
         const double cost = (double)((int64_t)((ctas + num_sms - 1) / num_sms)) / waves  // tail efficiency
                             + (waves < 2.0 ? (2.0 - waves) : 0.0)                        // too few waves
@@ -747,7 +813,7 @@ static KnnWork knn_work_layout(const KnnGeom& g) {
     w.pool = off;    off += al256((size_t)2 * g.S * g.Q * g.P * 8);  // 2 lists (column halves) per split
     w.cnt = off;     off += al256((size_t)2 * g.S * g.Q * 4);
     w.qthr = off;    off += al256((size_t)g.Q * 8);
-    w.prof = off;    off += al256((size_t)g.QT * g.S * KNN_MAX_EW * 16 * 8);  // MODE 3 counters
+    w.prof = off;    off += al256((size_t)g.QTp * g.S * KNN_MAX_EW * 16 * 8);  // MODE 3 counters
     w.total = off;
     return w;
 }
@@ -773,25 +839,37 @@ static cudaError_t knn_run(const float* ref, const float* query, const KnnGeom& 
     const int smem = KnnSmem::total(g);
     static const int mode_env = [] {
         const char* e = std::getenv("KSEL_KNN_MODE");
-        return (e && (e[0] == '2' || e[0] == '3')) ? e[0] - '0' : 0;
+        return (e && (e[0] == '2' || e[0] == '3' || e[0] == '4')) ? e[0] - '0' : 0;
     }();
     const bool ew8 = g.halves == 2;
     auto kern = dump ? (ew8 ? knn_fused_kernel<1, 8> : knn_fused_kernel<1, 4>)
               : mode_env == 2 ? (ew8 ? knn_fused_kernel<2, 8> : knn_fused_kernel<2, 4>)
               : mode_env == 3 ? (ew8 ? knn_fused_kernel<3, 8> : knn_fused_kernel<3, 4>)
+              : mode_env == 4 ? knn_fused_kernel<4, 4>
                               : (ew8 ? knn_fused_kernel<0, 8> : knn_fused_kernel<0, 4>);
     if (!dump && mode_env == 3) dump = reinterpret_cast<float*>(work + w.prof);
     e = ensure_smem_attr(reinterpret_cast<const void*>(kern), smem);
     if (e != cudaSuccess) return e;
     const int slot = dump ? -1 : timing_begin(stream);
-    kern<<<(unsigned)(g.QT * g.S), knn_threads(4 * g.halves), smem, stream>>>(
-        g, reinterpret_cast<const uint8_t*>(ref_img), reinterpret_cast<const uint8_t*>(q_img),
-        reinterpret_cast<unsigned long long*>(work + w.pool),
-        reinterpret_cast<int32_t*>(work + w.cnt),
-        reinterpret_cast<unsigned long long*>(work + w.qthr), dump);
+    cudaLaunchConfig_t cfg{};
+    cudaLaunchAttribute attr[1];
+    cfg.gridDim = dim3((unsigned)(g.QTp * g.S));
+    cfg.blockDim = dim3((unsigned)knn_threads(4 * g.halves));
+    cfg.dynamicSmemBytes = (size_t)smem;
+    cfg.stream = stream;
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = (unsigned)g.cs;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    e = cudaLaunchKernelEx(&cfg, kern, g, reinterpret_cast<const uint8_t*>(ref_img),
+                           reinterpret_cast<const uint8_t*>(q_img), reinterpret_cast<unsigned long long*>(work + w.pool),
+                           reinterpret_cast<int32_t*>(work + w.cnt), reinterpret_cast<unsigned long long*>(work + w.qthr),
+                           dump);
     note_launch();
     timing_end(slot, stream);
-    e = cudaGetLastError();
+    if (e == cudaSuccess) e = cudaGetLastError();
     if (e != cudaSuccess || (dump && mode_env != 3)) return e;
     return launch_merge_pools(reinterpret_cast<const unsigned long long*>(work + w.pool), g.P,
                               reinterpret_cast<const int32_t*>(work + w.cnt), g.halves * g.S, g.Q,

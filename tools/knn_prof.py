@@ -18,7 +18,9 @@ for rep in range(2):
     K.knn_search(ref, qry, k, workspace=ws)
     torch.cuda.synchronize()
 # the counters sit at the end of the workspace (layout: ... qthr | prof); S as in knn_geometry
+CS = int(os.environ.get('KSEL_KNN_CLUSTER', '1'))
 QT = (Q + 127) // 128
+QT = (QT + CS - 1) // CS * CS if QT >= CS else QT
 NT = (N + 255) // 256
 best, best_cost = 1, 1e30
 for s_ in range(1, min(NT, 64) + 1):

@@ -19,6 +19,7 @@ ap.add_argument("--D", type=int, default=128)
 ap.add_argument("--k", type=int, default=100)
 ap.add_argument("--kind", default="knn-U")
 ap.add_argument("--reps", type=int, default=3)
+ap.add_argument("--save", default="")
 a = ap.parse_args()
 ref = synth.knn_points(a.kind, 41, 0, a.N, a.D, device="cuda")
 qry = synth.knn_points(a.kind, 42, 0, a.Q, a.D, device="cuda")
@@ -35,3 +36,6 @@ for r in range(a.reps):
     torch.cuda.synchronize()
     ms = e0.elapsed_time(e1)
     print("rep %d: %.3f ms  %.1f TFLOP/s (1-pass algorithmic)  %.0f queries/s" % (r, ms, flops / ms / 1e9, a.Q / ms * 1e3), flush=True)
+if a.save:
+    import numpy as np
+    np.savez(a.save, v=ov.cpu().numpy(), i=oi.cpu().numpy())
