@@ -169,6 +169,45 @@ KSEL_API size_t knn_distances_workspace(int64_t N, int64_t Q, int D);
 KSEL_API int knn_distances(const float* ref, const float* query, int64_t N, int64_t Q, int D, float* out,
                            void* d_work, size_t work_bytes, void* stream);
 
+/* ---- Row-sharded k-NN exchange without a collective ----
+ * The final merge of the row-sharded k-NN (divide-and-merge)
+ * reading every shard's candidate lists in place -- local memory or a peer
+ * GPU's memory mapped over NVLink with CUDA IPC -- with stream-ordered
+ * device-side release/acquire flags instead of an NCCL all-gather + host
+ * barrier.  Orchestration (double buffering, epochs): dist.py KnnP2P.
+ *
+ * ksel_ipc_alloc -- cudaMalloc `bytes` (zero-filled) and export it: *d_ptr is the
+ *   device pointer, handle_out receives ksel_ipc_handle_size() bytes (a
+ *   cudaIpcMemHandle_t) that another process maps with ksel_ipc_open.  The
+ *   caller owns the allocation (ksel_ipc_free).  KSEL_ERR_CUDA on failure.
+ * ksel_ipc_open / ksel_ipc_close -- map / unmap another process's allocation
+ *   (cudaIpcOpenMemHandle with lazy peer access; not for the exporting process
+ *   itself, which uses its own pointer).
+ * ksel_flag_signal -- enqueue on `stream`: after all earlier work of the stream,
+ *   a system-scope fence then a release store of `value` to the u32 *d_flag
+ *   (local or peer memory, 4-byte aligned).
+ * ksel_flag_wait -- enqueue on `stream`: later work of the stream starts only
+ *   after every d_flags[j] (j < n <= 64, device pointers, local or peer) holds
+ *   a value v with (int32)(v - value) >= 0 (acquire at system scope).  The
+ *   pointer array itself is host memory, read during the call.
+ * ksel_merge_lists -- ksel_merge over S <= 64 lists given as pointer tables
+ *   (host arrays of device pointers): list s of query q (0 <= q < Q) is
+ *   vals[s] + q*kin / idxs[s] + q*kin, sorted ascending in (value, index) as
+ *   knn_search emits it; indices unique per query across lists.  With ready
+ *   != NULL, list s is read only after *ready[s] reached `epoch` (as in
+ *   ksel_flag_wait), with volatile loads.  Output, limits and errors as
+ *   ksel_merge. */
+KSEL_API size_t ksel_ipc_handle_size(void);
+KSEL_API int ksel_ipc_alloc(size_t bytes, void** d_ptr, void* handle_out);
+KSEL_API int ksel_ipc_open(const void* handle, void** d_ptr);
+KSEL_API int ksel_ipc_close(void* d_ptr);
+KSEL_API int ksel_ipc_free(void* d_ptr);
+KSEL_API int ksel_flag_signal(uint32_t* d_flag, uint32_t value, void* stream);
+KSEL_API int ksel_flag_wait(const uint32_t* const* d_flags, int n, uint32_t value, void* stream);
+KSEL_API int ksel_merge_lists(const float* const* vals, const int32_t* const* idxs, int S, int64_t Q, int kin,
+                              int k, float* out_val, int32_t* out_idx, const uint32_t* const* ready,
+                              uint32_t epoch, void* stream);
+
 /* Live per-kernel timing (measurement support for bench.py): while enabled,
  * every entry point records a pair of CUDA events on its stream around its
  * DOMINANT kernel (ksel_select: the selection kernel; knn_search: the fused

@@ -12,6 +12,9 @@ Entry points (same names as the C ABI):
 * :func:`ksel_merge`       -- top-k of the union of S sorted candidate lists.
 * :func:`knn_search`       -- fused distance + selection brute-force k-NN.
 * :func:`knn_graph`        -- k-NN graph of one point set (self excluded).
+* :func:`ksel_merge_lists` -- ksel_merge over pointer tables (peer lists, ready flags);
+  with :func:`ipc_alloc` / :func:`ipc_open` / :func:`flag_signal` / :func:`flag_wait`
+  the collective-free row-sharded k-NN exchange (dist.KnnP2P).
 """
 from __future__ import annotations
 
@@ -58,6 +61,17 @@ _lib.ksel_timing_collect.restype = ctypes.c_int
 _lib.ksel_strerror.argtypes = [_i32]
 _lib.ksel_strerror.restype = ctypes.c_char_p
 _lib.ksel_launch_count.restype = _i64
+_lib.ksel_ipc_handle_size.restype = _sz
+_lib.ksel_ipc_alloc.argtypes = [_sz, ctypes.POINTER(ctypes.c_void_p), _p]
+_lib.ksel_ipc_open.argtypes = [_p, ctypes.POINTER(ctypes.c_void_p)]
+_lib.ksel_ipc_close.argtypes = [_p]
+_lib.ksel_ipc_free.argtypes = [_p]
+_lib.ksel_flag_signal.argtypes = [_p, ctypes.c_uint32, _p]
+_lib.ksel_flag_wait.argtypes = [_p, _i32, ctypes.c_uint32, _p]
+_lib.ksel_merge_lists.argtypes = [_p, _p, _i32, _i64, _i32, _i32, _p, _p, _p, ctypes.c_uint32, _p]
+for _f in (_lib.ksel_ipc_alloc, _lib.ksel_ipc_open, _lib.ksel_ipc_close, _lib.ksel_ipc_free, _lib.ksel_flag_signal,
+           _lib.ksel_flag_wait, _lib.ksel_merge_lists):
+    _f.restype = ctypes.c_int
 for _f in (_lib.ksel_select, _lib.ksel_select_config, _lib.ksel_select_host, _lib.ksel_merge, _lib.knn_search, _lib.ksel_version):
     _f.restype = ctypes.c_int
 
@@ -65,7 +79,8 @@ KSEL_MAX_K = 1024
 ALGO_AUTO, ALGO_QUEUE, ALGO_POOL = 0, 1, 2
 EXPORTS = ("ksel_select", "ksel_select_workspace", "ksel_select_ex", "ksel_select_config", "ksel_select_host_workspace", "ksel_select_host", "ksel_merge",
            "knn_search_workspace", "knn_search", "knn_graph_workspace", "knn_graph", "knn_distances_workspace", "knn_distances", "ksel_timing_enable", "ksel_timing_collect", "ksel_strerror",
-           "ksel_version", "ksel_launch_count")
+           "ksel_version", "ksel_launch_count", "ksel_ipc_handle_size", "ksel_ipc_alloc", "ksel_ipc_open",
+           "ksel_ipc_close", "ksel_ipc_free", "ksel_flag_signal", "ksel_flag_wait", "ksel_merge_lists")
 
 
 class KselError(RuntimeError):
@@ -266,3 +281,73 @@ def knn_distances(ref: torch.Tensor, query: torch.Tensor, out: torch.Tensor | No
         _check("knn_distances", _lib.knn_distances(ref.data_ptr(), query.data_ptr(), N, Q, D, out.data_ptr(),
                                                    ws.data_ptr(), ws.numel(), _stream(ref.device)))
     return out
+
+
+# ---- collective-free exchange (ksel_ipc_*, ksel_flag_*, ksel_merge_lists) ----
+
+class _CudaMem:
+    """__cuda_array_interface__ over a raw device pointer (no ownership)."""
+
+    def __init__(self, ptr: int, nbytes: int):
+        self.__cuda_array_interface__ = {"shape": (nbytes,), "typestr": "|u1", "data": (ptr, False),
+                                         "version": 2, "strides": None}
+
+
+def device_bytes(ptr: int, nbytes: int) -> torch.Tensor:
+    """A uint8 CUDA tensor viewing [ptr, ptr + nbytes) of the current device (no copy)."""
+    return torch.as_tensor(_CudaMem(ptr, nbytes), device="cuda")
+
+
+def ipc_alloc(nbytes: int):
+    """(device pointer, handle bytes) of a fresh zero-filled exportable allocation."""
+    h = ctypes.create_string_buffer(int(_lib.ksel_ipc_handle_size()))
+    p = ctypes.c_void_p()
+    _check("ksel_ipc_alloc", _lib.ksel_ipc_alloc(nbytes, ctypes.byref(p), h))
+    return int(p.value), bytes(h.raw)
+
+
+def ipc_open(handle: bytes) -> int:
+    p = ctypes.c_void_p()
+    _check("ksel_ipc_open", _lib.ksel_ipc_open(handle, ctypes.byref(p)))
+    return int(p.value)
+
+
+def ipc_close(ptr: int) -> None:
+    _check("ksel_ipc_close", _lib.ksel_ipc_close(ptr))
+
+
+def ipc_free(ptr: int) -> None:
+    _check("ksel_ipc_free", _lib.ksel_ipc_free(ptr))
+
+
+def _ptr_array(ptrs):
+    return (ctypes.c_void_p * len(ptrs))(*[int(x) for x in ptrs])
+
+
+def flag_signal(flag_ptr: int, value: int) -> None:
+    """Stream-ordered release store of `value` to a u32 flag (local or peer memory)."""
+    _check("ksel_flag_signal", _lib.ksel_flag_signal(flag_ptr, value & 0xFFFFFFFF,
+                                                     torch.cuda.current_stream().cuda_stream))
+
+
+def flag_wait(flag_ptrs, value: int) -> None:
+    """Later work on the current stream waits until every flag reached `value`."""
+    arr = _ptr_array(flag_ptrs)
+    _check("ksel_flag_wait", _lib.ksel_flag_wait(arr, len(flag_ptrs), value & 0xFFFFFFFF,
+                                                 torch.cuda.current_stream().cuda_stream))
+
+
+def ksel_merge_lists(val_ptrs, idx_ptrs, Q: int, kin: int, k: int, out_val: torch.Tensor, out_idx: torch.Tensor,
+                     ready_ptrs=None, epoch: int = 0):
+    """ksel_merge over pointer tables: list s of query q at val_ptrs[s] + 4*q*kin (device pointers)."""
+    S = len(val_ptrs)
+    if len(idx_ptrs) != S or (ready_ptrs is not None and len(ready_ptrs) != S):
+        raise ValueError("pointer tables differ in length")
+    if out_val.shape != (Q, k) or out_idx.shape != (Q, k) or out_val.dtype != torch.float32 \
+            or out_idx.dtype != torch.int32 or not out_val.is_contiguous() or not out_idx.is_contiguous():
+        raise TypeError("out_val/out_idx must be contiguous [Q, k] float32/int32 tensors")
+    rd = _ptr_array(ready_ptrs) if ready_ptrs is not None else None
+    _check("ksel_merge_lists", _lib.ksel_merge_lists(_ptr_array(val_ptrs), _ptr_array(idx_ptrs), S, Q, kin, k,
+                                                     out_val.data_ptr(), out_idx.data_ptr(), rd,
+                                                     epoch & 0xFFFFFFFF, torch.cuda.current_stream().cuda_stream))
+    return out_val, out_idx

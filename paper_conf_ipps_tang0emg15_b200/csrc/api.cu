@@ -305,7 +305,12 @@ int ksel_merge(const float* cand_val, const int32_t* cand_idx, int64_t Q, int S,
     DevInfo di;
     int st = current_device_info(&di);
     if (st) return st;
-    cudaError_t e = launch_merge(cand_val, cand_idx, Q, S, kin, k, out_val, out_idx, (cudaStream_t)stream);
+    MergeLists L{};
+    for (int s = 0; s < S; ++s) {
+        L.v[s] = cand_val + (int64_t)s * Q * kin;
+        L.i[s] = cand_idx + (int64_t)s * Q * kin;
+    }
+    cudaError_t e = launch_merge(L, Q, S, kin, k, out_val, out_idx, (cudaStream_t)stream);
     return e == cudaSuccess ? KSEL_OK : KSEL_ERR_CUDA;
 }
 

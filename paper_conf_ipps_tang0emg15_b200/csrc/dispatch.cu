@@ -55,9 +55,9 @@ cudaError_t launch_select_pool(const float* dist, int64_t Q, int64_t N, int k, f
     KSEL_DISPATCH_R(launch_pool_r, queue_regs(k), dist, Q, N, k, ov, oi, wpr, seg, stream)
 }
 
-cudaError_t launch_merge(const float* cv, const int32_t* ci, int64_t Q, int S, int kin, int k, float* ov,
-                         int32_t* oi, cudaStream_t stream) {
-    KSEL_DISPATCH_R(launch_merge_r, queue_regs(k), cv, ci, Q, S, kin, k, ov, oi, stream)
+cudaError_t launch_merge(const MergeLists& L, int64_t Q, int S, int kin, int k, float* ov, int32_t* oi,
+                         cudaStream_t stream) {
+    KSEL_DISPATCH_R(launch_merge_r, queue_regs(k), L, Q, S, kin, k, ov, oi, stream)
 }
 
 cudaError_t launch_merge_pools(const unsigned long long* pools, int64_t P, const int32_t* cnt, int S, int64_t Q,

@@ -51,9 +51,20 @@ struct SegMap {
 cudaError_t launch_select_pool(const float* dist, int64_t Q, int64_t N, int k, float* out_val, int32_t* out_idx,
                                int wpr, cudaStream_t stream, SegMap seg = SegMap());
 
-// Merge of S sorted candidate lists (merge.cu).
-cudaError_t launch_merge(const float* cand_val, const int32_t* cand_idx, int64_t Q, int S, int kin,
-                         int k, float* out_val, int32_t* out_idx, cudaStream_t stream);
+// Merge of S sorted candidate lists (merge.cu).  List s of query q is
+// v[s] + q * kin / i[s] + q * kin (lists may live in different allocations, e.g.
+// peers' memory); ready[s] (optional) is waited for (>= epoch, acquire at system
+// scope) before list s is read, vol selects volatile loads (re-filled peer lists).
+constexpr int kMaxLists = 64;
+struct MergeLists {
+    const float* v[kMaxLists];
+    const int32_t* i[kMaxLists];
+    const uint32_t* ready[kMaxLists];
+    uint32_t epoch;
+    int vol;
+};
+cudaError_t launch_merge(const MergeLists& L, int64_t Q, int S, int kin, int k, float* out_val, int32_t* out_idx,
+                         cudaStream_t stream);
 
 // Top-k per query of the S split pools of the fused k-NN (merge.cu).
 cudaError_t launch_merge_pools(const unsigned long long* pools, int64_t P, const int32_t* cnt, int S, int64_t Q,
@@ -68,8 +79,8 @@ template <int R>
 cudaError_t launch_pool_r(const float* dist, int64_t Q, int64_t N, int k, float* ov, int32_t* oi, int wpr,
                           SegMap seg, cudaStream_t stream);
 template <int R>
-cudaError_t launch_merge_r(const float* cv, const int32_t* ci, int64_t Q, int S, int kin, int k, float* ov,
-                           int32_t* oi, cudaStream_t stream);
+cudaError_t launch_merge_r(const MergeLists& L, int64_t Q, int S, int kin, int k, float* ov, int32_t* oi,
+                           cudaStream_t stream);
 template <int R>
 cudaError_t launch_merge_pools_r(const unsigned long long* pools, int64_t P, const int32_t* cnt, int S, int64_t Q,
                                  const unsigned long long* thr, int k, int64_t idx_offset, float* ov, int32_t* oi,

@@ -42,28 +42,48 @@ __device__ __forceinline__ bool warr_is_sorted(const WArr<RL>& a, uint32_t lane)
     return !__any_sync(kFull, bad);
 }
 
-// Bits of the candidate (key, idx) of query q in the [S][Q][kin] lists: lanes take
+// Loads of list elements: through the read-only path for local lists; for lists in
+// a peer's memory that are re-filled every step (ksel_merge_lists with ready flags),
+// volatile (.cv) loads, so no stale line of an earlier step is ever used.
+__device__ __forceinline__ float ld_val(const MergeLists& L, const float* p) { return L.vol ? __ldcv(p) : __ldg(p); }
+__device__ __forceinline__ int32_t ld_idx(const MergeLists& L, const int32_t* p) { return L.vol ? __ldcv(p) : __ldg(p); }
+
+// Wait (one lane, acquire at system scope) until list s of this step is published.
+__device__ __forceinline__ void wait_ready(const MergeLists& L, int s) {
+    if (L.ready[s] == nullptr) return;
+    if (lane_id() == 0) {
+        uint32_t v;
+        while (true) {
+            asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(L.ready[s]) : "memory");
+            if ((int32_t)(v - L.epoch) >= 0) break;
+            __nanosleep(256);
+        }
+    }
+    __syncwarp();
+}
+
+// Bits of the candidate (key, idx) of query q in the S lists: lanes take
 // lists, binary search for the lexicographic lower bound of (key, idx) in a sorted
 // list (8-10 dependent loads); a warp-wide linear scan if no list has it at the
 // searched position (unsorted input lists).  Warp-uniform result.
-static __device__ __noinline__ uint32_t regather_bits(const float* __restrict__ cv, const int32_t* __restrict__ ci, int64_t q,
-                                               int64_t Q, int S, int kin, uint32_t key, uint32_t idx,
-                                               uint32_t lane) {
+static __device__ __noinline__ uint32_t regather_bits(const MergeLists& L, int64_t q, int S, int kin, uint32_t key,
+                                                      uint32_t idx, uint32_t lane) {
     for (int s0 = 0; s0 < S; s0 += 32) {
         const int s = s0 + (int)lane;
         bool hit = false;
         uint32_t hb = 0;
         if (s < S) {
-            const int64_t base = ((int64_t)s * Q + q) * kin;
+            const float* cv = L.v[s] + q * kin;
+            const int32_t* ci = L.i[s] + q * kin;
             int lo = 0, hi = kin;  // first position not below (key, idx)
             while (lo < hi) {
                 const int mid = (lo + hi) >> 1;
-                if (pair_lt(key_of(cv[base + mid]), (uint32_t)ci[base + mid], key, idx)) lo = mid + 1;
+                if (pair_lt(key_of(ld_val(L, cv + mid)), (uint32_t)ld_idx(L, ci + mid), key, idx)) lo = mid + 1;
                 else hi = mid;
             }
-            if (lo < kin && (uint32_t)ci[base + lo] == idx && key_of(cv[base + lo]) == key) {
+            if (lo < kin && (uint32_t)ld_idx(L, ci + lo) == idx && key_of(ld_val(L, cv + lo)) == key) {
                 hit = true;
-                hb = __float_as_uint(cv[base + lo]);
+                hb = __float_as_uint(ld_val(L, cv + lo));
             }
         }
         const uint32_t m = __ballot_sync(kFull, hit);
@@ -75,9 +95,10 @@ static __device__ __noinline__ uint32_t regather_bits(const float* __restrict__ 
         bool hit = false;
         uint32_t hb = 0;
         if (t < total) {
-            const int64_t a = ((t / kin) * Q + q) * kin + t % kin;
-            hit = (uint32_t)ci[a] == idx && key_of(cv[a]) == key;
-            hb = __float_as_uint(cv[a]);
+            const int64_t a = q * kin + t % kin;
+            const int s = (int)(t / kin);
+            hit = (uint32_t)ld_idx(L, L.i[s] + a) == idx && key_of(ld_val(L, L.v[s] + a)) == key;
+            hb = __float_as_uint(ld_val(L, L.v[s] + a));
         }
         const uint32_t m = __ballot_sync(kFull, hit);
         if (m) return __shfl_sync(kFull, hb, __ffs(m) - 1);
@@ -87,8 +108,8 @@ static __device__ __noinline__ uint32_t regather_bits(const float* __restrict__ 
 
 template <int R, int RL>
 __global__ void __launch_bounds__(32 * kMergeWarps)
-    ksel_merge_kernel(const float* __restrict__ cv, const int32_t* __restrict__ ci, int64_t Q, int S, int kin,
-                      int k, float* __restrict__ out_val, int32_t* __restrict__ out_idx) {
+    ksel_merge_kernel(const __grid_constant__ MergeLists L, int64_t Q, int S, int kin, int k,
+                      float* __restrict__ out_val, int32_t* __restrict__ out_idx) {
     const uint32_t lane = lane_id();
     const int64_t q = (int64_t)blockIdx.x * kMergeWarps + (threadIdx.x >> 5);
     if (q >= Q) return;
@@ -98,7 +119,9 @@ __global__ void __launch_bounds__(32 * kMergeWarps)
     warr_fill_sentinel<R>(acc);
 #pragma unroll 1
     for (int s = 0; s < S; ++s) {
-        const int64_t base = ((int64_t)s * Q + q) * kin;
+        wait_ready(L, s);
+        const float* cv = L.v[s] + q * kin;
+        const int32_t* ci = L.i[s] + q * kin;
         // A list longer than k' is folded in whole, k' at a time (only its k'
         // smallest can matter, but finding them must not assume sortedness).
 #pragma unroll 1
@@ -107,8 +130,8 @@ __global__ void __launch_bounds__(32 * kMergeWarps)
 #pragma unroll
             for (int r = 0; r < RL; ++r) {
                 const int e = off + r * 32 + (int)lane;
-                b.k[r] = (e < kin) ? key_of(cv[base + e]) : kSentKey;
-                b.i[r] = (e < kin) ? (uint32_t)ci[base + e] : kSentIdx;
+                b.k[r] = (e < kin) ? key_of(ld_val(L, cv + e)) : kSentKey;
+                b.i[r] = (e < kin) ? (uint32_t)ld_idx(L, ci + e) : kSentIdx;
             }
             const bool sorted = (kin <= LN) && warr_is_sorted<RL>(b, lane);
             if (!sorted) warr_sort<RL>(b, lane);
@@ -130,7 +153,7 @@ __global__ void __launch_bounds__(32 * kMergeWarps)
         while (need) {
             const int j = __ffs(need) - 1;
             need &= need - 1u;
-            const uint32_t b = regather_bits(cv, ci, q, Q, S, kin, __shfl_sync(kFull, key, j),
+            const uint32_t b = regather_bits(L, q, S, kin, __shfl_sync(kFull, key, j),
                                              __shfl_sync(kFull, idx, j), lane);
             if ((int)lane == j) bits = b;
         }
@@ -142,26 +165,26 @@ __global__ void __launch_bounds__(32 * kMergeWarps)
 }
 
 template <int R, int RL>
-static cudaError_t launch_merge_rl(const float* cv, const int32_t* ci, int64_t Q, int S, int kin, int k, float* ov,
-                                   int32_t* oi, cudaStream_t stream) {
+static cudaError_t launch_merge_rl(const MergeLists& L, int64_t Q, int S, int kin, int k, float* ov, int32_t* oi,
+                                   cudaStream_t stream) {
     const int64_t grid = (Q + kMergeWarps - 1) / kMergeWarps;
-    ksel_merge_kernel<R, RL><<<(unsigned)grid, 32 * kMergeWarps, 0, stream>>>(cv, ci, Q, S, kin, k, ov, oi);
+    ksel_merge_kernel<R, RL><<<(unsigned)grid, 32 * kMergeWarps, 0, stream>>>(L, Q, S, kin, k, ov, oi);
     note_launch();
     return cudaGetLastError();
 }
 
 template <int R>
-cudaError_t launch_merge_r(const float* cv, const int32_t* ci, int64_t Q, int S, int kin, int k, float* ov,
-                                  int32_t* oi, cudaStream_t stream) {
+cudaError_t launch_merge_r(const MergeLists& L, int64_t Q, int S, int kin, int k, float* ov, int32_t* oi,
+                           cudaStream_t stream) {
     const int lp = kin <= 32 ? 1 : kin <= 64 ? 2 : kin <= 128 ? 4 : kin <= 256 ? 8 : kin <= 512 ? 16 : 32;
     const int rl = lp < R ? lp : R;
     switch (rl) {
-        case 1: return launch_merge_rl<R, 1>(cv, ci, Q, S, kin, k, ov, oi, stream);
-        case 2: if constexpr (R >= 2) return launch_merge_rl<R, 2>(cv, ci, Q, S, kin, k, ov, oi, stream); break;
-        case 4: if constexpr (R >= 4) return launch_merge_rl<R, 4>(cv, ci, Q, S, kin, k, ov, oi, stream); break;
-        case 8: if constexpr (R >= 8) return launch_merge_rl<R, 8>(cv, ci, Q, S, kin, k, ov, oi, stream); break;
-        case 16: if constexpr (R >= 16) return launch_merge_rl<R, 16>(cv, ci, Q, S, kin, k, ov, oi, stream); break;
-        case 32: if constexpr (R >= 32) return launch_merge_rl<R, 32>(cv, ci, Q, S, kin, k, ov, oi, stream); break;
+        case 1: return launch_merge_rl<R, 1>(L, Q, S, kin, k, ov, oi, stream);
+        case 2: if constexpr (R >= 2) return launch_merge_rl<R, 2>(L, Q, S, kin, k, ov, oi, stream); break;
+        case 4: if constexpr (R >= 4) return launch_merge_rl<R, 4>(L, Q, S, kin, k, ov, oi, stream); break;
+        case 8: if constexpr (R >= 8) return launch_merge_rl<R, 8>(L, Q, S, kin, k, ov, oi, stream); break;
+        case 16: if constexpr (R >= 16) return launch_merge_rl<R, 16>(L, Q, S, kin, k, ov, oi, stream); break;
+        case 32: if constexpr (R >= 32) return launch_merge_rl<R, 32>(L, Q, S, kin, k, ov, oi, stream); break;
     }
     return cudaErrorInvalidValue;
 }
@@ -260,7 +283,7 @@ template cudaError_t launch_merge_pools_r<KSEL_ONLY_R>(const unsigned long long*
                                                        int64_t, const unsigned long long*, int, int64_t, float*,
                                                        int32_t*, cudaStream_t);
 
-template cudaError_t launch_merge_r<KSEL_ONLY_R>(const float*, const int32_t*, int64_t, int, int, int, float*,
-                                                 int32_t*, cudaStream_t);
+template cudaError_t launch_merge_r<KSEL_ONLY_R>(const MergeLists&, int64_t, int, int, int, float*, int32_t*,
+                                                 cudaStream_t);
 
 }  // namespace ksel

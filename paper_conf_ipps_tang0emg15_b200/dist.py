@@ -84,3 +84,106 @@ def knn_search_sharded(ref_shard: torch.Tensor, query: torch.Tensor, k: int, n_t
     cand_idx = cand[..., 1].contiguous()
     mv, mi = merge(cand_val, cand_idx, k)
     return mv, mi, (q0, q1)
+
+
+# ---------------------------------------------------------------------------
+# Collective-free exchange: the merge reads peers' lists
+# ---------------------------------------------------------------------------
+
+_P2P_HDR = 512  # bytes: ready[2] u32 at 0, consumed[world <= 64] u32 at 64
+
+
+def p2p_layout(Q: int, k: int, world: int) -> dict:
+    """Byte offsets inside each rank's exchange buffer.
+
+    ``ready(b)``: u32 epoch flag of double buffer b (written by the owner);
+    ``consumed(s)``: u32 epoch flag written by rank s once it merged the owner's
+    lists; ``val(b)`` / ``idx(b)``: the owner's [Q][k] fp32 / int32 top-k lists.
+    """
+    if not 1 <= world <= 64:
+        raise ValueError("world size must be in [1, 64]")
+    lst = Q * k * 4
+    return {
+        "ready": lambda b: 4 * b,
+        "consumed": lambda s: 64 + 4 * s,
+        "val": lambda b: _P2P_HDR + b * 2 * lst,
+        "idx": lambda b: _P2P_HDR + b * 2 * lst + lst,
+        "bytes": _P2P_HDR + 4 * lst,
+    }
+
+
+class KnnP2P:
+    """Row-sharded k-NN whose exchange is the merge reading peers' memory.
+
+    One exportable buffer per rank (``ipc_alloc``) holds two epochs of its
+    [Q][k] candidate lists plus flags; handles are exchanged once over the
+    process group and mapped with CUDA IPC (NVLink / NVSwitch peer memory; on a
+    single GPU, several processes share it the same way).  Per call (epoch e,
+    buffer b = e % 2), all stream-ordered on the current stream, no host sync:
+
+    1. (e >= 2) wait until every rank consumed epoch e - 2 of this buffer;
+    2. ``knn_search`` of the local shard (global indices) into buffer b;
+    3. signal ready[b] = e + 1;
+    4. ``ksel_merge_lists`` over the g lists of this rank's query slice,
+       straight from the peers' buffers, each list waited for (ready >= e + 1);
+    5. signal consumed[rank] = e + 1 in every peer's buffer.
+
+    Same result as :func:`knn_search_sharded` (bit-identical to unsharded).
+    """
+
+    def __init__(self, Q: int, k: int, n_total: int, group=None, local_knn=None):
+        from . import ipc_alloc, ipc_open
+        self.group = group
+        self.world = tdist.get_world_size(group)
+        self.rank = tdist.get_rank(group)
+        self.Q, self.k, self.n_total = Q, k, n_total
+        self.lay = p2p_layout(Q, k, self.world)
+        self.local_knn = local_knn
+        self.base, handle = ipc_alloc(self.lay["bytes"])
+        torch.cuda.synchronize()
+        handles = [None] * self.world
+        tdist.all_gather_object(handles, handle, group=group)
+        self.peer = [self.base if s == self.rank else ipc_open(handles[s]) for s in range(self.world)]
+        tdist.barrier(group=group)
+        self.epoch = 0
+
+    def __call__(self, ref_shard: torch.Tensor, query: torch.Tensor):
+        from . import device_bytes, flag_signal, flag_wait, ksel_merge_lists
+        L, e, Q, k = self.lay, self.epoch, self.Q, self.k
+        b = e & 1
+        r0, r1 = shard_range(self.n_total, self.world, self.rank)
+        assert ref_shard.shape[0] == r1 - r0 and query.shape[0] == Q
+        if e >= 2:  # buffer b was last filled at epoch e - 2: all ranks must be done reading it
+            flag_wait([self.base + L["consumed"](s) for s in range(self.world)], e - 1)
+        own = device_bytes(self.base, L["bytes"])
+        ov = own[L["val"](b): L["val"](b) + Q * k * 4].view(torch.float32).view(Q, k)
+        oi = own[L["idx"](b): L["idx"](b) + Q * k * 4].view(torch.int32).view(Q, k)
+        if self.local_knn is None:  # the library writes straight into the exchange buffer
+            from . import knn_search
+            knn_search(ref_shard, query, k, idx_offset=r0, out_dist=ov, out_idx=oi)
+        else:
+            v, i = self.local_knn(ref_shard, query, k, r0)
+            ov.copy_(v)
+            oi.copy_(i)
+        flag_signal(self.base + L["ready"](b), e + 1)
+        q0, q1 = shard_range(Q, self.world, self.rank)
+        mv = torch.empty((q1 - q0, k), dtype=torch.float32, device=query.device)
+        mi = torch.empty((q1 - q0, k), dtype=torch.int32, device=query.device)
+        if q1 > q0:
+            ksel_merge_lists([p + L["val"](b) + q0 * k * 4 for p in self.peer],
+                             [p + L["idx"](b) + q0 * k * 4 for p in self.peer], q1 - q0, k, k, mv, mi,
+                             ready_ptrs=[p + L["ready"](b) for p in self.peer], epoch=e + 1)
+        for p in self.peer:
+            flag_signal(p + L["consumed"](self.rank), e + 1)
+        self.epoch += 1
+        return mv, mi, (q0, q1)
+
+    def close(self):
+        from . import ipc_close, ipc_free
+        torch.cuda.synchronize()
+        tdist.barrier(group=self.group)
+        for s, p in enumerate(self.peer):
+            if s != self.rank:
+                ipc_close(p)
+        tdist.barrier(group=self.group)
+        ipc_free(self.base)

@@ -88,3 +88,18 @@ def test_query_rows_partition():
             assert spans[0][0] == 0 and spans[-1][1] == Q
             assert all(spans[r][1] == spans[r + 1][0] for r in range(world - 1))
             assert max(b - a for a, b in spans) - min(b - a for a, b in spans) <= 1
+
+
+def test_p2p_layout_regions_disjoint():
+    from paper_conf_ipps_tang0emg15_b200 import dist
+    for Q, k, world in [(1, 1, 1), (1000, 100, 8), (10000, 1024, 64), (7, 3, 5)]:
+        L = dist.p2p_layout(Q, k, world)
+        spans = [(L["ready"](b), 4) for b in range(2)] + [(L["consumed"](s), 4) for s in range(world)]
+        spans += [(L["val"](b), Q * k * 4) for b in range(2)] + [(L["idx"](b), Q * k * 4) for b in range(2)]
+        spans.sort()
+        for (a, n), (b_, _) in zip(spans, spans[1:]):
+            assert a + n <= b_
+        assert spans[-1][0] + spans[-1][1] <= L["bytes"]
+        assert all(off % 4 == 0 for off, _ in spans)
+    with pytest.raises(ValueError):
+        dist.p2p_layout(10, 10, 65)
