@@ -90,12 +90,18 @@ KSEL_API int ksel_select_ex(const float* dist, int64_t Q, int64_t N, int k, floa
  *                  warp-register bitonic queue at every buffer flush (Merge Queue +
  *                  Buffered Search), KSEL_ALGO_POOL (2):
  *                  candidate pool narrowed by radix-histogram select (Hierarchical
- *                  Partition's discard-by-group, L221-L231, with value buckets).
- *   warps_per_row  0 = automatic, else 1, 2, 4 or 8 warps cooperating on each row.
+ *                  Partition's discard-by-group, L221-L231, with value buckets),
+ *                  KSEL_ALGO_RADIX (3): N <= 65536 only (else KSEL_ERR_UNSUPPORTED):
+ *                  a cluster of <= 8 CTAs holds the row in registers and narrows
+ *                  the exact k-th key by four 8-bit radix passes over all of it
+ *                  (HP's value buckets, L225), then sorts the k selected pairs.
+ *   warps_per_row  0 = automatic, else 1, 2, 4 or 8 warps cooperating on each row
+ *                  (ignored by KSEL_ALGO_RADIX).
  * Other arguments as ksel_select; invalid algo / warps_per_row -> INVALID_ARG. */
 #define KSEL_ALGO_AUTO 0
 #define KSEL_ALGO_QUEUE 1
 #define KSEL_ALGO_POOL 2
+#define KSEL_ALGO_RADIX 3
 KSEL_API int ksel_select_config(const float* dist, int64_t Q, int64_t N, int k, float* out_val,
                                 int32_t* out_idx, int algo, int warps_per_row, void* stream);
 
@@ -196,7 +202,12 @@ KSEL_API int knn_distances(const float* ref, const float* query, int64_t N, int6
  *   knn_search emits it; indices unique per query across lists.  With ready
  *   != NULL, list s is read only after *ready[s] reached `epoch` (as in
  *   ksel_flag_wait), with volatile loads.  Output, limits and errors as
- *   ksel_merge. */
+ *   ksel_merge.
+ * Waits that do not complete within 60 s trap (the stream then reports a CUDA
+ * error) rather than hang.  Every kernel taking part in such an exchange must
+ * already be loaded when a wait is pending (CUDA lazy loading may otherwise
+ * serialise behind the spinning wait): run one warm-up call first, as KnnP2P
+ * does. */
 KSEL_API size_t ksel_ipc_handle_size(void);
 KSEL_API int ksel_ipc_alloc(size_t bytes, void** d_ptr, void* handle_out);
 KSEL_API int ksel_ipc_open(const void* handle, void** d_ptr);

@@ -76,7 +76,7 @@ for _f in (_lib.ksel_select, _lib.ksel_select_config, _lib.ksel_select_host, _li
     _f.restype = ctypes.c_int
 
 KSEL_MAX_K = 1024
-ALGO_AUTO, ALGO_QUEUE, ALGO_POOL = 0, 1, 2
+ALGO_AUTO, ALGO_QUEUE, ALGO_POOL, ALGO_RADIX = 0, 1, 2, 3
 EXPORTS = ("ksel_select", "ksel_select_workspace", "ksel_select_ex", "ksel_select_config", "ksel_select_host_workspace", "ksel_select_host", "ksel_merge",
            "knn_search_workspace", "knn_search", "knn_graph_workspace", "knn_graph", "knn_distances_workspace", "knn_distances", "ksel_timing_enable", "ksel_timing_collect", "ksel_strerror",
            "ksel_version", "ksel_launch_count", "ksel_ipc_handle_size", "ksel_ipc_alloc", "ksel_ipc_open",

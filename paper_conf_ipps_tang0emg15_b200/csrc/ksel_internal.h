@@ -51,6 +51,11 @@ struct SegMap {
 cudaError_t launch_select_pool(const float* dist, int64_t Q, int64_t N, int k, float* out_val, int32_t* out_idx,
                                int wpr, cudaStream_t stream, SegMap seg = SegMap());
 
+// Cluster radix selection for rows of <= 65536 values (select_radix.cu).
+bool radix_supported(int64_t N, int k);
+cudaError_t launch_select_radix(const float* dist, int64_t Q, int64_t N, int k, float* out_val, int32_t* out_idx,
+                                cudaStream_t stream);
+
 // Merge of S sorted candidate lists (merge.cu).  List s of query q is
 // v[s] + q * kin / i[s] + q * kin (lists may live in different allocations, e.g.
 // peers' memory); ready[s] (optional) is waited for (>= epoch, acquire at system

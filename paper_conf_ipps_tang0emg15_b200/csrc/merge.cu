@@ -53,10 +53,12 @@ __device__ __forceinline__ void wait_ready(const MergeLists& L, int s) {
     if (L.ready[s] == nullptr) return;
     if (lane_id() == 0) {
         uint32_t v;
+        const uint64_t t0 = globaltimer_ns();
         while (true) {
             asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(L.ready[s]) : "memory");
             if ((int32_t)(v - L.epoch) >= 0) break;
             __nanosleep(256);
+            if (globaltimer_ns() - t0 > kFlagTimeoutNs) __trap();  // a producer that never signals: fail loudly
         }
     }
     __syncwarp();

@@ -44,10 +44,12 @@ __global__ void flag_wait_kernel(const __grid_constant__ FlagSet fs, int n, uint
     const int j = (int)threadIdx.x;
     if (j < n) {
         uint32_t v;
+        const uint64_t t0 = globaltimer_ns();
         while (true) {
             asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(fs.f[j]) : "memory");
             if ((int32_t)(v - value) >= 0) break;
             __nanosleep(500);
+            if (globaltimer_ns() - t0 > kFlagTimeoutNs) __trap();  // a peer that never signals: fail loudly
         }
     }
     __syncthreads();

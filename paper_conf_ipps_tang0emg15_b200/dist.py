@@ -146,6 +146,24 @@ class KnnP2P:
         self.peer = [self.base if s == self.rank else ipc_open(handles[s]) for s in range(self.world)]
         tdist.barrier(group=group)
         self.epoch = 0
+        self.warm = False
+
+    def _warm_up(self, D: int, device):
+        # Load every kernel the exchange uses before any cross-process wait is pending:
+        # with CUDA lazy loading, a module load may otherwise queue behind a spinning wait.
+        from . import flag_signal, flag_wait, knn_search, ksel_merge_lists
+        k = self.k
+        ref = torch.zeros((max(k, 32), D), dtype=torch.float32, device=device)
+        v, i = knn_search(ref, ref[:1].contiguous(), k)
+        scratch = torch.zeros(1, dtype=torch.int32, device=device)
+        flag_signal(scratch.data_ptr(), 0)
+        flag_wait([scratch.data_ptr()], 0)
+        mv = torch.empty((1, k), dtype=torch.float32, device=device)
+        mi = torch.empty((1, k), dtype=torch.int32, device=device)
+        ksel_merge_lists([v.data_ptr()], [i.data_ptr()], 1, k, k, mv, mi, ready_ptrs=[scratch.data_ptr()], epoch=0)
+        torch.cuda.synchronize()
+        tdist.barrier(group=self.group)
+        self.warm = True
 
     def __call__(self, ref_shard: torch.Tensor, query: torch.Tensor):
         from . import device_bytes, flag_signal, flag_wait, ksel_merge_lists
@@ -153,6 +171,8 @@ class KnnP2P:
         b = e & 1
         r0, r1 = shard_range(self.n_total, self.world, self.rank)
         assert ref_shard.shape[0] == r1 - r0 and query.shape[0] == Q
+        if not self.warm:
+            self._warm_up(query.shape[1], query.device)
         if e >= 2:  # buffer b was last filled at epoch e - 2: all ranks must be done reading it
             flag_wait([self.base + L["consumed"](s) for s in range(self.world)], e - 1)
         own = device_bytes(self.base, L["bytes"])

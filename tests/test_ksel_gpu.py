@@ -52,10 +52,11 @@ def test_config1(K, oracle_mod):
     _check_select(K, oracle_mod, x, 32, "C1")
 
 
-@pytest.mark.parametrize("algo", [1, 2])
+@pytest.mark.parametrize("algo", [1, 2, 3])
 @pytest.mark.parametrize("dist", synth.DISTS)
 def test_k_sweep_all_distributions(K, oracle_mod, dist, algo):
-    # both kernel variants: 1 = bitonic queue per flush, 2 = pool + radix narrowing
+    # every kernel variant: 1 = bitonic queue per flush, 2 = pool + radix narrowing,
+    # 3 = cluster radix select (row in registers)
     x = synth.rows(dist, synth.seed_for(7, dist), 0, 48, 5003)  # ragged N (N % 4 != 0)
     for k in KS:
         _check_select(K, oracle_mod, x, k, "%s k=%d algo=%d" % (dist, k, algo), algo=algo)
@@ -86,6 +87,36 @@ def test_forced_warps_per_row(K, oracle_mod, wpr, algo):
             _check_select(K, oracle_mod, x, k, "%s wpr=%d algo=%d k=%d" % (dist, wpr, algo, k), algo, wpr)
 
 
+@pytest.mark.parametrize("N", [1, 3, 31, 1025, 8191, 8192, 8193, 16385, 24576 + 7, 40000, 57343, 65535, 65536])
+def test_radix_cluster_sizes(K, oracle_mod, N):
+    # KSEL_ALGO_RADIX: clusters of 1..8 CTAs (8192 values each), ragged and aligned rows,
+    # ties cut inside a CTA and across CTAs (T), specials (X), sorted rows
+    for dist in ("U", "T", "X", "SD", "DG"):
+        x = synth.rows(dist, 123, 0, 5, N)
+        for k in sorted({1, min(N, 2), min(N, 33), min(N, 256), min(N, 1000), min(N, 1024)}):
+            _check_select(K, oracle_mod, x, k, "radix %s N=%d k=%d" % (dist, N, k), algo=3)
+
+
+def test_radix_all_equal_and_unsupported(K, oracle_mod):
+    x = torch.full((3, 65536), 7.0)
+    x[1, 1000:] = -0.0
+    x[2, ::3] = float("nan")
+    for k in (1, 100, 1024):
+        _check_select(K, oracle_mod, x, k, "radix equal k=%d" % k, algo=3)
+    with pytest.raises(K.KselError):
+        K.ksel_select(torch.zeros((2, 65537), device="cuda"), 10, algo=3)
+
+
+@pytest.mark.parametrize("k", [1, 32, 256, 1024])
+@pytest.mark.parametrize("dist", ["U", "DG", "SD", "T"])
+def test_radix_config2_full_size(K, oracle_mod, dist, k):
+    x = synth.rows(dist, synth.seed_for(2, dist), 0, 1024, 65536, device="cuda")
+    gv, gi = K.ksel_select(x, k, algo=3)
+    torch.cuda.synchronize()
+    ev, ei = oracle_mod.select(x.cpu().numpy(), k)
+    assert_same(ev, ei, gv, gi, "C2 radix %s k=%d" % (dist, k))
+
+
 def test_unaligned_base_pointer(K, oracle_mod):
     # row starts that are not 16-byte aligned, including the base pointer itself
     big = synth.rows("U", 5, 0, 1, 7 * 4099 + 3)[0]
@@ -94,9 +125,10 @@ def test_unaligned_base_pointer(K, oracle_mod):
         xg = big.cuda()[off:off + 7 * 4099].view(7, 4099)
         assert xg.data_ptr() % 16 != 0
         for k in (1, 64, 300):
-            gv, gi = K.ksel_select(xg, k)
-            ev, ei = oracle_mod.select(x_cpu.numpy(), k)
-            assert_same(ev, ei, gv, gi, "off=%d k=%d" % (off, k))
+            for algo in (0, 3):
+                gv, gi = K.ksel_select(xg, k, algo=algo)
+                ev, ei = oracle_mod.select(x_cpu.numpy(), k)
+                assert_same(ev, ei, gv, gi, "off=%d k=%d algo=%d" % (off, k, algo))
 
 
 def test_special_rows(K, oracle_mod):
@@ -109,6 +141,7 @@ def test_special_rows(K, oracle_mod):
     x = torch.from_numpy(np.stack(rows))
     for k in (1, 5, 6, 32, 100, 1024):
         _check_select(K, oracle_mod, x, k, "special k=%d" % k)
+        _check_select(K, oracle_mod, x, k, "special radix k=%d" % k, algo=3)
 
 
 @pytest.mark.parametrize("k", [1, 8, 32, 128, 256, 1024])

@@ -75,6 +75,8 @@ def test_merge_lists_waits_for_ready_flags(K):
     is_[1].fill_(-1)
     flags = torch.zeros(S, dtype=torch.int32, device="cuda")
     K.flag_signal(flags.data_ptr(), 1)
+    torch.cuda._sleep(100)  # load every kernel of the concurrent part first (lazy loading)
+    target_v.copy_(target_v)
     torch.cuda.synchronize()
     ov = torch.empty((Q, k), dtype=torch.float32, device="cuda")
     oi = torch.empty((Q, k), dtype=torch.int32, device="cuda")
@@ -95,6 +97,11 @@ def test_merge_lists_waits_for_ready_flags(K):
 def test_flag_wait_orders_stream(K):
     flag = torch.zeros(1, dtype=torch.int32, device="cuda")
     out = torch.zeros(1, dtype=torch.int32, device="cuda")
+    K.flag_wait([flag.data_ptr()], 0)  # load every kernel of the concurrent part first (lazy loading)
+    K.flag_signal(out.data_ptr(), 0)
+    out.add_(flag)
+    torch.cuda._sleep(100)
+    torch.cuda.synchronize()
     a, b = torch.cuda.Stream(), torch.cuda.Stream()
     with torch.cuda.stream(a):
         K.flag_wait([flag.data_ptr()], 3)
@@ -145,11 +152,12 @@ def test_knn_p2p_processes_on_one_gpu(K, tmp_path, world):
     s.bind(("127.0.0.1", 0))
     port = str(s.getsockname()[1])
     s.close()
-    procs = [subprocess.Popen([sys.executable, "-c", _P2P_SCRIPT, ROOT, str(tmp_path), str(r), str(world), port])
+    procs = [subprocess.Popen([sys.executable, "-c", _P2P_SCRIPT, ROOT, str(tmp_path), str(r), str(world), port],
+                              env=dict(os.environ, CUDA_MODULE_LOADING="EAGER" if world == 3 else "LAZY"))
              for r in range(world)]
     try:
         for p in procs:
-            assert p.wait(timeout=300) == 0
+            assert p.wait(timeout=240) == 0
     finally:
         for p in procs:
             if p.poll() is None:
