@@ -175,6 +175,37 @@ KSEL_API size_t knn_distances_workspace(int64_t N, int64_t Q, int D);
 KSEL_API int knn_distances(const float* ref, const float* query, int64_t N, int64_t Q, int D, float* out,
                            void* d_work, size_t work_bytes, void* stream);
 
+/* ksel_select_paper -- ABLATION, not the hot path: the
+ * paper's own per-thread designs, one thread per query, on B200.
+ *   dist_t   device, [N][Q] fp32: QUERY-CONTIGUOUS (element (q, j) at j*Q + q),
+ *            the layout that makes a thread-per-query scan coalesced (PAPER.md
+ *            L225, L243; reading R10).
+ *   queue    KSEL_PQ_INSERT (sorted array, L37), KSEL_PQ_HEAP (L37),
+ *            KSEL_PQ_MERGE (Merge Queue, Alg. 2, L39-L41, level-1 size m),
+ *            KSEL_PQ_MERGE_ALIGNED (merges taken by the whole warp, L183).
+ *   buffer   KSEL_PB_NONE, KSEL_PB_BUFFER / KSEL_PB_FULL / KSEL_PB_FULL_SORTED
+ *            (Buffered Search, Alg. 3; bsize pairs per thread).
+ *   hp_G     0, or the Hierarchical Partition group size G >= 2 (Alg. 4).
+ *   d_work   device workspace >= ksel_select_paper_workspace(...) bytes (queues,
+ *            buffers and HP levels per thread; 0 returned for invalid arguments).
+ * Output as ksel_select (out_val/out_idx [Q][k], ascending, bit-identical for
+ * every variant).  Errors: INVALID_ARG (bad variant, m not a power of 2 in
+ * [1, 1024], bsize outside [1, 1024], G outside {0} U [2, 64], short workspace),
+ * UNSUPPORTED (k > 1024). */
+#define KSEL_PQ_INSERT 0
+#define KSEL_PQ_HEAP 1
+#define KSEL_PQ_MERGE 2
+#define KSEL_PQ_MERGE_ALIGNED 3
+#define KSEL_PB_NONE 0
+#define KSEL_PB_BUFFER 1
+#define KSEL_PB_FULL 2
+#define KSEL_PB_FULL_SORTED 3
+KSEL_API size_t ksel_select_paper_workspace(int64_t Q, int64_t N, int k, int queue, int buffer, int hp_G, int m,
+                                            int bsize);
+KSEL_API int ksel_select_paper(const float* dist_t, int64_t Q, int64_t N, int k, int queue, int buffer, int hp_G,
+                               int m, int bsize, float* out_val, int32_t* out_idx, void* d_work, size_t work_bytes,
+                               void* stream);
+
 /* ---- Row-sharded k-NN exchange without a collective ----
  * The final merge of the row-sharded k-NN (divide-and-merge)
  * reading every shard's candidate lists in place -- local memory or a peer

@@ -12,6 +12,8 @@ Entry points (same names as the C ABI):
 * :func:`ksel_merge`       -- top-k of the union of S sorted candidate lists.
 * :func:`knn_search`       -- fused distance + selection brute-force k-NN.
 * :func:`knn_graph`        -- k-NN graph of one point set (self excluded).
+* :func:`ksel_select_paper` -- ABLATION: the paper's per-thread queue / buffer / HP
+  designs (query-contiguous input), bit-identical results.
 * :func:`ksel_merge_lists` -- ksel_merge over pointer tables (peer lists, ready flags);
   with :func:`ipc_alloc` / :func:`ipc_open` / :func:`flag_signal` / :func:`flag_wait`
   the collective-free row-sharded k-NN exchange (dist.KnnP2P).
@@ -61,6 +63,10 @@ _lib.ksel_timing_collect.restype = ctypes.c_int
 _lib.ksel_strerror.argtypes = [_i32]
 _lib.ksel_strerror.restype = ctypes.c_char_p
 _lib.ksel_launch_count.restype = _i64
+_lib.ksel_select_paper_workspace.argtypes = [_i64, _i64, _i32, _i32, _i32, _i32, _i32, _i32]
+_lib.ksel_select_paper_workspace.restype = _sz
+_lib.ksel_select_paper.argtypes = [_p, _i64, _i64, _i32, _i32, _i32, _i32, _i32, _i32, _p, _p, _p, _sz, _p]
+_lib.ksel_select_paper.restype = ctypes.c_int
 _lib.ksel_ipc_handle_size.restype = _sz
 _lib.ksel_ipc_alloc.argtypes = [_sz, ctypes.POINTER(ctypes.c_void_p), _p]
 _lib.ksel_ipc_open.argtypes = [_p, ctypes.POINTER(ctypes.c_void_p)]
@@ -77,9 +83,11 @@ for _f in (_lib.ksel_select, _lib.ksel_select_config, _lib.ksel_select_host, _li
 
 KSEL_MAX_K = 1024
 ALGO_AUTO, ALGO_QUEUE, ALGO_POOL, ALGO_RADIX = 0, 1, 2, 3
+PQ_INSERT, PQ_HEAP, PQ_MERGE, PQ_MERGE_ALIGNED = 0, 1, 2, 3
+PB_NONE, PB_BUFFER, PB_FULL, PB_FULL_SORTED = 0, 1, 2, 3
 EXPORTS = ("ksel_select", "ksel_select_workspace", "ksel_select_ex", "ksel_select_config", "ksel_select_host_workspace", "ksel_select_host", "ksel_merge",
            "knn_search_workspace", "knn_search", "knn_graph_workspace", "knn_graph", "knn_distances_workspace", "knn_distances", "ksel_timing_enable", "ksel_timing_collect", "ksel_strerror",
-           "ksel_version", "ksel_launch_count", "ksel_ipc_handle_size", "ksel_ipc_alloc", "ksel_ipc_open",
+           "ksel_version", "ksel_launch_count", "ksel_select_paper_workspace", "ksel_select_paper", "ksel_ipc_handle_size", "ksel_ipc_alloc", "ksel_ipc_open",
            "ksel_ipc_close", "ksel_ipc_free", "ksel_flag_signal", "ksel_flag_wait", "ksel_merge_lists")
 
 
@@ -351,3 +359,23 @@ def ksel_merge_lists(val_ptrs, idx_ptrs, Q: int, kin: int, k: int, out_val: torc
                                                      out_val.data_ptr(), out_idx.data_ptr(), rd,
                                                      epoch & 0xFFFFFFFF, torch.cuda.current_stream().cuda_stream))
     return out_val, out_idx
+
+
+def ksel_select_paper(dist_t: torch.Tensor, k: int, queue: int = PQ_MERGE_ALIGNED, buffer: int = PB_FULL_SORTED,
+                      hp_G: int = 4, m: int = 8, bsize: int = 16, workspace: torch.Tensor | None = None):
+    """ABLATION: the paper's thread-per-query designs.  dist_t is [N, Q]
+    (query-contiguous: column q is query q's row); returns ([Q, k] values, [Q, k] indices)."""
+    _dev_f32(dist_t, "dist_t", 2)
+    N, Q = dist_t.shape
+    need = int(_lib.ksel_select_paper_workspace(Q, N, k, queue, buffer, hp_G, m, bsize))
+    if need == 0:
+        raise KselError("ksel_select_paper_workspace", 1)
+    if workspace is None or workspace.numel() < need:
+        workspace = torch.empty(need, dtype=torch.uint8, device=dist_t.device)
+    ov = torch.empty((Q, k), dtype=torch.float32, device=dist_t.device)
+    oi = torch.empty((Q, k), dtype=torch.int32, device=dist_t.device)
+    with torch.cuda.device(dist_t.device):
+        _check("ksel_select_paper", _lib.ksel_select_paper(dist_t.data_ptr(), Q, N, k, queue, buffer, hp_G, m, bsize,
+                                                           ov.data_ptr(), oi.data_ptr(), workspace.data_ptr(),
+                                                           workspace.numel(), _stream(dist_t.device)))
+    return ov, oi

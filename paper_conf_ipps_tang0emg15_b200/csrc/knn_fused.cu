@@ -80,6 +80,16 @@ struct KnnGeom {
                          // share every reference stage through one multicast load
     int QTp;             // query tiles padded to a multiple of cs (padding tiles select nothing)
     int passes;          // 3 (hi.hi + hi.lo + lo.hi); 1 = hi.hi only (experiments: pipeline timing)
+    int cold_splits;     // leading splits run by first-wave CTAs (no published bound yet)
+    int cold_w;          // their share of the reference tiles relative to the others (per mille)
+    // first logical tile of split s: split s weighs cold_w / 1000 if s < cold_splits, else 1
+    __host__ __device__ int split_begin(int s) const {
+        auto W = [&](int x) -> int64_t {
+            const int c = x < cold_splits ? x : cold_splits;
+            return (int64_t)c * cold_w + (int64_t)(x - c) * 1000;
+        };
+        return (int)((int64_t)ntiles * W(s) / W(S));
+    }
     __host__ __device__ size_t tile_bytes() const { return (size_t)KS * KNN_STAGE_BYTES + KNN_NORM_B_BYTES; }
     __host__ __device__ int a_bytes() const { return Dp * 512 + KNN_NORM_A_BYTES; }
 };
@@ -337,8 +347,8 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
     const int split = blockIdx.x / g.QTp;
     const uint32_t crank = g.cs > 1 ? cluster_rank() : 0u;
     const uint16_t cmask = (uint16_t)((1u << g.cs) - 1u);
-    const int t0 = (int)((int64_t)g.ntiles * split / g.S);  // logical tile range of this CTA
-    const int t1 = (int)((int64_t)g.ntiles * (split + 1) / g.S);
+    const int t0 = g.split_begin(split);  // logical tile range of this CTA
+    const int t1 = g.split_begin(split + 1);
     // Cold CTAs (the first wave: no split of their queries has published a bound
     // yet) first stream their first Fs tiles through the pipeline for a distance
     // histogram per query (starting bound, see the epilogue), then all t1 - t0.
@@ -797,11 +807,17 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
         if (cost < best_cost) { best_cost = cost; best = s; }
     }
     g.S = best;
+    static const int coldw_env = [] {
+        const char* e = std::getenv("KSEL_KNN_COLDW");  // experiments: first-wave split weight (per mille)
+        return e ? std::atoi(e) : 1000;
+    }();
+    g.cold_w = (coldw_env > 0 && coldw_env <= 1000) ? coldw_env : 1000;
     static const int splits_env = [] {
         const char* e = std::getenv("KSEL_KNN_SPLITS");  // experiments: force the split count
         return e ? std::atoi(e) : 0;
     }();
     if (splits_env > 0) g.S = std::min(splits_env, smax);
+    g.cold_splits = std::min(g.S, (num_sms + g.QTp - 1) / g.QTp);
     return g;
 }
 
