@@ -22,6 +22,7 @@ ap.add_argument("--reps", type=int, default=5)
 ap.add_argument("--algo", type=int, default=0)
 ap.add_argument("--wpr", type=int, default=0)
 ap.add_argument("--nosplit", action="store_true", help="force one CTA per row (no split rows)")
+ap.add_argument("--inner", type=int, default=1, help="calls per timed region (hides host launch latency)")
 a = ap.parse_args()
 x = synth.rows(a.dist, synth.seed_for(2, a.dist), 0, a.Q, a.N, device="cuda")
 v = torch.empty((a.Q, a.k), dtype=torch.float32, device="cuda")
@@ -32,9 +33,10 @@ e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=Tr
 for r in range(a.reps):
     torch.cuda.synchronize()
     e0.record()
-    K.ksel_select(x, a.k, v, i, algo=a.algo, warps_per_row=a.wpr, workspace=ws, split_rows=not a.nosplit)
+    for _ in range(a.inner):
+        K.ksel_select(x, a.k, v, i, algo=a.algo, warps_per_row=a.wpr, workspace=ws, split_rows=not a.nosplit)
     e1.record()
     torch.cuda.synchronize()
-    ms = e0.elapsed_time(e1)
+    ms = e0.elapsed_time(e1) / a.inner
     gbs = a.Q * (4.0 * a.N + 8 * a.k) / (ms / 1e3) / 1e9
     print("rep %d: %.4f ms  %.1f GB/s  %.3g rows/s" % (r, ms, gbs, a.Q / (ms / 1e3)), flush=True)
