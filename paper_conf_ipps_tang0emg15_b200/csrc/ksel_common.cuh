@@ -40,8 +40,10 @@ __device__ __forceinline__ bool key_needs_regather(uint32_t key) {
 }
 
 // Lexicographic (key, idx) "strictly before".
+// As one 64-bit unsigned compare of (key << 32 | idx): two ISETPs instead of three
+// or four instructions.
 __device__ __forceinline__ bool pair_lt(uint32_t ka, uint32_t ia, uint32_t kb, uint32_t ib) {
-    return (ka < kb) || (ka == kb && ia < ib);
+    return (((uint64_t)ka << 32) | ia) < (((uint64_t)kb << 32) | ib);
 }
 
 __device__ __forceinline__ uint32_t lane_id() {
@@ -71,8 +73,10 @@ __device__ __forceinline__ void warr_fill_sentinel(WArr<R>& a) {
 }
 
 // In-register compare-exchange: lower position gets the smaller pair when asc.
+// (One comparison: when descending, equal pairs are swapped too -- harmless, since
+// equal pairs are identical; (key, idx) pairs are distinct except sentinels.)
 __device__ __forceinline__ void cx_reg(uint32_t& ka, uint32_t& ia, uint32_t& kb, uint32_t& ib, bool asc) {
-    const bool swap = asc ? pair_lt(kb, ib, ka, ia) : pair_lt(ka, ia, kb, ib);
+    const bool swap = pair_lt(kb, ib, ka, ia) == asc;
     const uint32_t tk = ka, ti = ia;
     ka = swap ? kb : ka; ia = swap ? ib : ia;
     kb = swap ? tk : kb; ib = swap ? ti : ib;
@@ -83,8 +87,8 @@ __device__ __forceinline__ void cx_reg(uint32_t& ka, uint32_t& ia, uint32_t& kb,
 __device__ __forceinline__ void cx_lane(uint32_t& k, uint32_t& i, int s, bool keep_min) {
     const uint32_t ok = __shfl_xor_sync(kFull, k, s);
     const uint32_t oi = __shfl_xor_sync(kFull, i, s);
-    const bool other_first = pair_lt(ok, oi, k, i);
-    const bool take = keep_min ? other_first : pair_lt(k, i, ok, oi);
+    // one comparison for both directions (the max side also takes an equal partner: identical)
+    const bool take = pair_lt(ok, oi, k, i) == keep_min;
     k = take ? ok : k;
     i = take ? oi : i;
 }
