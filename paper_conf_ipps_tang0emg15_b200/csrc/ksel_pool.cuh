@@ -75,9 +75,27 @@ __device__ __noinline__ static unsigned long long pool_kth(const uint32_t* __res
                                                     int n, uint32_t want, uint32_t* __restrict__ hist,
                                                     uint32_t* ties_out = nullptr) {
     const uint32_t lane = lane_id();
-    uint32_t prefix = 0, cnt = 0;
+    // Digits above the highest bit where the pool's smallest and largest keys differ
+    // are common to all keys: start at the pass holding that bit (pools of keys near
+    // one bound usually share their top byte or two).
+    uint32_t kmin = 0xffffffffu, kmax = 0u;
+    for (int e = (int)lane; e < n; e += 32) {
+        const uint32_t key = pk[e];
+        kmin = min(kmin, key);
+        kmax = max(kmax, key);
+    }
+    kmin = __reduce_min_sync(kFull, kmin);
+    kmax = __reduce_max_sync(kFull, kmax);
+    uint32_t prefix = 0, cnt = (uint32_t)n;
+    int first = 4;  // all keys equal: no pass, the k-th key is kmin and every key ties
+    if (kmin != kmax) {
+        first = __clz(kmin ^ kmax) >> 3;
+        prefix = first ? (kmin & (0xffffffffu << (32 - 8 * first))) : 0u;
+    } else {
+        prefix = kmin;
+    }
 #pragma unroll 1
-    for (int pass = 0; pass < 4; ++pass) {
+    for (int pass = first; pass < 4; ++pass) {
         const int shift = 24 - 8 * pass;
 #pragma unroll
         for (int j = 0; j < 8; ++j) hist[j * 32 + lane] = 0u;
@@ -85,7 +103,7 @@ __device__ __noinline__ static unsigned long long pool_kth(const uint32_t* __res
 #pragma unroll 4
         for (int e = (int)lane; e < n; e += 32) {
             const uint32_t key = pk[e];
-            const bool sel = (pass == 0) || ((key ^ prefix) >> (shift + 8)) == 0u;
+            const bool sel = (pass == first) || ((key ^ prefix) >> (shift + 8)) == 0u;
             if (sel) atomicAdd(&hist[hist_slot((key >> shift) & 255u)], 1u);
         }
         __syncwarp();
@@ -103,9 +121,20 @@ __device__ __noinline__ static unsigned long long pool_kth(const uint32_t* __res
             if (pk[e] == vkey) m = max(m, pi[e]);
         idx = __reduce_max_sync(kFull, m);
     } else {
-        uint32_t ip = 0;
+        // the same prefix skip over the tied keys' indices (row indices < 2^16 share
+        // their top two bytes)
+        uint32_t imin = 0xffffffffu, imax = 0u;
+        for (int e = (int)lane; e < n; e += 32)
+            if (pk[e] == vkey) {
+                imin = min(imin, pi[e]);
+                imax = max(imax, pi[e]);
+            }
+        imin = __reduce_min_sync(kFull, imin);
+        imax = __reduce_max_sync(kFull, imax);  // (>= 2 distinct ties here: cnt > want >= 1)
+        const int ifirst = __clz(imin ^ imax) >> 3;
+        uint32_t ip = ifirst ? (imin & (0xffffffffu << (32 - 8 * ifirst))) : 0u;
 #pragma unroll 1
-        for (int pass = 0; pass < 4; ++pass) {
+        for (int pass = ifirst; pass < 4; ++pass) {
             const int shift = 24 - 8 * pass;
 #pragma unroll
             for (int j = 0; j < 8; ++j) hist[j * 32 + lane] = 0u;
@@ -113,7 +142,7 @@ __device__ __noinline__ static unsigned long long pool_kth(const uint32_t* __res
             for (int e = (int)lane; e < n; e += 32) {
                 if (pk[e] != vkey) continue;
                 const uint32_t id = pi[e];
-                const bool sel = (pass == 0) || ((id ^ ip) >> (shift + 8)) == 0u;
+                const bool sel = (pass == ifirst) || ((id ^ ip) >> (shift + 8)) == 0u;
                 if (sel) atomicAdd(&hist[hist_slot((id >> shift) & 255u)], 1u);
             }
             __syncwarp();
