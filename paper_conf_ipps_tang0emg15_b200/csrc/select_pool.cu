@@ -336,8 +336,8 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads)
             // Bisection on the key bits below the common prefix of the smallest and
             // largest real key, stopped at bit kLow: the k-th key then lies in
             // [vkey, vkey + 2^kLow), so vkey | (2^kLow - 1) bounds it (>= k keys are
-            // <= it; looser by < 2^-15 relative for floats, for ~40% fewer steps).
-            constexpr int kLow = 8;
+            // <= it; looser by < 2^-7 relative for floats, for about half the steps).
+            constexpr int kLow = 16;
             uint32_t kmin = 0xffffffffu, kmax = 0u;
 #pragma unroll
             for (int j = 0; j < NB * CH / 128 * 4; ++j) {
