@@ -379,14 +379,25 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads)
         for (int g = 0; g < CH / 128; g += G) {
             float x[NS];
             const float inf = __int_as_float(0x7f800000);  // never passes x <= tv in fast mode
+            if (len == (uint32_t)CH) {  // (every chunk but a row's last: no per-element bounds)
 #pragma unroll
-            for (int u = 0; u < G; ++u) {
-                const uint32_t e4 = (uint32_t)(g + u) * 32u + lane;
-                const float4 v = (len == (uint32_t)CH || e4 * 4u < len) ? src[e4] : make_float4(inf, inf, inf, inf);
-                x[4 * u + 0] = v.x;
-                x[4 * u + 1] = v.y;
-                x[4 * u + 2] = v.z;
-                x[4 * u + 3] = v.w;
+                for (int u = 0; u < G; ++u) {
+                    const float4 v = src[(uint32_t)(g + u) * 32u + lane];
+                    x[4 * u + 0] = v.x;
+                    x[4 * u + 1] = v.y;
+                    x[4 * u + 2] = v.z;
+                    x[4 * u + 3] = v.w;
+                }
+            } else {
+#pragma unroll
+                for (int u = 0; u < G; ++u) {
+                    const uint32_t e4 = (uint32_t)(g + u) * 32u + lane;
+                    const float4 v = (e4 * 4u < len) ? src[e4] : make_float4(inf, inf, inf, inf);
+                    x[4 * u + 0] = v.x;
+                    x[4 * u + 1] = v.y;
+                    x[4 * u + 2] = v.z;
+                    x[4 * u + 3] = v.w;
+                }
             }
             bool go = true;
             if (fast) {
@@ -394,9 +405,14 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads)
                 // candidate).  Past the bound's index (col0 >= Ti) an element equal to the bound
                 // value cannot precede the bound pair, so the test is strict: rows with heavy
                 // ties then skip the sub-steps that only hold copies of the bound value.
-                float mn = x[0];
+                // (a tree, not a 15-deep chain: the sub-step is latency-bound when few warps run)
+                float gm[G];
 #pragma unroll
-                for (int j = 1; j < NS; ++j) mn = fminf(mn, x[j]);
+                for (int u = 0; u < G; ++u)
+                    gm[u] = fminf(fminf(x[4 * u], x[4 * u + 1]), fminf(x[4 * u + 2], x[4 * u + 3]));
+                float mn = gm[0];
+#pragma unroll
+                for (int u = 1; u < G; ++u) mn = fminf(mn, gm[u]);
                 go = __any_sync(kFull, col0 >= Ti ? mn < tv : mn <= tv);
             }
             if (go) exact(srcf, (uint32_t)g, len, col0, x);
