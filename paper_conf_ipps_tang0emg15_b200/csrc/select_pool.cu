@@ -37,7 +37,13 @@ namespace ksel {
 template <int R, int WPR, int RPC, int SD = 3>
 struct PoolCfg {
     static constexpr int kQueue = 32 * R;  // k'
-    static constexpr int kPool = (2 * kQueue > kQueue + 512) ? 2 * kQueue : kQueue + 512;
+    // k' = 1024 with the shallow ring (many rows: shared memory limits the warps per SM):
+    // k' + 512 pairs (one sub-step of room) -- 19 KB per warp instead of 23 KB, 11 warps
+    // per SM instead of 9 (C3 k = 1024: 17.5 -> 15.7 ms).  With few rows (deep ring) the
+    // larger pool's fewer narrowings win (C2 k = 1024: 0.24 vs 0.29 ms).
+    static constexpr int kPool = (kQueue >= 1024 && SD <= 3)
+                                     ? kQueue + 512
+                                     : ((2 * kQueue > kQueue + 512) ? 2 * kQueue : kQueue + 512);
     static constexpr int CH = 512;         // floats per staged chunk (2 KB bulk copy)
     static constexpr int NB = (2048 / CH < SD) ? 2048 / CH : SD;  // chunks feeding the starting bound
     static constexpr int S = SD;           // ring stages per warp (3, or 6 when few warps run per SM)
