@@ -48,7 +48,9 @@ def parse():
     ap.add_argument("--k", type=int, default=None)
     ap.add_argument("--dist", default=None)
     ap.add_argument("--scaling", choices=["weak", "strong"], default="weak")
-    ap.add_argument("--e2e-rows", type=int, default=2048, help="rows per end-to-end step (host buffers)")
+    ap.add_argument("--e2e-rows", type=int, default=0,
+                    help="rows per end-to-end step per rank (host buffers); 0 = 2048 on one GPU, "
+                         "512 per rank on several (pinned host memory: 4 MB per row)")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--cpu-sample-rows", type=int, default=0, help="0 = auto (~10-30 s of CPU work)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -332,7 +334,7 @@ def bench_select(args, rank, world, local_rank, dev, K, tdist):
 
     # ---- end-to-end through the public host API --------------------------------------
     if not args.no_e2e:
-        er = min(args.e2e_rows, Qr)
+        er = min(args.e2e_rows or (2048 if world == 1 else 512), Qr)
         hx = torch.empty((er, N), dtype=torch.float32, pin_memory=True)
         hx.copy_(x[:er])
         hv = torch.empty((er, k), dtype=torch.float32, pin_memory=True)
