@@ -319,3 +319,25 @@ def test_synth_same_bits_on_gpu_and_cpu(dist):
         p = synth.knn_points(kind, 9, 100, 50, 128, device="cuda").cpu()
         q = synth.knn_points(kind, 9, 100, 50, 128)
         assert torch.equal(p.view(torch.int32), q.view(torch.int32))
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_fuzz_shapes_all_algorithms(K, oracle_mod, seed):
+    # random row counts / lengths / k / distributions / alignment, every kernel variant
+    rng = np.random.default_rng(1000 + seed)
+    for case in range(10):
+        N = int(np.exp(rng.uniform(0, np.log(70000))))
+        Q = int(max(1, min(300, 4_000_000 // max(N, 1), int(np.exp(rng.uniform(0, np.log(300)))))))
+        k = int(rng.integers(1, min(N, 1024) + 1))
+        dist = str(rng.choice(synth.DISTS))
+        off = int(rng.integers(0, 4))
+        big = synth.rows(dist, 7000 + seed * 10 + case, 0, 1, Q * N + off)[0]
+        x_cpu = big[off:off + Q * N].reshape(Q, N).contiguous()
+        xg = big.cuda()[off:off + Q * N].view(Q, N)
+        ev, ei = oracle_mod.select(x_cpu.numpy(), k)
+        algos = [0, 1, 2] + ([3] if N <= 65536 else [])
+        for algo in algos:
+            gv, gi = K.ksel_select(xg, k, algo=algo)
+            torch.cuda.synchronize()
+            assert_same(ev, ei, gv, gi, "fuzz seed=%d case=%d Q=%d N=%d k=%d %s off=%d algo=%d"
+                        % (seed, case, Q, N, k, dist, off, algo))
