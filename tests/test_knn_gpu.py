@@ -264,3 +264,18 @@ def test_fuzz_knn_shapes(K, oracle_mod, seed):
         gv, gi = K.knn_search(ref.cuda(), qry.cuda(), k)
         torch.cuda.synchronize()
         check_knn(oracle_mod, ref, qry, k, gv, gi, exact=(kind == "knn-S"))
+
+
+@pytest.mark.parametrize("seed", range(2))
+def test_fuzz_knn_graph(K, oracle_mod, seed):
+    rng = np.random.default_rng(700 + seed)
+    for case in range(4):
+        kind = "knn-S" if case % 2 == 0 else "knn-U"
+        N = int(rng.integers(2, 4000))
+        D = int(rng.choice([2, 5, 32, 64, 128]))
+        k = int(rng.integers(1, min(N - 1, 1023) + 1))
+        x = synth.knn_points(kind, 980 + 10 * seed + case, 0, N, D)
+        gv, gi = K.knn_graph(x.cuda(), k)
+        torch.cuda.synchronize()
+        check_knn(oracle_mod, x, x, k, gv, gi, exact=(kind == "knn-S"),
+                  oracle_out=oracle_mod.knn_graph(x.numpy(), k), rows=list(range(N)))

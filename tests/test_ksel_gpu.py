@@ -341,3 +341,43 @@ def test_fuzz_shapes_all_algorithms(K, oracle_mod, seed):
             torch.cuda.synchronize()
             assert_same(ev, ei, gv, gi, "fuzz seed=%d case=%d Q=%d N=%d k=%d %s off=%d algo=%d"
                         % (seed, case, Q, N, k, dist, off, algo))
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_fuzz_split_rows(K, oracle_mod, seed):
+    # few long rows (the split-row path: segments per SM + a second selection)
+    rng = np.random.default_rng(2000 + seed)
+    for case in range(4):
+        Q = int(rng.integers(1, 24))
+        N = int(rng.integers(70000, 4_000_000 // Q + 70001))
+        k = int(rng.integers(1, 1025))
+        dist = str(rng.choice(synth.DISTS))
+        x_cpu = synth.rows(dist, 8000 + seed * 10 + case, 0, Q, N)
+        gv, gi = K.ksel_select(x_cpu.cuda(), k)
+        torch.cuda.synchronize()
+        ev, ei = oracle_mod.select(x_cpu.numpy(), k)
+        assert_same(ev, ei, gv, gi, "split fuzz seed=%d case=%d Q=%d N=%d k=%d %s" % (seed, case, Q, N, k, dist))
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_fuzz_merge(K, oracle_mod, seed):
+    # random list counts / lengths / k, lists from selections of random column blocks
+    rng = np.random.default_rng(3000 + seed)
+    for case in range(5):
+        S = int(rng.integers(1, 9))
+        kin = int(rng.integers(1, 1025))
+        k = int(rng.integers(1, min(S * kin, 1024) + 1))
+        Q = int(rng.integers(1, 200))
+        W = max(kin, 64)
+        dist = str(rng.choice(synth.DISTS))
+        x = synth.rows(dist, 9000 + seed * 10 + case, 0, Q, S * W, device="cuda")
+        vs, is_ = [], []
+        for s in range(S):
+            v, i = K.ksel_select(x[:, s * W:(s + 1) * W].contiguous(), kin)
+            vs.append(v)
+            is_.append(i + s * W)
+        cv, ci = torch.stack(vs), torch.stack(is_)
+        gv, gi = K.ksel_merge(cv, ci, k)
+        torch.cuda.synchronize()
+        ev, ei = oracle_mod.merge(cv.cpu().numpy(), ci.cpu().numpy(), k)  # top-k of the union of the lists
+        assert_same(ev, ei, gv, gi, "merge fuzz seed=%d case=%d S=%d kin=%d k=%d Q=%d %s" % (seed, case, S, kin, k, Q, dist))
