@@ -65,6 +65,11 @@ void timing_end(int slot, cudaStream_t stream) {
     cudaEventRecord(g_tm[slot].b, stream);
 }
 
+int env_int(const char* name, int dflt) {
+    const char* e = std::getenv(name);
+    return (e && e[0]) ? std::atoi(e) : dflt;
+}
+
 int chunk_order_mode() {
     // bits 0-1: chunk visit order (KSEL_ORDER, default 2); bit 2: loose admission
     // experiment (KSEL_LOOSE=1).  Experiments only; the defaults are the product.

@@ -742,8 +742,7 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     g.NT = (int)((N + KNN_BN - 1) / KNN_BN);
     g.QT = (int)((Q + KNN_BM - 1) / KNN_BM);
     static const int cs_env = [] {
-        const char* e = std::getenv("KSEL_KNN_CLUSTER");  // experiments: cluster size 1, 2 or 4
-        const int v = e ? std::atoi(e) : 1;
+        const int v = env_int("KSEL_KNN_CLUSTER", 1);  // experiments: cluster size 1, 2 or 4
         return (v == 2 || v == 4) ? v : 1;
     }();
     // Every CTA streams its whole reference range through L2 -> shared memory (4 B per
@@ -755,10 +754,7 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     // 5.14 ms), so L2 is not the floor and the default is cs = 1.
     g.cs = (g.QT >= cs_env) ? cs_env : 1;
     g.QTp = (g.QT + g.cs - 1) / g.cs * g.cs;
-    static const int passes_env = [] {
-        const char* e = std::getenv("KSEL_KNN_PASSES");  // experiments only: 1 breaks the accuracy bound
-        return (e && std::atoi(e) == 1) ? 1 : 3;
-    }();
+    static const int passes_env = env_int("KSEL_KNN_PASSES", 3) == 1 ? 1 : 3;  // experiments only: 1 breaks the accuracy bound
     g.passes = passes_env;
     g.k = k;
     const int kk = k < 32 ? 32 : k;
@@ -772,15 +768,9 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     g.NS = (kMaxSmemPerBlock - fixed) / KNN_STAGE_BYTES;
     if (g.NS > 6) g.NS = 6;
     g.idx_offset = idx_offset;
-    static const int ew_env = [] {
-        const char* e = std::getenv("KSEL_KNN_EW");  // experiments: 4 or 8 epilogue warps
-        return (e && std::atoi(e) == 8) ? 8 : 4;
-    }();
+    static const int ew_env = env_int("KSEL_KNN_EW", 4) == 8 ? 8 : 4;  // experiments: 4 or 8 epilogue warps
     g.halves = ew_env / 4;
-    static const int cap_env = [] {
-        const char* e = std::getenv("KSEL_KNN_SOFTCAP");  // experiments: narrow early (pool fill cap)
-        return e ? std::atoi(e) : 0;
-    }();
+    static const int cap_env = env_int("KSEL_KNN_SOFTCAP", 0);  // experiments: narrow early (pool fill cap)
     // narrow before a pool reaches P when queues are small: the bound then tracks the
     // k-th of what has been seen more closely in cold CTAs (measured: 512 for k <= 128)
     const int cap = cap_env > 0 ? cap_env : (kk <= 128 ? 512 : g.P);
@@ -788,10 +778,7 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     g.ntiles = g.NT;
     g.tstride = 1;
     // first-wave CTAs sample 16 tiles (4096 references) for their starting bound
-    static const int sample_env = [] {
-        const char* e = std::getenv("KSEL_KNN_SAMPLE");  // experiments: tiles sampled (0 = off)
-        return e ? std::atoi(e) : 16;
-    }();
+    static const int sample_env = env_int("KSEL_KNN_SAMPLE", 16);  // experiments: tiles sampled (0 = off)
     g.sample_tiles = sample_env;
     g.sample_ctas = g.sample_tiles > 0 ? num_sms / g.cs * g.cs : 0;  // whole clusters
     // reference splits: enough CTAs for the SMs, waves as full as possible, <= 64 lists to merge
@@ -807,15 +794,9 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
         if (cost < best_cost) { best_cost = cost; best = s; }
     }
     g.S = best;
-    static const int coldw_env = [] {
-        const char* e = std::getenv("KSEL_KNN_COLDW");  // experiments: first-wave split weight (per mille)
-        return e ? std::atoi(e) : 1000;
-    }();
+    static const int coldw_env = env_int("KSEL_KNN_COLDW", 1000);  // experiments: first-wave split weight (per mille)
     g.cold_w = (coldw_env > 0 && coldw_env <= 1000) ? coldw_env : 1000;
-    static const int splits_env = [] {
-        const char* e = std::getenv("KSEL_KNN_SPLITS");  // experiments: force the split count
-        return e ? std::atoi(e) : 0;
-    }();
+    static const int splits_env = env_int("KSEL_KNN_SPLITS", 0);  // experiments: force the split count
     if (splits_env > 0) g.S = std::min(splits_env, smax);
     g.cold_splits = std::min(g.S, (num_sms + g.QTp - 1) / g.QTp);
     return g;
@@ -853,9 +834,9 @@ static cudaError_t knn_run(const float* ref, const float* query, const KnnGeom& 
     e = cudaMemsetAsync(work + w.qthr, 0xff, (size_t)g.Q * 8, stream);  // "no bound yet"
     if (e != cudaSuccess) return e;
     const int smem = KnnSmem::total(g);
-    static const int mode_env = [] {
-        const char* e = std::getenv("KSEL_KNN_MODE");
-        return (e && (e[0] == '2' || e[0] == '3' || e[0] == '4')) ? e[0] - '0' : 0;
+    static const int mode_env = [] {  // experiments: 2 pipeline only, 3 counters, 4 no TMEM reads
+        const int m = env_int("KSEL_KNN_MODE", 0);
+        return (m >= 2 && m <= 4) ? m : 0;
     }();
     const bool ew8 = g.halves == 2;
     auto kern = dump ? (ew8 ? knn_fused_kernel<1, 8> : knn_fused_kernel<1, 4>)

@@ -8,6 +8,11 @@ namespace ksel {
 
 constexpr int kMaxSmemPerBlock = 227 * 1024;  // sm_100 opt-in dynamic shared memory per CTA
 
+// Integer value of an environment variable, or `dflt` when unset/empty.  Only the
+// experiment knobs (KSEL_* variables) read the environment; the defaults
+// are the product.
+int env_int(const char* name, int dflt);
+
 // Chunk visit order of the streaming kernels (experiments only; env KSEL_ORDER):
 // 0 = address order, 1 = spread prologue + address order, 2 = strided permutation (default).
 int chunk_order_mode();
