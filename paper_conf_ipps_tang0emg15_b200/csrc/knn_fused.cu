@@ -51,8 +51,6 @@ namespace ksel {
 constexpr int KNN_BM = 128;                              // queries per tile (TMEM lanes)
 constexpr int KNN_BN = 256;                              // references per tile (accumulator columns)
 constexpr int KNN_KS = 32;                               // dims per pipeline stage
-constexpr int KNN_STAGE_BYTES = 2 * KNN_KS * KNN_BN * 2;  // hi + lo bf16 = 32 KB
-constexpr int KNN_NORM_B_BYTES = 16 * KNN_BN * 2;         // norm block of a reference tile (hi only)
 constexpr int KNN_NORM_A_BYTES = 16 * KNN_BM * 2;         // norm block of a query tile
 // epilogue warps EW: 4 (one per TMEM lane quadrant, all 256 columns of a tile) or
 // 8 (two per quadrant, 128 columns each); + producer + MMA issuer
@@ -90,7 +88,12 @@ struct KnnGeom {
         };
         return (int)((int64_t)ntiles * W(s) / W(S));
     }
-    __host__ __device__ size_t tile_bytes() const { return (size_t)KS * KNN_STAGE_BYTES + KNN_NORM_B_BYTES; }
+    int BN;              // references per tile (accumulator columns): 256, or 128 with QPC = 2
+    int QPC;             // query tiles per CTA sharing every reference stage (1 or 2)
+    int EW;              // epilogue warps of the launch (4, or 8)
+    __host__ __device__ int stage_bytes() const { return 2 * KNN_KS * BN * 2; }  // hi + lo bf16
+    __host__ __device__ int norm_b_bytes() const { return 16 * BN * 2; }
+    __host__ __device__ size_t tile_bytes() const { return (size_t)KS * stage_bytes() + norm_b_bytes(); }
     __host__ __device__ int a_bytes() const { return Dp * 512 + KNN_NORM_A_BYTES; }
 };
 
@@ -125,7 +128,7 @@ __global__ void __launch_bounds__(KNN_PREP_THREADS)
     __shared__ float tile[KNN_BN][KNN_KS + 1];
     const bool is_q = blockIdx.x >= (unsigned)g.NT;
     const int64_t t = is_q ? (int64_t)blockIdx.x - g.NT : (int64_t)blockIdx.x;
-    const int rows = is_q ? KNN_BM : KNN_BN;
+    const int rows = is_q ? KNN_BM : g.BN;
     const int64_t n = is_q ? g.Q : g.N;
     const float* x = is_q ? qry : ref;
     const float scale = is_q ? -2.f : 1.f;  // exact
@@ -146,11 +149,11 @@ __global__ void __launch_bounds__(KNN_PREP_THREADS)
             if (is_q) {  // [hi,lo][Dp/8 chunks][128 rows][8]
                 dst = q_img + t * (int64_t)(g.a_bytes() / 16) + (int64_t)(ks * 4) * KNN_BM + tid;
                 cstride = KNN_BM;
-            } else {     // [stage][hi,lo][4 chunks][256 rows][8]
-                dst = ref_img + t * (int64_t)(g.tile_bytes() / 16) + (int64_t)ks * (KNN_STAGE_BYTES / 16) + tid;
-                cstride = KNN_BN;
+            } else {     // [stage][hi,lo][4 chunks][BN rows][8]
+                dst = ref_img + t * (int64_t)(g.tile_bytes() / 16) + (int64_t)ks * (g.stage_bytes() / 16) + tid;
+                cstride = g.BN;
             }
-            const int64_t lo_off = is_q ? (int64_t)(g.Dp / 8) * KNN_BM : 4 * KNN_BN;
+            const int64_t lo_off = is_q ? (int64_t)(g.Dp / 8) * KNN_BM : 4 * (int64_t)g.BN;
 #pragma unroll
             for (int kc = 0; kc < 4; ++kc) {
                 uint32_t h[4], l[4];
@@ -181,7 +184,7 @@ __global__ void __launch_bounds__(KNN_PREP_THREADS)
             blk = q_img + (t * (int64_t)g.a_bytes() + (int64_t)g.Dp * 512) / 16;
             c0 = make_uint4(bf2(n1, n2), bf2(n3, one), bf2(one, one), 0u);
         } else {
-            blk = ref_img + (t * (int64_t)g.tile_bytes() + (int64_t)g.KS * KNN_STAGE_BYTES) / 16;
+            blk = ref_img + (t * (int64_t)g.tile_bytes() + (int64_t)g.KS * g.stage_bytes()) / 16;
             c0 = make_uint4(bf2(one, one), bf2(one, n1), bf2(n2, n3), 0u);
         }
         blk[tid] = c0;
@@ -300,11 +303,12 @@ __device__ __forceinline__ void umma_commit_mc(uint64_t* bar, uint16_t mask) {
 // the fused kernel
 // ---------------------------------------------------------------------------
 struct KnnSmem {
-    static constexpr int kHistBytes = KNN_MAX_EW * 256 * 4;        // radix histogram per warp (pool_select64)
-    static constexpr int kWarpScratch = KNN_SB * 32 * 4;      // per warp: sampling histogram, one per lane
-    static constexpr int kDStageBytes = KNN_MAX_EW * kWarpScratch;
+    static constexpr int kHistWarp = 256 * 4;                  // per epilogue warp: radix histogram (pool_select64)
+    static constexpr int kWarpScratch = KNN_SB * 32 * 4;      // per epilogue warp: sampling histogram, one per lane
+    // scratch of `ew` epilogue warps (sized for the launch: every KB left goes to the ring)
+    __host__ __device__ static int scratch(int ew) { return ew * (kHistWarp + kWarpScratch); }
     __host__ __device__ static int total(const KnnGeom& g) {
-        return 1024 /*align slack*/ + g.a_bytes() + g.NS * KNN_STAGE_BYTES + kHistBytes + kDStageBytes +
+        return 1024 /*align slack*/ + g.QPC * g.a_bytes() + g.NS * g.stage_bytes() + scratch(g.EW) +
                (2 * g.NS + 5) * 8 + 16;
     }
 };
@@ -313,13 +317,18 @@ struct KnnSmem {
 // 2: pipeline only -- the epilogue reads the accumulators and drops them
 // (experiments: isolates the TMA + MMA + TMEM pipeline from the selection);
 // 3: selection + per-warp cycle counters; 4: pipeline without any TMEM read.
-template <int MODE, int EW>
+// BN: references per tile; QPC: query tiles per CTA (each B stage feeds QPC x 128
+// queries: with QPC = 2, BN = 128 and four 128-column accumulators, half the bytes
+// land in shared memory per output)
+template <int MODE, int EW, int BN, int QPC>
 __global__ void __launch_bounds__(knn_threads(EW), 1)
     knn_fused_kernel(KnnGeom g, const uint8_t* __restrict__ ref_img, const uint8_t* __restrict__ q_img,
                      unsigned long long* __restrict__ pool64, int32_t* __restrict__ cnt_out,
                      unsigned long long* __restrict__ qthr, float* __restrict__ dump) {
-    constexpr int HALVES = EW / 4;
-    constexpr int WCOLS = KNN_BN / HALVES;  // columns of each tile this epilogue warp scans
+    constexpr int HALVES = (QPC == 1) ? EW / 4 : 1;
+    constexpr int WCOLS = BN / HALVES;  // columns of each tile this epilogue warp scans
+    constexpr int SB = 2 * KNN_KS * BN * 2;   // bytes of one reference stage
+    constexpr int NBB = 16 * BN * 2;          // bytes of a reference tile's norm block
     constexpr bool DUMP = (MODE == 1);
     constexpr bool PIPE_ONLY = (MODE == 2 || MODE == 4);
     constexpr bool NO_READ = (MODE == 4);  // pipeline only, accumulators never read (experiments)
@@ -330,10 +339,10 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
     uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
     const int NS = g.NS;
     uint8_t* sA = smem;
-    uint8_t* sB = sA + g.a_bytes();
-    uint32_t* hist_all = reinterpret_cast<uint32_t*>(sB + NS * KNN_STAGE_BYTES);
-    float* dstage_all = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(hist_all) + KnnSmem::kHistBytes);
-    uint64_t* bars = reinterpret_cast<uint64_t*>(reinterpret_cast<uint8_t*>(dstage_all) + KnnSmem::kDStageBytes);
+    uint8_t* sB = sA + QPC * g.a_bytes();
+    uint32_t* hist_all = reinterpret_cast<uint32_t*>(sB + NS * SB);
+    float* dstage_all = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(hist_all) + EW * KnnSmem::kHistWarp);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(reinterpret_cast<uint8_t*>(dstage_all) + EW * KnnSmem::kWarpScratch);
     uint64_t* full = bars;
     uint64_t* empty = bars + NS;
     uint64_t* accf = bars + 2 * NS;
@@ -343,7 +352,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
 
     const int warp = threadIdx.x >> 5;
     const uint32_t lane = lane_id();
-    const int qt = blockIdx.x % g.QTp;  // >= QT: padding tile of a cluster (loads, MMAs, no queries)
+    const int grp = blockIdx.x % g.QTp;  // query tiles grp*QPC.. (>= QT: padding, no queries)
     const int split = blockIdx.x / g.QTp;
     const uint32_t crank = g.cs > 1 ? cluster_rank() : 0u;
     const uint16_t cmask = (uint16_t)((1u << g.cs) - 1u);
@@ -352,8 +361,8 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
     // Cold CTAs (the first wave: no split of their queries has published a bound
     // yet) first stream their first Fs tiles through the pipeline for a distance
     // histogram per query (starting bound, see the epilogue), then all t1 - t0.
-    const int Fs = (!DUMP && !PIPE_ONLY && (int)blockIdx.x < g.sample_ctas && g.k <= KNN_BN && g.tstride == 1 &&
-                    t1 - t0 >= 4 * g.sample_tiles && (int64_t)(t0 + g.sample_tiles) * KNN_BN <= g.N)
+    const int Fs = (!DUMP && !PIPE_ONLY && (int)blockIdx.x < g.sample_ctas && g.k <= BN && g.tstride == 1 &&
+                    t1 - t0 >= 4 * g.sample_tiles && (int64_t)(t0 + g.sample_tiles) * BN <= g.N)
                        ? g.sample_tiles
                        : 0;
     const int nsteps = Fs + (t1 - t0);
@@ -387,22 +396,26 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
         // (per tile: KS dims stages of 32 KB, then the 8 KB norm block)
         if (lane == 0) {
             const uint32_t abytes = (uint32_t)g.a_bytes();
-            mbar_arrive_expect_tx(afull, abytes);
-            bulk_g2s(sA, q_img + (size_t)(qt < g.QT ? qt : 0) * abytes, abytes, afull);
+            mbar_arrive_expect_tx(afull, QPC * abytes);
+#pragma unroll
+            for (int h = 0; h < QPC; ++h) {
+                const int qtile = grp * QPC + h;
+                bulk_g2s(sA + h * abytes, q_img + (size_t)(qtile < g.QT ? qtile : 0) * abytes, abytes, afull);
+            }
             uint32_t it = 0;
             for (int lt = 0; lt < nsteps; ++lt) {
                 const int t = (lt < Fs ? t0 + lt : t0 + lt - Fs) * g.tstride;
                 for (int ks = 0; ks <= g.KS; ++ks, ++it) {
                     const int st = (int)(it % NS);
-                    const uint32_t bytes = (ks < g.KS) ? KNN_STAGE_BYTES : KNN_NORM_B_BYTES;
+                    const uint32_t bytes = (ks < g.KS) ? SB : NBB;
                     mbar_wait_sleep(&empty[st], ((it / NS) & 1u) ^ 1u);
                     mbar_arrive_expect_tx(&full[st], bytes);
-                    const uint8_t* src = ref_img + (size_t)t * g.tile_bytes() + (size_t)ks * KNN_STAGE_BYTES;
+                    const uint8_t* src = ref_img + (size_t)t * g.tile_bytes() + (size_t)ks * SB;
                     if (g.cs == 1) {
-                        bulk_g2s(sB + st * KNN_STAGE_BYTES, src, bytes, &full[st]);
+                        bulk_g2s(sB + st * SB, src, bytes, &full[st]);
                     } else {  // this CTA's slice of the stage, into every CTA of the cluster
                         const uint32_t sl = bytes / g.cs;
-                        bulk_g2s_mc(sB + st * KNN_STAGE_BYTES + crank * sl, src + crank * sl, sl, &full[st], cmask);
+                        bulk_g2s_mc(sB + st * SB + crank * sl, src + crank * sl, sl, &full[st], cmask);
                     }
                 }
             }
@@ -410,10 +423,8 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
     } else if (warp == 1) {
         // ===== MMA issuer (one thread) =====
         if (lane == 0) {
-            constexpr uint32_t idesc = umma_idesc_bf16(KNN_BM, KNN_BN);
-            const uint32_t a0 = smem_u32(sA);
-            const uint32_t alo = a0 + (uint32_t)(g.Dp / 8) * (KNN_BM * 16);
-            const uint32_t anorm = a0 + (uint32_t)(g.Dp * 512);
+            constexpr uint32_t idesc = umma_idesc_bf16(KNN_BM, BN);
+            const uint32_t abytes = (uint32_t)g.a_bytes();
             mbar_wait(afull, 0);
             tc_fence_after();
             uint32_t it = 0;
@@ -421,32 +432,34 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                 const int b = lt & 1;
                 mbar_wait_sleep(&acce[b], (((uint32_t)lt >> 1) & 1u) ^ 1u);
                 tc_fence_after();
-                const uint32_t d_tmem = tmem_base + (uint32_t)(b * KNN_BN);
                 for (int ks = 0; ks <= g.KS; ++ks, ++it) {
                     const int st = (int)(it % NS);
                     mbar_wait_sleep(&full[st], (it / NS) & 1u);
                     tc_fence_after();
-                    const uint32_t bs = smem_u32(sB + st * KNN_STAGE_BYTES);
-                    if (ks == g.KS) {  // norm block: |q|^2 + |r|^2 into the same accumulator
-                        const uint64_t an = umma_desc(anorm, KNN_BM * 16, 128);
-                        const uint64_t bn = umma_desc(bs, KNN_BN * 16, 128);
-                        umma_bf16(d_tmem, an, bn, idesc, 1u);
-                        if (g.cs == 1) umma_commit(&empty[st]);
-                        else umma_commit_mc(&empty[st], cmask);
-                        continue;
-                    }
+                    const uint32_t bs = smem_u32(sB + st * SB);
 #pragma unroll
-                    for (int j = 0; j < 2; ++j) {
-                        const int kk = ks * 2 + j;
-                        const uint64_t ah = umma_desc(a0 + (uint32_t)(2 * kk) * (KNN_BM * 16), KNN_BM * 16, 128);
-                        const uint64_t al = umma_desc(alo + (uint32_t)(2 * kk) * (KNN_BM * 16), KNN_BM * 16, 128);
-                        const uint64_t bh = umma_desc(bs + (uint32_t)(2 * j) * (KNN_BN * 16), KNN_BN * 16, 128);
-                        const uint64_t bl =
-                            umma_desc(bs + KNN_STAGE_BYTES / 2 + (uint32_t)(2 * j) * (KNN_BN * 16), KNN_BN * 16, 128);
-                        umma_bf16(d_tmem, ah, bh, idesc, (ks | j) ? 1u : 0u);
-                        if (g.passes == 3) {
-                            umma_bf16(d_tmem, ah, bl, idesc, 1u);
-                            umma_bf16(d_tmem, al, bh, idesc, 1u);
+                    for (int h = 0; h < QPC; ++h) {  // every query tile of the CTA on this stage
+                        const uint32_t d_tmem = tmem_base + (uint32_t)((b * QPC + h) * BN);
+                        const uint32_t a0 = smem_u32(sA) + (uint32_t)h * abytes;
+                        if (ks == g.KS) {  // norm block: |q|^2 + |r|^2 into the same accumulator
+                            const uint64_t an = umma_desc(a0 + (uint32_t)(g.Dp * 512), KNN_BM * 16, 128);
+                            const uint64_t bn = umma_desc(bs, BN * 16, 128);
+                            umma_bf16(d_tmem, an, bn, idesc, 1u);
+                            continue;
+                        }
+                        const uint32_t alo = a0 + (uint32_t)(g.Dp / 8) * (KNN_BM * 16);
+#pragma unroll
+                        for (int j = 0; j < 2; ++j) {
+                            const int kk = ks * 2 + j;
+                            const uint64_t ah = umma_desc(a0 + (uint32_t)(2 * kk) * (KNN_BM * 16), KNN_BM * 16, 128);
+                            const uint64_t al = umma_desc(alo + (uint32_t)(2 * kk) * (KNN_BM * 16), KNN_BM * 16, 128);
+                            const uint64_t bh = umma_desc(bs + (uint32_t)(2 * j) * (BN * 16), BN * 16, 128);
+                            const uint64_t bl = umma_desc(bs + SB / 2 + (uint32_t)(2 * j) * (BN * 16), BN * 16, 128);
+                            umma_bf16(d_tmem, ah, bh, idesc, (ks | j) ? 1u : 0u);
+                            if (g.passes == 3) {
+                                umma_bf16(d_tmem, ah, bl, idesc, 1u);
+                                umma_bf16(d_tmem, al, bh, idesc, 1u);
+                            }
                         }
                     }
                     // frees the stage (in every CTA of the cluster) when these MMAs complete
@@ -460,7 +473,9 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
         // ===== epilogue: one thread per query =====
         const int e = warp - 2;                   // 0..EW-1
         const int quad = warp & 3;                // TMEM lane quadrant this warp may access
-        const int half = e >> 2;                  // columns [half * WCOLS, (half + 1) * WCOLS) of every tile
+        const int half = (QPC == 1) ? (e >> 2) : 0;  // columns [half * WCOLS, (half + 1) * WCOLS) of every tile
+        const int hq = (QPC == 1) ? 0 : (e >> 2);    // query tile of the CTA this warp serves
+        const int qt = grp * QPC + hq;
         const int row = quad * 32 + (int)lane;    // query row within the tile
         const int64_t q = (int64_t)qt * KNN_BM + row;
         const bool qvalid = q < g.Q;
@@ -530,8 +545,8 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
             if (PROF) prof_wait += clock64() - cw0;
             const unsigned long long cc0 = PROF ? clock64() : 0;
             tc_fence_after();
-            const uint32_t taddr = tmem_base + ((uint32_t)(quad * 32) << 16) + (uint32_t)(b * KNN_BN);
-            if (!DUMP && !PIPE_ONLY && lt == 0 && g.k <= KNN_BN && (int64_t)t * KNN_BN + KNN_BN <= g.N &&
+            const uint32_t taddr = tmem_base + ((uint32_t)(quad * 32) << 16) + (uint32_t)((b * QPC + hq) * BN);
+            if (!DUMP && !PIPE_ONLY && lt == 0 && g.k <= BN && (int64_t)t * BN + BN <= g.N &&
                 (Fs > 0 || __any_sync(kFull, qvalid && (uint32_t)(T >> 32) == kSentKey))) {
                 // Starting bound without a fill phase: the exact k-th smallest distance of
                 // this first (full) tile, by bisection on the bits of the clamped value
@@ -544,7 +559,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                     const uint32_t cand = vb | (1u << bit);
                     uint32_t cnt = 0;
 #pragma unroll 1
-                    for (int c = 0; c < KNN_BN / 32; ++c) {
+                    for (int c = 0; c < BN / 32; ++c) {
                         uint32_t v[32];
                         tmem_ld32(taddr + (uint32_t)(c * 32), v);
 #pragma unroll
@@ -560,7 +575,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                     // histogram range: [max(0, tile minimum), k-th of the tile]
                     float mn = __int_as_float(0x7f800000);
 #pragma unroll 1
-                    for (int c = 0; c < KNN_BN / KNN_CW; ++c) {
+                    for (int c = 0; c < BN / KNN_CW; ++c) {
                         uint32_t v[KNN_CW];
                         tmem_ld64(taddr + (uint32_t)(c * KNN_CW), v);
 #pragma unroll
@@ -618,8 +633,8 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                 // 4-column group, one warp vote of the chunk minimum against each lane's
                 // bound; on a hit, one warp-uniform vote per group, and only groups some
                 // lane needs are visited (candidates appended, predicated, from registers).
-                const uint32_t colt = (uint32_t)t * KNN_BN;  // N < 2^31
-                const int nlim = (int)min((int64_t)KNN_BN, g.N - (int64_t)colt);  // valid columns of the tile
+                const uint32_t colt = (uint32_t)t * BN;  // N < 2^31
+                const int nlim = (int)min((int64_t)BN, g.N - (int64_t)colt);  // valid columns of the tile
                 auto scan32 = [&](const uint32_t(&v)[32], int c0) {
                     float gmn[8];
 #pragma unroll
@@ -681,7 +696,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                     if (v[0] == 0x7fc00001u && v[KNN_CW - 1] == 0x7fc00001u) n++;  // keep the load alive
                     continue;
                 }
-                const int64_t col0 = (int64_t)t * KNN_BN + c * KNN_CW;
+                const int64_t col0 = (int64_t)t * BN + c * KNN_CW;
                 // (knn_distances) the accumulator is d = |q|^2 + |r|^2 - 2 q.r; clamped at 0
                 float d[KNN_CW];
 #pragma unroll
@@ -739,8 +754,14 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     g.D = D;
     g.Dp = (D + KNN_KS - 1) / KNN_KS * KNN_KS;
     g.KS = g.Dp / KNN_KS;
-    g.NT = (int)((N + KNN_BN - 1) / KNN_BN);
     g.QT = (int)((Q + KNN_BM - 1) / KNN_BM);
+    // two query tiles per CTA on 128-reference tiles: every reference stage feeds 256
+    // queries (half the bytes landed in shared memory per distance); the pair of
+    // query images must fit next to the ring (D <= 128)
+    static const int qpc_env = env_int("KSEL_KNN_QPC", 1);
+    g.QPC = (qpc_env == 2 && g.Dp <= 128 && g.QT >= 2) ? 2 : 1;
+    g.BN = (g.QPC == 2) ? 128 : 256;
+    g.NT = (int)((N + g.BN - 1) / g.BN);
     static const int cs_env = [] {
         const int v = env_int("KSEL_KNN_CLUSTER", 1);  // experiments: cluster size 1, 2 or 4
         return (v == 2 || v == 4) ? v : 1;
@@ -752,8 +773,8 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     // multicast to all), cutting the L2 traffic per MMA by cs.  Measured on C4: no
     // gain (cs = 1 / 2 / 4: 6.79 / 6.95 / 8.16 ms; pipeline-only 1-pass 4.08 / 4.36 /
     // 5.14 ms), so L2 is not the floor and the default is cs = 1.
-    g.cs = (g.QT >= cs_env) ? cs_env : 1;
-    g.QTp = (g.QT + g.cs - 1) / g.cs * g.cs;
+    g.cs = (g.QPC == 1 && g.QT >= cs_env) ? cs_env : 1;
+    g.QTp = (g.QPC == 2) ? (g.QT + 1) / 2 : (g.QT + g.cs - 1) / g.cs * g.cs;  // CTA rows of the grid
     static const int passes_env = env_int("KSEL_KNN_PASSES", 3) == 1 ? 1 : 3;  // experiments only: 1 breaks the accuracy bound
     g.passes = passes_env;
     g.k = k;
@@ -761,20 +782,22 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     // room for >= 1 tile of candidates after narrowing to k; register narrowing holds 1152
     // register narrowing (<= 1280 pairs) for k' <= 128; larger queues get a pool with
     // room for 8 tiles of candidates between narrowings (radix select, pool_select64)
-    int P = (kk <= 128) ? 1152 : kk + 8 * KNN_BN;
+    int P = (kk <= 128) ? 1152 : kk + 8 * 256;
     g.P = (P + 31) / 32 * 32;
-    // ring depth: as many 32 KB stages as fit next to the resident query tile
-    const int fixed = 1024 + (g.Dp * 512 + KNN_NORM_A_BYTES) + KnnSmem::kHistBytes + KnnSmem::kDStageBytes + 512;
-    g.NS = (kMaxSmemPerBlock - fixed) / KNN_STAGE_BYTES;
+    static const int ew_env = env_int("KSEL_KNN_EW", 4) == 8 ? 8 : 4;  // experiments: 4 or 8 epilogue warps
+    g.halves = (g.QPC == 2) ? 1 : ew_env / 4;
+    g.EW = (g.QPC == 2) ? 8 : 4 * g.halves;
+    // ring depth: as many stages as fit next to the resident query tile(s)
+    const int fixed =
+        1024 + g.QPC * (g.Dp * 512 + KNN_NORM_A_BYTES) + KnnSmem::scratch(g.EW) + 512;
+    g.NS = (kMaxSmemPerBlock - fixed) / g.stage_bytes();
     if (g.NS > 6) g.NS = 6;
     g.idx_offset = idx_offset;
-    static const int ew_env = env_int("KSEL_KNN_EW", 4) == 8 ? 8 : 4;  // experiments: 4 or 8 epilogue warps
-    g.halves = ew_env / 4;
     static const int cap_env = env_int("KSEL_KNN_SOFTCAP", 0);  // experiments: narrow early (pool fill cap)
     // narrow before a pool reaches P when queues are small: the bound then tracks the
     // k-th of what has been seen more closely in cold CTAs (measured: 512 for k <= 128)
     const int cap = cap_env > 0 ? cap_env : (kk <= 128 ? 512 : g.P);
-    g.pcap = std::max(kk + 32 + KNN_BN / g.halves, std::min(g.P, cap));
+    g.pcap = std::max(kk + 32 + g.BN / g.halves, std::min(g.P, cap));
     g.ntiles = g.NT;
     g.tstride = 1;
     // first-wave CTAs sample 16 tiles (4096 references) for their starting bound
@@ -839,11 +862,17 @@ static cudaError_t knn_run(const float* ref, const float* query, const KnnGeom& 
         return (m >= 2 && m <= 4) ? m : 0;
     }();
     const bool ew8 = g.halves == 2;
-    auto kern = dump ? (ew8 ? knn_fused_kernel<1, 8> : knn_fused_kernel<1, 4>)
-              : mode_env == 2 ? (ew8 ? knn_fused_kernel<2, 8> : knn_fused_kernel<2, 4>)
-              : mode_env == 3 ? (ew8 ? knn_fused_kernel<3, 8> : knn_fused_kernel<3, 4>)
-              : mode_env == 4 ? knn_fused_kernel<4, 4>
-                              : (ew8 ? knn_fused_kernel<0, 8> : knn_fused_kernel<0, 4>);
+    auto kern = (g.QPC == 2)
+                    ? (dump ? knn_fused_kernel<1, 8, 128, 2>
+                       : mode_env == 2 ? knn_fused_kernel<2, 8, 128, 2>
+                       : mode_env == 3 ? knn_fused_kernel<3, 8, 128, 2>
+                       : mode_env == 4 ? knn_fused_kernel<4, 8, 128, 2>
+                                       : knn_fused_kernel<0, 8, 128, 2>)
+                : dump ? (ew8 ? knn_fused_kernel<1, 8, 256, 1> : knn_fused_kernel<1, 4, 256, 1>)
+                : mode_env == 2 ? (ew8 ? knn_fused_kernel<2, 8, 256, 1> : knn_fused_kernel<2, 4, 256, 1>)
+                : mode_env == 3 ? (ew8 ? knn_fused_kernel<3, 8, 256, 1> : knn_fused_kernel<3, 4, 256, 1>)
+                : mode_env == 4 ? knn_fused_kernel<4, 4, 256, 1>
+                                : (ew8 ? knn_fused_kernel<0, 8, 256, 1> : knn_fused_kernel<0, 4, 256, 1>);
     if (!dump && mode_env == 3) dump = reinterpret_cast<float*>(work + w.prof);
     e = ensure_smem_attr(reinterpret_cast<const void*>(kern), smem);
     if (e != cudaSuccess) return e;
@@ -851,7 +880,7 @@ static cudaError_t knn_run(const float* ref, const float* query, const KnnGeom& 
     cudaLaunchConfig_t cfg{};
     cudaLaunchAttribute attr[1];
     cfg.gridDim = dim3((unsigned)(g.QTp * g.S));
-    cfg.blockDim = dim3((unsigned)knn_threads(4 * g.halves));
+    cfg.blockDim = dim3((unsigned)knn_threads(g.EW));
     cfg.dynamicSmemBytes = (size_t)smem;
     cfg.stream = stream;
     attr[0].id = cudaLaunchAttributeClusterDimension;
