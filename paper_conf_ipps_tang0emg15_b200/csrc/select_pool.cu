@@ -176,9 +176,16 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads)
     uint32_t it_i = 0, it_blk = 0, it_off = 1, it_tail = np * step, it_p = 0;
     auto next_chunk = [&]() -> uint32_t {  // lane 0 only; chunk index relative to c_begin
         if ((order_mode & 3) == 2) {
-            const uint32_t c = it_p;
-            it_p += pstride;
-            if (it_p >= nm) it_p -= nm;
+            // the first and the last chunk first (they feed the starting bound: sorted rows,
+            // ascending or descending, then start from their exact k-th when k <= 512),
+            // then the strided permutation without those two
+            if (it_i < 2u && nm > 2u) return (it_i++ == 0u) ? 0u : nm - 1u;
+            uint32_t c;
+            do {
+                c = it_p;
+                it_p += pstride;
+                if (it_p >= nm) it_p -= nm;
+            } while (nm > 2u && (c == 0u || c == nm - 1u));
             return c;
         }
         if (it_i < np) return (it_i++) * step;
