@@ -381,3 +381,25 @@ def test_fuzz_merge(K, oracle_mod, seed):
         torch.cuda.synchronize()
         ev, ei = oracle_mod.merge(cv.cpu().numpy(), ci.cpu().numpy(), k)  # top-k of the union of the lists
         assert_same(ev, ei, gv, gi, "merge fuzz seed=%d case=%d S=%d kin=%d k=%d Q=%d %s" % (seed, case, S, kin, k, Q, dist))
+
+
+@pytest.mark.parametrize("seed", range(2))
+def test_fuzz_select_host(K, oracle_mod, seed):
+    # the host-buffer entry (double-buffered H2D / select / D2H): pinned and pageable
+    # inputs, workspaces from one block to many
+    rng = np.random.default_rng(4000 + seed)
+    for case in range(4):
+        N = int(rng.integers(1, 200000))
+        Q = int(rng.integers(1, max(2, 3_000_000 // N)))
+        k = int(rng.integers(1, min(N, 1024) + 1))
+        dist = str(rng.choice(synth.DISTS))
+        x = synth.rows(dist, 4100 + seed * 10 + case, 0, Q, N)
+        if case % 2 == 0:
+            x = x.pin_memory()
+        need = K.ksel_select_host_workspace(N, k)
+        ws = torch.empty(max(need // int(rng.integers(1, 9)), need // 8 + 1), dtype=torch.uint8, device="cuda")
+        if ws.numel() < need // 8:
+            ws = torch.empty(need, dtype=torch.uint8, device="cuda")
+        gv, gi = K.ksel_select_host(x, k, workspace=ws)
+        ev, ei = oracle_mod.select(x.numpy(), k)
+        assert_same(ev, ei, gv.numpy(), gi.numpy(), "host fuzz seed=%d case=%d Q=%d N=%d k=%d %s" % (seed, case, Q, N, k, dist))
