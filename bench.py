@@ -312,6 +312,21 @@ def bench_select(args, rank, world, local_rank, dev, K, tdist):
     # roofline of the dominant (only) kernel, timed live on the launching stream
     peak, peak_src = load_peaks()
     alg_bytes = Qr * (4.0 * N + 8.0 * k)
+    # context for the denominator: a plain read-only stream over the same resident
+    # input (torch's amax reduction, not our code), best of 3
+    stream_gbs = None
+    if rank == 0:
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        best = None
+        for _ in range(3):
+            torch.cuda.synchronize()
+            e0.record()
+            torch.amax(x, dim=1)
+            e1.record()
+            torch.cuda.synchronize()
+            t = e0.elapsed_time(e1)
+            best = t if best is None else min(best, t)
+        stream_gbs = Qr * N * 4.0 / (best / 1e3) / 1e9
     achieved = alg_bytes / (kern_ms / 1e3) / 1e9
     cfg = select_config(Qr, N, k, dist, world)
     workload = cfg["workload"]
@@ -327,7 +342,9 @@ def bench_select(args, rank, world, local_rank, dev, K, tdist):
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": load_traffic(workload), "peak_source": peak_src,
                          "kernel": "ksel_pool_kernel", "kernel_ms": kern_ms, "kernel_launches_timed": kern_n,
-                         "bytes_per_launch": alg_bytes, "bytes_formula": "Q*(4N+8k)"},
+                         "bytes_per_launch": alg_bytes, "bytes_formula": "Q*(4N+8k)",
+                         "read_stream_gbs": stream_gbs,
+                         "read_stream_note": "torch.amax over the same resident input (context, not the peak)"},
             "gpu_launches": launches,
             "clocks": clocks,
         }
