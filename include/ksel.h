@@ -48,7 +48,8 @@ typedef enum {
     KSEL_ERR_INVALID_ARG = 1, /* null pointer, bad size, misalignment, aliasing */
     KSEL_ERR_UNSUPPORTED = 2, /* valid request outside this build's range (k > 1024) */
     KSEL_ERR_CUDA = 3,        /* a CUDA runtime call or kernel launch failed */
-    KSEL_ERR_NO_DEVICE = 4    /* no sm_100 device is current */
+    KSEL_ERR_NO_DEVICE = 4,   /* no sm_100 device is current */
+    KSEL_ERR_TIMEOUT = 5      /* a device-side flag wait gave up (ksel_device_status) */
 } ksel_status;
 
 #define KSEL_MAX_K 1024
@@ -112,8 +113,12 @@ KSEL_API int ksel_select_config(const float* dist, int64_t Q, int64_t N, int k, 
  * blocks host->device, selects, and copies results back, double-buffered
  * across two internal copy streams, using the caller's device workspace
  * `d_work` of `work_bytes` bytes (query the minimum with
- * ksel_select_host_workspace).  Returns after the results are in host memory
- * (this call synchronises).  Same ordering/bit-exactness as ksel_select. */
+ * ksel_select_host_workspace).  The copies start only after all work already
+ * queued on `stream` (the workspace and the output buffers may still be in use
+ * by it).  Returns after the results are in host memory (this call
+ * synchronises; on an error it also waits for every copy it issued, so no
+ * transfer touches the host buffers after it returns).  Same ordering /
+ * bit-exactness as ksel_select. */
 KSEL_API size_t ksel_select_host_workspace(int64_t N, int k);
 KSEL_API int ksel_select_host(const float* h_dist, int64_t Q, int64_t N, int k, float* h_out_val,
                      int32_t* h_out_idx, void* d_work, size_t work_bytes, void* stream);
@@ -234,11 +239,15 @@ KSEL_API int ksel_select_paper(const float* dist_t, int64_t Q, int64_t N, int k,
  *   != NULL, list s is read only after *ready[s] reached `epoch` (as in
  *   ksel_flag_wait), with volatile loads.  Output, limits and errors as
  *   ksel_merge.
- * Waits that do not complete within 60 s trap (the stream then reports a CUDA
- * error) rather than hang.  Every kernel taking part in such an exchange must
- * already be loaded when a wait is pending (CUDA lazy loading may otherwise
- * serialise behind the spinning wait): run one warm-up call first, as KnnP2P
- * does. */
+ * A wait that does not complete within the flag timeout (ksel_set_flag_timeout,
+ * default 600 s) gives up instead of hanging: the waiting kernel records
+ * KSEL_ERR_TIMEOUT in a library-owned word of mapped host memory and returns
+ * (the CUDA context stays usable; the results of that exchange are invalid).
+ * ksel_device_status() -- call it after synchronising the stream -- returns
+ * KSEL_OK or KSEL_ERR_TIMEOUT; ksel_device_status_clear() resets it.  Every
+ * kernel taking part in such an exchange must already be loaded when a wait is
+ * pending (CUDA lazy loading may otherwise serialise behind the spinning wait):
+ * run one warm-up call first, as KnnP2P does. */
 KSEL_API size_t ksel_ipc_handle_size(void);
 KSEL_API int ksel_ipc_alloc(size_t bytes, void** d_ptr, void* handle_out);
 KSEL_API int ksel_ipc_open(const void* handle, void** d_ptr);
@@ -249,6 +258,10 @@ KSEL_API int ksel_flag_wait(const uint32_t* const* d_flags, int n, uint32_t valu
 KSEL_API int ksel_merge_lists(const float* const* vals, const int32_t* const* idxs, int S, int64_t Q, int kin,
                               int k, float* out_val, int32_t* out_idx, const uint32_t* const* ready,
                               uint32_t epoch, void* stream);
+/* seconds > 0: flag-wait timeout of waits enqueued from now on (KSEL_ERR_INVALID_ARG otherwise). */
+KSEL_API int ksel_set_flag_timeout(double seconds);
+KSEL_API int ksel_device_status(void);
+KSEL_API int ksel_device_status_clear(void);
 
 /* Live per-kernel timing (measurement support for bench.py): while enabled,
  * every entry point records a pair of CUDA events on its stream around its

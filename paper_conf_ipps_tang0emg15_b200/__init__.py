@@ -75,8 +75,10 @@ _lib.ksel_ipc_free.argtypes = [_p]
 _lib.ksel_flag_signal.argtypes = [_p, ctypes.c_uint32, _p]
 _lib.ksel_flag_wait.argtypes = [_p, _i32, ctypes.c_uint32, _p]
 _lib.ksel_merge_lists.argtypes = [_p, _p, _i32, _i64, _i32, _i32, _p, _p, _p, ctypes.c_uint32, _p]
+_lib.ksel_set_flag_timeout.argtypes = [ctypes.c_double]
 for _f in (_lib.ksel_ipc_alloc, _lib.ksel_ipc_open, _lib.ksel_ipc_close, _lib.ksel_ipc_free, _lib.ksel_flag_signal,
-           _lib.ksel_flag_wait, _lib.ksel_merge_lists):
+           _lib.ksel_flag_wait, _lib.ksel_merge_lists, _lib.ksel_set_flag_timeout, _lib.ksel_device_status,
+           _lib.ksel_device_status_clear):
     _f.restype = ctypes.c_int
 for _f in (_lib.ksel_select, _lib.ksel_select_config, _lib.ksel_select_host, _lib.ksel_merge, _lib.knn_search, _lib.ksel_version):
     _f.restype = ctypes.c_int
@@ -88,7 +90,8 @@ PB_NONE, PB_BUFFER, PB_FULL, PB_FULL_SORTED = 0, 1, 2, 3
 EXPORTS = ("ksel_select", "ksel_select_workspace", "ksel_select_ex", "ksel_select_config", "ksel_select_host_workspace", "ksel_select_host", "ksel_merge",
            "knn_search_workspace", "knn_search", "knn_graph_workspace", "knn_graph", "knn_distances_workspace", "knn_distances", "ksel_timing_enable", "ksel_timing_collect", "ksel_strerror",
            "ksel_version", "ksel_launch_count", "ksel_select_paper_workspace", "ksel_select_paper", "ksel_ipc_handle_size", "ksel_ipc_alloc", "ksel_ipc_open",
-           "ksel_ipc_close", "ksel_ipc_free", "ksel_flag_signal", "ksel_flag_wait", "ksel_merge_lists")
+           "ksel_ipc_close", "ksel_ipc_free", "ksel_flag_signal", "ksel_flag_wait", "ksel_merge_lists",
+           "ksel_set_flag_timeout", "ksel_device_status", "ksel_device_status_clear")
 
 
 class KselError(RuntimeError):
@@ -138,6 +141,29 @@ def _stream(device) -> int:
     return torch.cuda.current_stream(device).cuda_stream
 
 
+def _out(t, name: str, shape, dtype, device):
+    """A caller-supplied output: exact shape, dtype, contiguous, on `device` (the kernels
+    write every element through the raw pointer, so a mismatch would corrupt memory)."""
+    if not isinstance(t, torch.Tensor):
+        raise TypeError("%s must be a tensor" % name)
+    if tuple(t.shape) != tuple(shape) or t.dtype != dtype or not t.is_contiguous() or t.device != device:
+        raise TypeError("%s must be a contiguous %s tensor of shape %s on %s (got %s %s on %s%s)"
+                        % (name, dtype, tuple(shape), device, t.dtype, tuple(t.shape), t.device,
+                           "" if t.is_contiguous() else ", non-contiguous"))
+
+
+def _workspace(ws, need: int, device, name: str = "workspace"):
+    if not isinstance(ws, torch.Tensor) or ws.device != device or not ws.is_contiguous():
+        raise TypeError("%s must be a contiguous tensor on %s" % (name, device))
+    if ws.numel() * ws.element_size() < need:
+        raise ValueError("%s holds %d bytes, %d needed" % (name, ws.numel() * ws.element_size(), need))
+
+
+def _same_device(a: torch.Tensor, b: torch.Tensor, an: str, bn: str):
+    if a.device != b.device:
+        raise ValueError("%s and %s must be on the same device (%s vs %s)" % (an, bn, a.device, b.device))
+
+
 def ksel_select_workspace(Q: int, N: int, k: int) -> int:
     return int(_lib.ksel_select_workspace(Q, N, k))
 
@@ -157,15 +183,19 @@ def ksel_select(dist: torch.Tensor, k: int, out_val: torch.Tensor | None = None,
     Q, N = dist.shape
     if out_val is None:
         out_val = torch.empty((Q, k), dtype=torch.float32, device=dist.device)
+    _out(out_val, "out_val", (Q, k), torch.float32, dist.device)
     if out_idx is None:
         out_idx = torch.empty((Q, k), dtype=torch.int32, device=dist.device)
+    _out(out_idx, "out_idx", (Q, k), torch.int32, dist.device)
     with torch.cuda.device(dist.device):
         need = ksel_select_workspace(Q, N, k) if (algo == ALGO_AUTO and warps_per_row == 0 and split_rows) else 0
         if need > 0:
             if workspace is None:
                 workspace = torch.empty(need, dtype=torch.uint8, device=dist.device)
+            _workspace(workspace, need, dist.device)
             st = _lib.ksel_select_ex(dist.data_ptr(), Q, N, k, out_val.data_ptr(), out_idx.data_ptr(),
-                                     workspace.data_ptr(), workspace.numel(), _stream(dist.device))
+                                     workspace.data_ptr(), workspace.numel() * workspace.element_size(),
+                                     _stream(dist.device))
         elif algo == ALGO_AUTO and warps_per_row == 0:
             st = _lib.ksel_select(dist.data_ptr(), Q, N, k, out_val.data_ptr(), out_idx.data_ptr(),
                                   _stream(dist.device))
@@ -193,14 +223,19 @@ def ksel_select_host(dist: torch.Tensor, k: int, out_val: torch.Tensor | None = 
     dev = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
     if out_val is None:
         out_val = torch.empty((Q, k), dtype=torch.float32, pin_memory=dist.is_pinned())
+    _out(out_val, "out_val", (Q, k), torch.float32, torch.device("cpu"))
     if out_idx is None:
         out_idx = torch.empty((Q, k), dtype=torch.int32, pin_memory=dist.is_pinned())
+    _out(out_idx, "out_idx", (Q, k), torch.int32, torch.device("cpu"))
     if workspace is None:
         workspace = torch.empty(ksel_select_host_workspace(N, k), dtype=torch.uint8, device=dev)
+    if workspace.device.type != "cuda" or not workspace.is_contiguous():
+        raise TypeError("workspace must be a contiguous CUDA tensor")
+    dev = workspace.device
     with torch.cuda.device(dev):
         _check("ksel_select_host", _lib.ksel_select_host(
             dist.data_ptr(), Q, N, k, out_val.data_ptr(), out_idx.data_ptr(), workspace.data_ptr(),
-            workspace.numel(), _stream(dev)))
+            workspace.numel() * workspace.element_size(), _stream(dev)))
     return out_val, out_idx
 
 
@@ -210,11 +245,14 @@ def ksel_merge(cand_val: torch.Tensor, cand_idx: torch.Tensor, k: int,
     _dev_f32(cand_val, "cand_val", 3)
     if cand_idx.dtype != torch.int32 or cand_idx.shape != cand_val.shape or not cand_idx.is_contiguous():
         raise TypeError("cand_idx must be a contiguous int32 tensor shaped like cand_val")
+    _same_device(cand_val, cand_idx, "cand_val", "cand_idx")
     S, Q, kin = cand_val.shape
     if out_val is None:
         out_val = torch.empty((Q, k), dtype=torch.float32, device=cand_val.device)
+    _out(out_val, "out_val", (Q, k), torch.float32, cand_val.device)
     if out_idx is None:
         out_idx = torch.empty((Q, k), dtype=torch.int32, device=cand_val.device)
+    _out(out_idx, "out_idx", (Q, k), torch.int32, cand_val.device)
     with torch.cuda.device(cand_val.device):
         _check("ksel_merge", _lib.ksel_merge(cand_val.data_ptr(), cand_idx.data_ptr(), Q, S, kin, k,
                                              out_val.data_ptr(), out_idx.data_ptr(),
@@ -232,19 +270,24 @@ def knn_search(ref: torch.Tensor, query: torch.Tensor, k: int, idx_offset: int =
     """k nearest references (squared L2) of every query; ref [N, D], query [Q, D]."""
     _dev_f32(ref, "ref", 2)
     _dev_f32(query, "query", 2)
+    _same_device(ref, query, "ref", "query")
     N, D = ref.shape
     Q = query.shape[0]
     if query.shape[1] != D:
         raise ValueError("ref and query must share D")
     if out_dist is None:
         out_dist = torch.empty((Q, k), dtype=torch.float32, device=ref.device)
+    _out(out_dist, "out_dist", (Q, k), torch.float32, ref.device)
     if out_idx is None:
         out_idx = torch.empty((Q, k), dtype=torch.int32, device=ref.device)
+    _out(out_idx, "out_idx", (Q, k), torch.int32, ref.device)
     need = knn_search_workspace(N, Q, D, k)
     if workspace is None and need > 0:
         workspace = torch.empty(need, dtype=torch.uint8, device=ref.device)
+    if workspace is not None:
+        _workspace(workspace, need, ref.device)
     wptr = workspace.data_ptr() if workspace is not None else 0
-    wlen = workspace.numel() if workspace is not None else 0
+    wlen = workspace.numel() * workspace.element_size() if workspace is not None else 0
     with torch.cuda.device(ref.device):
         _check("knn_search", _lib.knn_search(ref.data_ptr(), query.data_ptr(), N, Q, D, k,
                                              out_dist.data_ptr(), out_idx.data_ptr(), idx_offset,
@@ -263,13 +306,17 @@ def knn_graph(points: torch.Tensor, k: int, out_dist: torch.Tensor | None = None
     N, D = points.shape
     if out_dist is None:
         out_dist = torch.empty((N, k), dtype=torch.float32, device=points.device)
+    _out(out_dist, "out_dist", (N, k), torch.float32, points.device)
     if out_idx is None:
         out_idx = torch.empty((N, k), dtype=torch.int32, device=points.device)
+    _out(out_idx, "out_idx", (N, k), torch.int32, points.device)
     need = knn_graph_workspace(N, D, k)
     if workspace is None and need > 0:
         workspace = torch.empty(need, dtype=torch.uint8, device=points.device)
+    if workspace is not None:
+        _workspace(workspace, need, points.device)
     wptr = workspace.data_ptr() if workspace is not None else 0
-    wlen = workspace.numel() if workspace is not None else 0
+    wlen = workspace.numel() * workspace.element_size() if workspace is not None else 0
     with torch.cuda.device(points.device):
         _check("knn_graph", _lib.knn_graph(points.data_ptr(), N, D, k, out_dist.data_ptr(), out_idx.data_ptr(),
                                            wptr, wlen, _stream(points.device)))
@@ -282,8 +329,10 @@ def knn_distances(ref: torch.Tensor, query: torch.Tensor, out: torch.Tensor | No
     _dev_f32(query, "query", 2)
     N, D = ref.shape
     Q = query.shape[0]
+    _same_device(ref, query, "ref", "query")
     if out is None:
         out = torch.empty((Q, N), dtype=torch.float32, device=ref.device)
+    _out(out, "out", (Q, N), torch.float32, ref.device)
     ws = torch.empty(max(1, int(_lib.knn_distances_workspace(N, Q, D))), dtype=torch.uint8, device=ref.device)
     with torch.cuda.device(ref.device):
         _check("knn_distances", _lib.knn_distances(ref.data_ptr(), query.data_ptr(), N, Q, D, out.data_ptr(),
@@ -343,6 +392,21 @@ def flag_wait(flag_ptrs, value: int) -> None:
     arr = _ptr_array(flag_ptrs)
     _check("ksel_flag_wait", _lib.ksel_flag_wait(arr, len(flag_ptrs), value & 0xFFFFFFFF,
                                                  torch.cuda.current_stream().cuda_stream))
+
+
+def set_flag_timeout(seconds: float) -> None:
+    """Timeout of device-side flag waits enqueued from now on (default 600 s)."""
+    _check("ksel_set_flag_timeout", _lib.ksel_set_flag_timeout(float(seconds)))
+
+
+def device_status() -> int:
+    """0, or 5 (KSEL_ERR_TIMEOUT) if a device-side flag wait gave up since the last clear.
+    Synchronise the stream(s) first."""
+    return int(_lib.ksel_device_status())
+
+
+def device_status_clear() -> None:
+    _lib.ksel_device_status_clear()
 
 
 def ksel_merge_lists(val_ptrs, idx_ptrs, Q: int, kin: int, k: int, out_val: torch.Tensor, out_idx: torch.Tensor,

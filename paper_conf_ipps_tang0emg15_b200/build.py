@@ -28,6 +28,11 @@ NVCC_FLAGS = [
     "-Xptxas", "-warn-spills",
     "-I" + INCLUDE, "-I" + CSRC,
 ]
+# Timing-experiment kernel variants (pipeline-only / counter modes, 1-pass MMA, other
+# epilogue shapes) are compiled only into an experiments build; the product library
+# (the default) contains none of them and reads no result-affecting knob.
+if os.environ.get("KSEL_BUILD_EXPERIMENTS") == "1":
+    NVCC_FLAGS.append("-DKSEL_EXPERIMENTS")
 
 
 def _sources():

@@ -165,6 +165,7 @@ const char* ksel_strerror(int status) {
         case KSEL_ERR_UNSUPPORTED: return "unsupported configuration (k > 1024?)";
         case KSEL_ERR_CUDA: return "CUDA runtime error";
         case KSEL_ERR_NO_DEVICE: return "no sm_100 (B200) device is current";
+        case KSEL_ERR_TIMEOUT: return "a device-side flag wait timed out (exchange results invalid)";
         default: return "unknown ksel status";
     }
 }
@@ -375,6 +376,7 @@ int ksel_select_host(const float* h_dist, int64_t Q, int64_t N, int k, float* h_
 
     cudaStream_t h2d = nullptr, d2h = nullptr;
     cudaEvent_t ev_in[2] = {nullptr, nullptr}, ev_comp[2] = {nullptr, nullptr}, ev_out[2] = {nullptr, nullptr};
+    cudaEvent_t ev_entry = nullptr;
     cudaError_t e = cudaStreamCreateWithFlags(&h2d, cudaStreamNonBlocking);
     if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&d2h, cudaStreamNonBlocking);
     for (int s = 0; s < 2 && e == cudaSuccess; ++s) {
@@ -382,6 +384,14 @@ int ksel_select_host(const float* h_dist, int64_t Q, int64_t N, int k, float* h_
         if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ev_comp[s], cudaEventDisableTiming);
         if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ev_out[s], cudaEventDisableTiming);
     }
+    // Stream order: the copy streams start only after everything already queued on the
+    // caller's stream (the workspace may be memory a pending kernel of that stream still
+    // uses, e.g. a block just recycled by a caching allocator; a pending D2H copy may still
+    // be filling the output host buffers).
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ev_entry, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventRecord(ev_entry, cs);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(h2d, ev_entry, 0);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(d2h, ev_entry, 0);
     int64_t blk = 0;
     for (int64_t r0 = 0; r0 < Q && e == cudaSuccess; r0 += rows, ++blk) {
         const int s = (int)(blk & 1);
@@ -401,7 +411,15 @@ int ksel_select_host(const float* h_dist, int64_t Q, int64_t N, int k, float* h_
             e = cudaMemcpyAsync(h_out_idx + r0 * k, si[s], (size_t)nr * (size_t)k * 4u, cudaMemcpyDeviceToHost, d2h);
         if (e == cudaSuccess) e = cudaEventRecord(ev_out[s], d2h);
     }
-    if (e == cudaSuccess) e = cudaStreamSynchronize(d2h);
+    if (e == cudaSuccess) {
+        e = cudaStreamSynchronize(d2h);
+    } else {
+        // error path: no copy may still touch the caller's host buffers after return
+        if (h2d) cudaStreamSynchronize(h2d);
+        cudaStreamSynchronize(cs);
+        if (d2h) cudaStreamSynchronize(d2h);
+    }
+    if (ev_entry) cudaEventDestroy(ev_entry);
     for (int s = 0; s < 2; ++s) {
         if (ev_in[s]) cudaEventDestroy(ev_in[s]);
         if (ev_comp[s]) cudaEventDestroy(ev_comp[s]);

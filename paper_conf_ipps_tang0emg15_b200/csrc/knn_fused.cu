@@ -758,14 +758,22 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     // two query tiles per CTA on 128-reference tiles: every reference stage feeds 256
     // queries (half the bytes landed in shared memory per distance); the pair of
     // query images must fit next to the ring (D <= 128)
+#ifdef KSEL_EXPERIMENTS
     static const int qpc_env = env_int("KSEL_KNN_QPC", 1);
+#else
+    constexpr int qpc_env = 1;
+#endif
     g.QPC = (qpc_env == 2 && g.Dp <= 128 && g.QT >= 2) ? 2 : 1;
     g.BN = (g.QPC == 2) ? 128 : 256;
     g.NT = (int)((N + g.BN - 1) / g.BN);
+#ifdef KSEL_EXPERIMENTS
     static const int cs_env = [] {
         const int v = env_int("KSEL_KNN_CLUSTER", 1);  // experiments: cluster size 1, 2 or 4
         return (v == 2 || v == 4) ? v : 1;
     }();
+#else
+    constexpr int cs_env = 1;
+#endif
     // Every CTA streams its whole reference range through L2 -> shared memory (4 B per
     // dim and reference per 128 queries): with one CTA per query tile that stream, not
     // the tensor pipe, is the floor (measured: ~40 B/clk/SM, the chip's L2 -> SM rate).
@@ -775,7 +783,11 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     // 5.14 ms), so L2 is not the floor and the default is cs = 1.
     g.cs = (g.QPC == 1 && g.QT >= cs_env) ? cs_env : 1;
     g.QTp = (g.QPC == 2) ? (g.QT + 1) / 2 : (g.QT + g.cs - 1) / g.cs * g.cs;  // CTA rows of the grid
+#ifdef KSEL_EXPERIMENTS
     static const int passes_env = env_int("KSEL_KNN_PASSES", 3) == 1 ? 1 : 3;  // experiments only: 1 breaks the accuracy bound
+#else
+    constexpr int passes_env = 3;
+#endif
     g.passes = passes_env;
     g.k = k;
     const int kk = k < 32 ? 32 : k;
@@ -784,7 +796,11 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     // room for 8 tiles of candidates between narrowings (radix select, pool_select64)
     int P = (kk <= 128) ? 1152 : kk + 8 * 256;
     g.P = (P + 31) / 32 * 32;
+#ifdef KSEL_EXPERIMENTS
     static const int ew_env = env_int("KSEL_KNN_EW", 4) == 8 ? 8 : 4;  // experiments: 4 or 8 epilogue warps
+#else
+    constexpr int ew_env = 4;
+#endif
     g.halves = (g.QPC == 2) ? 1 : ew_env / 4;
     g.EW = (g.QPC == 2) ? 8 : 4 * g.halves;
     // ring depth: as many stages as fit next to the resident query tile(s)
@@ -857,7 +873,10 @@ static cudaError_t knn_run(const float* ref, const float* query, const KnnGeom& 
     e = cudaMemsetAsync(work + w.qthr, 0xff, (size_t)g.Q * 8, stream);  // "no bound yet"
     if (e != cudaSuccess) return e;
     const int smem = KnnSmem::total(g);
-    static const int mode_env = [] {  // experiments: 2 pipeline only, 3 counters, 4 no TMEM reads
+#ifdef KSEL_EXPERIMENTS
+    // Timing experiments only (a -DKSEL_EXPERIMENTS build; the product library has none of
+    // these): 2 pipeline only, 3 counters, 4 no TMEM reads -- modes 2 and 4 return no result.
+    static const int mode_env = [] {
         const int m = env_int("KSEL_KNN_MODE", 0);
         return (m >= 2 && m <= 4) ? m : 0;
     }();
@@ -873,6 +892,10 @@ static cudaError_t knn_run(const float* ref, const float* query, const KnnGeom& 
                 : mode_env == 3 ? (ew8 ? knn_fused_kernel<3, 8, 256, 1> : knn_fused_kernel<3, 4, 256, 1>)
                 : mode_env == 4 ? knn_fused_kernel<4, 4, 256, 1>
                                 : (ew8 ? knn_fused_kernel<0, 8, 256, 1> : knn_fused_kernel<0, 4, 256, 1>);
+#else
+    constexpr int mode_env = 0;
+    auto kern = dump ? knn_fused_kernel<1, 4, 256, 1> : knn_fused_kernel<0, 4, 256, 1>;
+#endif
     if (!dump && mode_env == 3) dump = reinterpret_cast<float*>(work + w.prof);
     e = ensure_smem_attr(reinterpret_cast<const void*>(kern), smem);
     if (e != cudaSuccess) return e;

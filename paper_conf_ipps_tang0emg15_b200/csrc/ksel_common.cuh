@@ -192,9 +192,15 @@ __device__ __forceinline__ void warr_get(const WArr<R>& a, int pos, uint32_t& k,
     i = __shfl_sync(kFull, ti, pos & 31);
 }
 
-// Device-side flag waits (ksel_flag_wait, ksel_merge_lists) give up after this long
-// with a trap (a sticky CUDA error the host sees) instead of hanging forever.
-constexpr uint64_t kFlagTimeoutNs = 60ull * 1000000000ull;
+// Device-side flag waits (ksel_flag_wait, ksel_merge_lists) give up after a timeout
+// (a kernel parameter) and record it in a mapped host word instead of hanging or
+// trapping (a trap would kill the context; ksel_device_status reports it).
+__device__ __forceinline__ void note_timeout(uint32_t* err) {
+    if (err) {
+        atomicOr(err, 1u);
+        __threadfence_system();
+    }
+}
 __device__ __forceinline__ uint64_t globaltimer_ns() {
     uint64_t t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));

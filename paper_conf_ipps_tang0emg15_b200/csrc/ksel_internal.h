@@ -72,7 +72,15 @@ struct MergeLists {
     const uint32_t* ready[kMaxLists];
     uint32_t epoch;
     int vol;
+    uint32_t* err;        // device view of the timeout word (ready != NULL only)
+    uint64_t timeout_ns;  // flag-wait timeout
 };
+
+// Device-side flag waits give up after flag_timeout_ns() and OR KSEL_ERR_TIMEOUT's bit
+// into a word of mapped (host) memory; device_error_word() is its device pointer
+// (lazily created once per process; nullptr if the mapping failed).
+uint32_t* device_error_word();
+uint64_t flag_timeout_ns();
 cudaError_t launch_merge(const MergeLists& L, int64_t Q, int S, int kin, int k, float* out_val, int32_t* out_idx,
                          cudaStream_t stream);
 

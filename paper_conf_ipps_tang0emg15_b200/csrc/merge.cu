@@ -58,7 +58,10 @@ __device__ __forceinline__ void wait_ready(const MergeLists& L, int s) {
             asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(L.ready[s]) : "memory");
             if ((int32_t)(v - L.epoch) >= 0) break;
             __nanosleep(256);
-            if (globaltimer_ns() - t0 > kFlagTimeoutNs) __trap();  // a producer that never signals: fail loudly
+            if (globaltimer_ns() - t0 > L.timeout_ns) {  // a producer that never signals: give up, report
+                note_timeout(L.err);
+                break;
+            }
         }
     }
     __syncwarp();

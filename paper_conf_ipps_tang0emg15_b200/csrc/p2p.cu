@@ -19,7 +19,9 @@
 // acquire flags, the pointer-table merge); the orchestration lives in
 // paper_conf_ipps_tang0emg15_b200/dist.py (KnnP2P).
 #include <cstdint>
+#include <atomic>
 #include <cstring>
+#include <mutex>
 
 #include <cuda_runtime.h>
 
@@ -40,7 +42,8 @@ struct FlagSet {
     const uint32_t* f[kMaxLists];
 };
 
-__global__ void flag_wait_kernel(const __grid_constant__ FlagSet fs, int n, uint32_t value) {
+__global__ void flag_wait_kernel(const __grid_constant__ FlagSet fs, int n, uint32_t value, uint32_t* err,
+                                 uint64_t timeout_ns) {
     const int j = (int)threadIdx.x;
     if (j < n) {
         uint32_t v;
@@ -49,18 +52,63 @@ __global__ void flag_wait_kernel(const __grid_constant__ FlagSet fs, int n, uint
             asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(fs.f[j]) : "memory");
             if ((int32_t)(v - value) >= 0) break;
             __nanosleep(500);
-            if (globaltimer_ns() - t0 > kFlagTimeoutNs) __trap();  // a peer that never signals: fail loudly
+            if (globaltimer_ns() - t0 > timeout_ns) {  // a peer that never signals: give up, report
+                note_timeout(err);
+                break;
+            }
         }
     }
     __syncthreads();
     __threadfence_system();
 }
 
+static std::mutex g_err_mu;
+static uint32_t* g_err_host = nullptr;  // mapped pinned host word (written by the device)
+static uint32_t* g_err_dev = nullptr;
+static std::atomic<uint64_t> g_timeout_ns{600ull * 1000000000ull};
+
+uint32_t* device_error_word() {
+    std::lock_guard<std::mutex> lock(g_err_mu);
+    if (!g_err_dev) {
+        void* h = nullptr;
+        if (cudaHostAlloc(&h, 64, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) return nullptr;
+        void* d = nullptr;
+        if (cudaHostGetDevicePointer(&d, h, 0) != cudaSuccess) {
+            cudaFreeHost(h);
+            return nullptr;
+        }
+        static_cast<volatile uint32_t*>(h)[0] = 0u;
+        g_err_host = static_cast<uint32_t*>(h);
+        g_err_dev = static_cast<uint32_t*>(d);
+    }
+    return g_err_dev;
+}
+
+uint64_t flag_timeout_ns() { return g_timeout_ns.load(std::memory_order_relaxed); }
+
 }  // namespace ksel
 
 using namespace ksel;
 
 extern "C" {
+
+int ksel_set_flag_timeout(double seconds) {
+    if (!(seconds > 0.0) || seconds > 1e9) return KSEL_ERR_INVALID_ARG;
+    g_timeout_ns.store((uint64_t)(seconds * 1e9), std::memory_order_relaxed);
+    return KSEL_OK;
+}
+
+int ksel_device_status(void) {
+    std::lock_guard<std::mutex> lock(g_err_mu);
+    if (!g_err_host) return KSEL_OK;
+    return (static_cast<volatile uint32_t*>(g_err_host)[0] != 0u) ? KSEL_ERR_TIMEOUT : KSEL_OK;
+}
+
+int ksel_device_status_clear(void) {
+    std::lock_guard<std::mutex> lock(g_err_mu);
+    if (g_err_host) static_cast<volatile uint32_t*>(g_err_host)[0] = 0u;
+    return KSEL_OK;
+}
 
 size_t ksel_ipc_handle_size(void) { return sizeof(cudaIpcMemHandle_t); }
 
@@ -109,7 +157,7 @@ int ksel_flag_wait(const uint32_t* const* d_flags, int n, uint32_t value, void* 
         if (!d_flags[j] || (reinterpret_cast<uintptr_t>(d_flags[j]) & 3u)) return KSEL_ERR_INVALID_ARG;
         fs.f[j] = d_flags[j];
     }
-    flag_wait_kernel<<<1, 64, 0, (cudaStream_t)stream>>>(fs, n, value);
+    flag_wait_kernel<<<1, 64, 0, (cudaStream_t)stream>>>(fs, n, value, device_error_word(), flag_timeout_ns());
     note_launch();
     return cudaGetLastError() == cudaSuccess ? KSEL_OK : KSEL_ERR_CUDA;
 }
@@ -132,6 +180,8 @@ int ksel_merge_lists(const float* const* vals, const int32_t* const* idxs, int S
     }
     L.epoch = epoch;
     L.vol = ready ? 1 : 0;
+    L.err = ready ? device_error_word() : nullptr;
+    L.timeout_ns = flag_timeout_ns();
     DevInfo di;
     int st = current_device_info(&di);
     if (st) return st;

@@ -198,6 +198,15 @@ class KnnP2P:
         self.epoch += 1
         return mv, mi, (q0, q1)
 
+    def check(self):
+        """Synchronise and raise if a device-side flag wait of the exchange timed out
+        (a peer that never signalled: the results of that step are invalid)."""
+        from . import KselError, device_status
+        torch.cuda.synchronize()
+        st = device_status()
+        if st:
+            raise KselError("KnnP2P exchange", st)
+
     def close(self):
         from . import ipc_close, ipc_free
         torch.cuda.synchronize()

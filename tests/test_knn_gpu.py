@@ -1,19 +1,25 @@
 """GPU parity of knn_search / knn_distances (tcgen05 distance GEMM) vs the oracle.
 
-Tolerance (reading R19, derived from the arithmetic of the bf16x3
-split): |d_gpu - d_ora| <= 1e-4 * d_ora + 6*2^-16 * sum_i |q_i||r_i|
-+ (D+2)*2^-24 * (|q|^2 + |r|^2): each operand is hi + lo with a residue below
-2^-16 of its value (bf16 unit roundoff 2^-8, twice), the dropped lo*lo term is
-below 2^-16 of the product -- 3*2^-16 of each product of the MMA operands,
-which are -2q_i and r_i, hence 6*2^-16 |q_i r_i| -- and fp32 accumulation over
-D terms and the rounded norms add the last term.  On the paper's workload (uniform [0,1]^128) the
-north star's plain relative bound |d_gpu - d_ora| <= 1e-4 * d_ora is asserted
-as well.  Integer data in [0,255] (knn-S) is bit-exact.
+Two tolerances:
 
-Neighbour sets (reading R20): every GPU neighbour's oracle distance is within
-tolerance of the oracle's k-th distance, every oracle neighbour clearly inside
-(d < d_k - tol) is returned, the GPU list is sorted by its own (d, idx) and has
-distinct in-range indices.
+* the north star's contract (BASELINE.json): distances within a relative error
+  of 1e-4, |d_gpu - d_ora| <= 1e-4 * d_ora, on every returned neighbour, and
+  neighbour sets equal except where oracle distances differ from the oracle's
+  k-th distance d_k by less than that tolerance (every returned index has
+  d_ora <= d_k (1 + 1e-4); every oracle neighbour with d_ora < d_k (1 - 1e-4) is
+  returned) -- asserted on the paper's workload (uniform [0,1]^D)
+  and every non-cancelling shape (D >= 32, no self matches);
+* DESIGN.md reading R19 only for cancellation-prone shapes (small D, a query
+  equal to a reference): |d_gpu - d_ora| <= 1e-4 * d_ora + 6*2^-16 * sum_i |q_i||r_i|
+  + (D+2)*2^-24 * (|q|^2 + |r|^2) -- the bf16x3 split's residue (each operand is
+  hi + lo with a residue below 2^-16 of its value, the dropped lo*lo term below
+  2^-16 of the product; the MMA operands are -2q_i and r_i) and fp32 accumulation
+  over D terms plus the rounded norms.  Near d = 0 the GEMM expansion
+  |q|^2 + |r|^2 - 2 q.r cancels, so no relative bound can hold there.
+
+Integer data in [0,255] (knn-S) is bit-exact.  The oracle's distances
+(oracle.knn_dist: double accumulation, one rounding to fp32) are the reference
+for every returned index.
 """
 import numpy as np
 import pytest
@@ -42,14 +48,18 @@ def tol_pairs(q, r, d_ora):
     return 1e-4 * d_ora + 6 * 2.0 ** -16 * absdot + (D + 2) * 2.0 ** -24 * ((q * q).sum() + (r * r).sum(axis=1))
 
 
-def check_knn(oracle_mod, ref, qry, k, gv, gi, idx_offset=0, exact=False, oracle_out=None, rows=None):
+def check_knn(oracle_mod, ref, qry, k, gv, gi, idx_offset=0, exact=False, oracle_out=None, rows=None,
+              contract=None):
     """oracle_out: precomputed (ov, oi) (e.g. the k-NN graph oracle); rows: global row id of
-    each query for the k-NN graph (its own index must not appear)."""
+    each query for the k-NN graph (its own index must not appear); contract: assert the
+    north star's plain 1e-4 tolerance (default: D >= 32), else reading R19."""
     ref = ref.numpy() if torch.is_tensor(ref) else ref
     qry = qry.numpy() if torch.is_tensor(qry) else qry
     gv = gv.cpu().numpy() if torch.is_tensor(gv) else gv
     gi = gi.cpu().numpy() if torch.is_tensor(gi) else gi
     N, D = ref.shape
+    if contract is None:
+        contract = D >= 32
     ov, oi = oracle_out if oracle_out is not None else oracle_mod.knn(ref, qry, k, idx_offset=idx_offset)
     if exact:
         assert np.array_equal(gi, oi)
@@ -64,15 +74,24 @@ def check_knn(oracle_mod, ref, qry, k, gv, gi, idx_offset=0, exact=False, oracle
         # sorted by its own (d, idx)
         for t in range(k - 1):
             assert gv[q][t] < gv[q][t + 1] or (gv[q][t] == gv[q][t + 1] and gi[q][t] < gi[q][t + 1])
-        qq = qry[q].astype(np.float64)
-        d_true = ((ref[idx].astype(np.float64) - qq) ** 2).sum(axis=1)
-        tol = tol_pairs(qq, ref[idx].astype(np.float64), d_true)
-        assert np.all(np.abs(gv[q].astype(np.float64) - d_true) <= tol), q
+        # the oracle's distance of every returned neighbour
+        d_ora = oracle_mod.knn_dist(ref[idx], qry[q:q + 1])[0].astype(np.float64)
         dk = float(ov[q][-1])
-        tol_k = 1e-4 * dk + 6 * 2.0 ** -16 * np.sqrt(qn[q] * rn.max()) + (D + 2) * 2.0 ** -24 * (qn[q] + rn.max())
-        assert np.all(d_true <= dk + 2 * tol_k), q
-        must = oi[q][ov[q].astype(np.float64) < dk - 2 * tol_k].astype(np.int64) - idx_offset
-        assert set(must.tolist()) <= set(idx.tolist()), q
+        g = gv[q].astype(np.float64)
+        must = oi[q][ov[q].astype(np.float64) < dk * (1 - 1e-4)] if contract else None
+        if contract:
+            # the north star's contract: relative 1e-4, neighbour sets exact outside the
+            # 1e-4 band around the oracle's k-th distance
+            assert np.all(np.abs(g - d_ora) <= 1e-4 * d_ora), (q, float(np.max(np.abs(g - d_ora) / d_ora)))
+            assert np.all(d_ora <= dk * (1 + 1e-4)), q
+        else:
+            qq = qry[q].astype(np.float64)
+            tol = tol_pairs(qq, ref[idx].astype(np.float64), d_ora)
+            assert np.all(np.abs(g - d_ora) <= tol), q
+            tol_k = 1e-4 * dk + 6 * 2.0 ** -16 * np.sqrt(qn[q] * rn.max()) + (D + 2) * 2.0 ** -24 * (qn[q] + rn.max())
+            assert np.all(d_ora <= dk + 2 * tol_k), q
+            must = oi[q][ov[q].astype(np.float64) < dk - 2 * tol_k]
+        assert set((must.astype(np.int64) - idx_offset).tolist()) <= set(idx.tolist()), q
 
 
 @pytest.mark.parametrize("kind,N,Q,D", [("knn-S", 700, 200, 128), ("knn-U", 700, 200, 128),
@@ -119,7 +138,7 @@ def test_knn_search_idx_offset_and_self_match(K, oracle_mod):
     assert gi[:, 0].tolist() == [1000000, 1000017, 1001234, 1003999]
     # d(q, q) = |q|^2 + |q|^2 - 2 q.q cancels: 0 up to the R19 floor, not exactly
     assert np.all(gv[:, 0].cpu().numpy() <= 3 * 2.0 ** -16 * 2 * norms(qry.numpy()))
-    check_knn(oracle_mod, ref, qry, 10, gv, gi, idx_offset=1000000)
+    check_knn(oracle_mod, ref, qry, 10, gv, gi, idx_offset=1000000, contract=False)  # d = 0 cancels
 
 
 def test_knn_search_duplicates_tie_by_index(K, oracle_mod):
@@ -155,6 +174,21 @@ def test_config4_full_size_sampled_queries(K, oracle_mod, kind):
     check_knn(oracle_mod, ref.cpu(), qry[sample].cpu(), k, gv[sample], gi[sample], exact=(kind == "knn-S"))
 
 
+@pytest.mark.slow
+@pytest.mark.parametrize("kind", ["knn-U", "knn-S"])
+def test_config5_per_rank_shape_k1024(K, oracle_mod, kind):
+    # configs[4] per rank: N = 8M references sharded over 8 GPUs -> N = 10^6 per rank,
+    # Q = 10^4, k = 1024 ("k up to 1024"); 48 sampled queries vs the oracle
+    N, Q, D, k = 1000000, 10000, 128, 1024
+    ref = synth.knn_points(kind, 43, 0, N, D, device="cuda")
+    qry = synth.knn_points(kind, 44, 0, Q, D, device="cuda")
+    gv, gi = K.knn_search(ref, qry, k, idx_offset=3000000)
+    torch.cuda.synchronize()
+    sample = list(range(16)) + list(range(101, Q, Q // 32))[:32]
+    check_knn(oracle_mod, ref.cpu(), qry[sample].cpu(), k, gv[sample], gi[sample], idx_offset=3000000,
+              exact=(kind == "knn-S"))
+
+
 _SAMPLED_SCRIPT = r"""
 import sys, numpy as np, torch
 sys.path.insert(0, sys.argv[1])
@@ -186,7 +220,7 @@ def test_knn_search_sampled_start(oracle_mod, tmp_path, kind, k):
     check_knn(oracle_mod, ref, qry[sample], k, gv[sample], gi[sample], exact=(kind == "knn-S"))
 
 
-_EW8_SCRIPT = r"""
+_KNOB_SCRIPT = r"""
 import sys, numpy as np, torch
 sys.path.insert(0, sys.argv[1])
 import paper_conf_ipps_tang0emg15_b200 as K, synth
@@ -197,18 +231,24 @@ v, i = K.knn_search(ref, qry, k)
 np.save(sys.argv[2] + "/v.npy", v.cpu().numpy()); np.save(sys.argv[2] + "/i.npy", i.cpu().numpy())
 """
 
+# every experiment knob the kernels ever read, at a result-breaking setting: the product
+# library is built without -DKSEL_EXPERIMENTS, so none of them may change the result
+_BREAKING_KNOBS = {"KSEL_KNN_PASSES": "1", "KSEL_KNN_MODE": "2", "KSEL_KNN_EW": "8", "KSEL_KNN_QPC": "2",
+                   "KSEL_KNN_CLUSTER": "4", "KSEL_KNN_SOFTCAP": "40", "KSEL_KNN_SPLITS": "3",
+                   "KSEL_KNN_COLDW": "7", "KSEL_KNN_SAMPLE": "1", "KSEL_ORDER": "0", "KSEL_LOOSE": "1"}
 
-@pytest.mark.parametrize("kind,k", [("knn-U", 100), ("knn-S", 32), ("knn-U", 512)])
-def test_knn_search_eight_epilogue_warps(oracle_mod, tmp_path, kind, k):
-    # the 8-epilogue-warp variant (two warps per TMEM lane quadrant, 128 columns each,
-    # 2 S pool lists per query) in a fresh process (KSEL_KNN_EW is read once)
+
+@pytest.mark.parametrize("kind,k", [("knn-U", 100), ("knn-S", 32)])
+def test_knn_search_ignores_experiment_knobs(oracle_mod, tmp_path, kind, k):
+    """knobs that broke results (1-pass MMA, pipeline-only modes) exist only in
+    a -DKSEL_EXPERIMENTS build; with all of them set, knn_search still matches the oracle."""
     import os
     import subprocess
     import sys
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     N, Q = 40000, 2000
-    env = dict(os.environ, KSEL_KNN_EW="8")
-    subprocess.run([sys.executable, "-c", _EW8_SCRIPT, root, str(tmp_path), kind, str(N), str(Q), str(k)],
+    env = dict(os.environ, **_BREAKING_KNOBS)
+    subprocess.run([sys.executable, "-c", _KNOB_SCRIPT, root, str(tmp_path), kind, str(N), str(Q), str(k)],
                    check=True, env=env, timeout=300)
     gv, gi = np.load(tmp_path / "v.npy"), np.load(tmp_path / "i.npy")
     ref = synth.knn_points(kind, 61, 0, N, 128)

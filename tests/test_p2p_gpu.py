@@ -1,11 +1,14 @@
 """GPU tests of the collective-free row-sharded k-NN exchange.
 
-* ksel_merge_lists (pointer tables, optional ready flags) == ksel_merge, bit for bit;
-* the ready-flag wait really orders the merge after a producer on another stream;
-* KnnP2P with 2 processes on ONE GPU: the exchange buffers are mapped across
+* ksel_merge_lists (pointer tables, optional ready flags) == oracle.merge (the
+  divide-and-merge definition), bit for bit, and == ksel_merge;
+* the ready-flag wait really orders the merge after a producer on another stream
+  (the merged result is again checked against oracle.merge);
+* KnnP2P with 2 and 3 processes on ONE GPU: the exchange buffers are mapped across
   processes with CUDA IPC (the same mechanism as NVLink peer mappings on a
-  multi-GPU box), several epochs (double buffering, consumed flags), results
-  bit-identical to the unsharded knn_search.
+  multi-GPU box), several epochs (double buffering, consumed flags); every rank's
+  slice is checked against oracle.knn (bit-exact on integer data, the north star's
+  1e-4 contract on uniform data) and is bit-identical to the unsharded knn_search.
 """
 import os
 import socket
@@ -41,10 +44,14 @@ def _lists(K, S, Q, kin, seed):
 
 
 @pytest.mark.parametrize("S,kin,k", [(2, 32, 32), (3, 100, 64), (8, 256, 256), (5, 1024, 1000)])
-def test_merge_lists_equals_merge(K, S, kin, k):
+def test_merge_lists_equals_merge(K, oracle_mod, S, kin, k):
     Q = 300
     vs, is_ = _lists(K, S, Q, kin, 7 + S)
     ev, ei = K.ksel_merge(torch.stack(vs), torch.stack(is_), k)
+    # the oracle's merge of the same lists (concatenate, stable sort by (value, index), truncate)
+    xv, xi = oracle_mod.merge(torch.stack(vs).cpu().numpy(), torch.stack(is_).cpu().numpy(), k)
+    assert np.array_equal(ei.cpu().numpy(), xi)
+    assert np.array_equal(ev.cpu().numpy().view(np.uint32), xv.view(np.uint32))
     ov = torch.empty((Q, k), dtype=torch.float32, device="cuda")
     oi = torch.empty((Q, k), dtype=torch.int32, device="cuda")
     K.ksel_merge_lists([v.data_ptr() for v in vs], [i.data_ptr() for i in is_], Q, kin, k, ov, oi)
@@ -63,13 +70,14 @@ def test_merge_lists_equals_merge(K, S, kin, k):
     assert torch.equal(oi2, ei[q0:q1]) and torch.equal(ov2.view(torch.int32), ev[q0:q1].view(torch.int32))
 
 
-def test_merge_lists_waits_for_ready_flags(K):
+def test_merge_lists_waits_for_ready_flags(K, oracle_mod):
     # the producer fills list 1 on another stream after a long busy kernel and only then
     # signals; the merge (launched first) must wait for the flag and see the new data
     S, Q, kin, k = 2, 256, 64, 64
     vs, is_ = _lists(K, S, Q, kin, 3)
-    ev, ei = K.ksel_merge(torch.stack(vs), torch.stack(is_), k)
     torch.cuda.synchronize()
+    xv, xi = oracle_mod.merge(torch.stack(vs).cpu().numpy(), torch.stack(is_).cpu().numpy(), k)
+    ev, ei = torch.from_numpy(xv).cuda(), torch.from_numpy(xi).cuda()
     target_v, target_i = vs[1].clone(), is_[1].clone()
     vs[1].fill_(float("inf"))
     is_[1].fill_(-1)
@@ -141,13 +149,15 @@ for ep in range(4):
     torch.cuda.synchronize()
     np.save(out + "/v_%d_%d.npy" % (ep, rank), mv.cpu().numpy())
     np.save(out + "/i_%d_%d.npy" % (ep, rank), mi.cpu().numpy())
+p2p.check()
 p2p.close()
 tdist.destroy_process_group()
 """
 
 
 @pytest.mark.parametrize("world", [2, 3])
-def test_knn_p2p_processes_on_one_gpu(K, tmp_path, world):
+def test_knn_p2p_processes_on_one_gpu(K, oracle_mod, tmp_path, world):
+    from test_knn_gpu import check_knn
     s = socket.socket()
     s.bind(("127.0.0.1", 0))
     port = str(s.getsockname()[1])
@@ -170,9 +180,38 @@ def test_knn_p2p_processes_on_one_gpu(K, tmp_path, world):
         qry = synth.knn_points(kind, 80 + ep, 0, Q, D, device="cuda")
         ev, ei = K.knn_search(ref, qry, k)
         ev, ei = ev.cpu().numpy(), ei.cpu().numpy()
+        gv = np.concatenate([np.load(tmp_path / ("v_%d_%d.npy" % (ep, r))) for r in range(world)])
+        gi = np.concatenate([np.load(tmp_path / ("i_%d_%d.npy" % (ep, r))) for r in range(world)])
+        # against the oracle (all Q queries of all ranks' slices, in rank order)
+        check_knn(oracle_mod, ref.cpu(), qry.cpu(), k, gv, gi, exact=(kind == "knn-S"))
         for r in range(world):
             q0, q1 = dist.shard_range(Q, world, r)
-            gv = np.load(tmp_path / ("v_%d_%d.npy" % (ep, r)))
-            gi = np.load(tmp_path / ("i_%d_%d.npy" % (ep, r)))
-            assert np.array_equal(gi, ei[q0:q1]), (ep, r)
-            assert np.array_equal(gv.view(np.uint32), ev[q0:q1].view(np.uint32)), (ep, r)
+            assert np.array_equal(gi[q0:q1], ei[q0:q1]), (ep, r)
+            assert np.array_equal(gv[q0:q1].view(np.uint32), ev[q0:q1].view(np.uint32)), (ep, r)
+
+
+def test_flag_wait_timeout_reports_without_killing_the_context(K):
+    # a wait whose flag never arrives gives up after the timeout, records
+    # KSEL_ERR_TIMEOUT in the library's status word and leaves the context usable
+    flag = torch.zeros(1, dtype=torch.int32, device="cuda")
+    K.device_status_clear()
+    K.set_flag_timeout(0.05)
+    try:
+        K.flag_wait([flag.data_ptr()], 7)  # nobody ever signals 7
+        vs = [torch.full((4, 8), 1.0, device="cuda"), torch.full((4, 8), 2.0, device="cuda")]
+        ids = [torch.arange(32, dtype=torch.int32, device="cuda").view(4, 8),
+               torch.arange(32, 64, dtype=torch.int32, device="cuda").view(4, 8)]
+        ov = torch.empty((4, 8), dtype=torch.float32, device="cuda")
+        oi = torch.empty((4, 8), dtype=torch.int32, device="cuda")
+        K.ksel_merge_lists([v.data_ptr() for v in vs], [i.data_ptr() for i in ids], 4, 8, 8, ov, oi,
+                           ready_ptrs=[flag.data_ptr(), flag.data_ptr()], epoch=9)
+        torch.cuda.synchronize()
+        assert K.device_status() == 5
+    finally:
+        K.set_flag_timeout(600.0)
+        K.device_status_clear()
+    assert K.device_status() == 0
+    x = torch.rand(8, 1000, device="cuda")  # the context still works
+    v, i = K.ksel_select(x, 5)
+    torch.cuda.synchronize()
+    assert torch.equal(i.long(), torch.sort(x, dim=1, stable=True).indices[:, :5])
