@@ -5,12 +5,20 @@
     torchrun --nproc-per-node N bench.py --gpus N ...
 
 Workload (BASELINE.json configs[2], the 1/2/4/8-GPU config): ksel_select over
-Q = 16384 rows per GPU of N = 2^20 uniform fp32 distances, k = 256,
-query-sharded (rank r owns global rows [r*Q, (r+1)*Q); no communication;
-weak scaling).  A step is one ksel_select call over the rank's rows, inputs
-resident in HBM (64 GiB per GPU, far larger than the 126 MB L2, so no flush is
-needed between steps).  Metric: selected rows/s (whole job) and achieved HBM
-GB/s vs the measured peak.
+Q = 16384 rows in total of N = 2^20 uniform fp32 distances, k = 256,
+query-sharded (rank r owns global rows [r*Q/g, (r+1)*Q/g); no communication;
+strong scaling by default -- the total work is fixed, as configs[2] states;
+--scaling weak keeps 16384 rows per rank).  A step is one ksel_select call
+over the rank's rows, inputs resident in HBM (64 GiB at g = 1, far larger than
+the 126 MB L2, so no flush is needed between steps).  Metric: selected rows/s
+(whole job) and achieved HBM GB/s vs the measured peak.
+
+At N = 1 the same JSON line also carries a `sweep`: the north star's k sweep
+(BASELINE configs[1]: Q = 1024, N = 65536, k in {1, 8, 32, 128, 256, 1024} on
+uniform / Gaussian / sorted ascending / sorted descending / tied rows), the
+fused kNN of configs[3] (C4) and the per-rank shape of configs[4] (C5: N = 10^6
+references, Q = 10^4, k = 1024), each as device time, throughput and roofline
+fraction.
 
 Rank 0 prints ONE JSON line.  --impl reference times the CPU oracle (oracle/)
 on this host's cores on a bounded sample of the same workload.
@@ -47,7 +55,8 @@ def parse():
     ap.add_argument("--config", choices=["c1", "c2", "c3", "c4", "c5"], default="c3")
     ap.add_argument("--k", type=int, default=None)
     ap.add_argument("--dist", default=None)
-    ap.add_argument("--scaling", choices=["weak", "strong"], default="weak")
+    ap.add_argument("--scaling", choices=["weak", "strong"], default="strong")
+    ap.add_argument("--no-sweep", action="store_true", help="skip the k x distribution / kNN sweep (N = 1)")
     ap.add_argument("--e2e-rows", type=int, default=0,
                     help="rows per end-to-end step per rank (host buffers); 0 = 2048 on one GPU, "
                          "512 per rank on several (pinned host memory: 4 MB per row)")
@@ -138,6 +147,30 @@ def cpu_count():
         return os.cpu_count() or 1
 
 
+def cpu_info():
+    """Host CPU model and socket count (lscpu), for the cpu_baseline record."""
+    model, sockets = None, None
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for ln in out.splitlines():
+            key, _, val = ln.partition(":")
+            if key.strip() == "Model name":
+                model = val.strip()
+            elif key.strip() == "Socket(s)":
+                sockets = int(val.strip())
+    except Exception:
+        pass
+    if model is None:
+        try:
+            with open("/proc/cpuinfo") as f:
+                for ln in f:
+                    if ln.startswith("model name"):
+                        model = ln.partition(":")[2].strip()
+                        break
+        except Exception:
+            pass
+    return {"cpu_model": model, "sockets": sockets}
+
 def oracle_rows_per_s(dist: str, seed: int, N: int, k: int, rows: list, threads: int, device="cpu"):
     """Time the oracle (as it stands) on a bounded sample of rows; returns rows/s.
 
@@ -201,7 +234,7 @@ def run_reference_knn(args, rank, world):
         "dtype": "f64", "data": "synthetic",
         "config": knn_config(N, nref, Q, D, k, kind, mode, world),
         "cpu_baseline": {"value": value, "unit": "queries/s", "cores": threads, "kind": "oracle",
-                         "sample": "%d queries vs %d references per step" % (nq, nref)},
+                         "sample": "%d queries vs %d references per step" % (nq, nref), **cpu_info()},
         "e2e": {"value": value, "unit": "queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -220,8 +253,9 @@ def run_reference(args, rank, world):
     seed = synth.seed_for(3, dist)
     rows_per_step = max(4, 2 * threads)
     times = []
+    q_all = Qr if args.scaling == "strong" else Qr * max(1, world)
     for s in range(args.warmup + args.steps):
-        rows = [(s * rows_per_step + t) % (Qr * max(1, world)) for t in range(rows_per_step)]
+        rows = [(s * rows_per_step + t) % q_all for t in range(rows_per_step)]
         _, dt = oracle_rows_per_s(dist, seed, N, k, rows, threads)
         if s >= args.warmup:
             times.append(dt)
@@ -232,10 +266,10 @@ def run_reference(args, rank, world):
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * total / args.steps,
         "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None, "dtype": "f32",
         "data": "synthetic",
-        "config": select_config(Qr, N, k, dist, world),
+        "config": select_config(Qr // world if args.scaling == "strong" else Qr, N, k, dist, world),
         "cpu_baseline": {"value": value, "unit": "rows/s", "cores": threads, "kind": "oracle",
                          "sample": "%d rows of N=%d per step (stable sort by (value,index), truncate to k)"
-                                   % (rows_per_step, N)},
+                                   % (rows_per_step, N), **cpu_info()},
         "e2e": {"value": value, "unit": "rows/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -294,9 +328,11 @@ def bench_select(args, rank, world, local_rank, dev, K, tdist):
     Qr, N, k, dist = CONFIGS[args.config]
     k = args.k or k
     dist = args.dist or dist
-    if args.scaling == "strong":
-        Qr = Qr // world
-    row0 = rank * Qr
+    if args.scaling == "strong":  # configs[2]: Q rows in total, Q/g per rank
+        row0, row1 = rank * Qr // world, (rank + 1) * Qr // world
+        Qr = row1 - row0
+    else:
+        row0 = rank * Qr
     seed = synth.seed_for(3, dist)
     # ---- inputs resident in HBM (generation is not timed) ----------------------
     x = synth.rows(dist, seed, row0, Qr, N, device=dev)
@@ -381,8 +417,92 @@ def bench_select(args, rank, world, local_rank, dev, K, tdist):
         sample = sorted({(b * 2048 + t) % Qr for b in range(max(1, Qr // 2048)) for t in range(per_blk)})[:nrows]
         rps, dt = oracle_rows_per_s(dist, seed, N, k, [row0 + r for r in sample], threads, device=dev)
         line["cpu_baseline"] = {"value": rps, "unit": "rows/s", "cores": threads, "kind": "oracle",
-                                "sample": "%d rows of the same workload (%.1f s)" % (len(sample), dt)}
+                                "sample": "%d rows of the same workload (%.1f s)" % (len(sample), dt),
+                                **cpu_info()}
     return line
+
+
+SWEEP_C2 = (1024, 65536, (1, 8, 32, 128, 256, 1024), ("U", "G", "DG", "SA", "SD", "T"))
+
+
+def _kernel_ms(K, fn, reps):
+    """Average device time of the dominant kernel of `fn` (the library's live CUDA
+    events around each launch) and of the whole call (events around `reps`
+    back-to-back calls on the current stream), after 3 warm-up calls."""
+    import torch
+    for _ in range(3):
+        fn()
+    torch.cuda.synchronize()
+    K.timing_collect()
+    K.timing_enable(True)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(reps):
+        fn()
+    e1.record()
+    torch.cuda.synchronize()
+    K.timing_enable(False)
+    kms, kn = K.timing_collect()
+    return kms / max(1, kn), e0.elapsed_time(e1) / reps
+
+
+def run_sweep(dev, K, peak_hbm, peak_bf16):
+    """The north star's k x distribution sweep (configs[1]) plus the kNN configs
+    (configs[3] and configs[4]'s per-rank shape), one GPU, each entry's device
+    time and roofline fraction.  Inputs (268 MB for C2, 512 MB of references for
+    C4/C5) exceed the 126 MB L2 and are streamed anew by every call."""
+    import torch
+
+    import synth
+    out = []
+    Q, N, ks, dists = SWEEP_C2
+    x = torch.empty((Q, N), dtype=torch.float32, device=dev)
+    ov = torch.empty((Q, 1024), dtype=torch.float32, device=dev)
+    oi = torch.empty((Q, 1024), dtype=torch.int32, device=dev)
+    read_ms = None
+    for dist in dists:
+        synth.rows(dist, synth.seed_for(2, dist), 0, Q, N, out=x)
+        torch.cuda.synchronize()
+        if read_ms is None:  # same-run read ceiling: torch row reductions over the same matrix (best)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            best = None
+            for red in (lambda: torch.amin(x, dim=1), lambda: torch.amin(x), lambda: torch.sum(x, dim=1)):
+                for _ in range(6):
+                    e0.record()
+                    red()
+                    e1.record()
+                    torch.cuda.synchronize()
+                    t = e0.elapsed_time(e1)
+                    best = t if best is None else min(best, t)
+            read_ms = best
+        for k in ks:
+            v, i = ov[:, :k].contiguous(), oi[:, :k].contiguous()
+            kms, cms = _kernel_ms(K, lambda: K.ksel_select(x, k, v, i), 20)
+            gbs = Q * (4.0 * N + 8.0 * k) / (kms / 1e3) / 1e9
+            out.append({"config": "c2", "op": "ksel_select", "Q": Q, "N": N, "k": k, "dist": dist,
+                        "kernel": "ksel_pool_kernel", "ms": kms, "call_ms": cms, "rows_per_s": Q / (cms / 1e3),
+                        "gbs": gbs, "frac_hbm": gbs / peak_hbm, "frac_read_ceiling": read_ms / kms})
+    out.append({"config": "c2", "op": "read ceiling: best of torch.amin(x, dim=1), torch.amin(x), torch.sum(x, dim=1)",
+                "Q": Q, "N": N, "ms": read_ms,
+                "gbs": Q * N * 4.0 / (read_ms / 1e3) / 1e9})
+    del x, ov, oi
+    torch.cuda.empty_cache()
+    for name, (Nr, Qk, D, k) in (("c4", (1000000, 10000, 128, 100)), ("c5-per-rank", (1000000, 10000, 128, 1024))):
+        ref = synth.knn_points("knn-U", 41, 0, Nr, D, device=dev)
+        qry = synth.knn_points("knn-U", 42, 0, Qk, D, device=dev)
+        ws = torch.empty(K.knn_search_workspace(Nr, Qk, D, k), dtype=torch.uint8, device=dev)
+        dv = torch.empty((Qk, k), dtype=torch.float32, device=dev)
+        di = torch.empty((Qk, k), dtype=torch.int32, device=dev)
+        kms, cms = _kernel_ms(K, lambda: K.knn_search(ref, qry, k, out_dist=dv, out_idx=di, workspace=ws), 5)
+        tf = 2.0 * Qk * Nr * D / (kms / 1e3) / 1e12
+        tf_call = 2.0 * Qk * Nr * D / (cms / 1e3) / 1e12
+        out.append({"config": name, "op": "knn_search", "N": Nr, "Q": Qk, "D": D, "k": k, "points": "knn-U",
+                    "kernel": "knn_fused_kernel", "ms": kms, "call_ms": cms, "queries_per_s": Qk / (cms / 1e3),
+                    "tflops": tf, "frac_tensor": tf / peak_bf16, "frac_tensor_call": tf_call / peak_bf16,
+                    "flops_formula": "2*Q*N*D (algorithmic, one pass)"})
+        del ref, qry, ws, dv, di
+        torch.cuda.empty_cache()
+    return out
 
 
 KNN_CONFIGS = {
@@ -520,7 +640,7 @@ def bench_knn(args, rank, world, local_rank, dev, K, tdist):
         oracle.knn(hr, hq, k, nthreads=threads)
         dt = time.perf_counter() - t0
         line["cpu_baseline"] = {"value": nq / dt, "unit": "queries/s", "cores": threads, "kind": "oracle",
-                                "sample": "%d queries vs all %d references (%.1f s)" % (nq, Nl, dt)}
+                                "sample": "%d queries vs all %d references (%.1f s)" % (nq, Nl, dt), **cpu_info()}
     return line
 
 
@@ -548,6 +668,16 @@ def main():
         line = bench_knn(args, rank, world, local_rank, dev, K, tdist)
     else:
         line = bench_select(args, rank, world, local_rank, dev, K, tdist)
+        if rank == 0 and world == 1 and not args.no_sweep and args.config == "c3":
+            import torch
+            torch.cuda.empty_cache()
+            peak_bf16 = 1646.1
+            try:
+                with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+                    peak_bf16 = float(json.load(f)["bf16_tflops"])
+            except Exception:
+                pass
+            line["sweep"] = run_sweep(dev, K, line["roofline"]["peak"], peak_bf16)
     if rank == 0:
         print(json.dumps(line), flush=True)
     if world > 1:

@@ -27,6 +27,9 @@ import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libksel.so")
+# tools/ timing experiments only: load the -DKSEL_EXPERIMENTS build (libksel_exp.so)
+if os.environ.get("KSEL_EXPERIMENTS_LIB") == "1":
+    LIB_PATH = os.path.join(_HERE, "libksel_exp.so")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(

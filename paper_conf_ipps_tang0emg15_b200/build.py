@@ -33,6 +33,7 @@ NVCC_FLAGS = [
 # (the default) contains none of them and reads no result-affecting knob.
 if os.environ.get("KSEL_BUILD_EXPERIMENTS") == "1":
     NVCC_FLAGS.append("-DKSEL_EXPERIMENTS")
+    LIB = os.path.join(HERE, "libksel_exp.so")  # never the product library
 
 
 def _sources():

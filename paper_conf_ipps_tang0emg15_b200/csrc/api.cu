@@ -78,6 +78,11 @@ int chunk_order_mode() {
         int m = (e && (e[0] == '0' || e[0] == '1' || e[0] == '2')) ? e[0] - '0' : 2;
         const char* l = std::getenv("KSEL_LOOSE");
         if (l && l[0] == '1') m |= 4;
+#ifdef KSEL_EXPERIMENTS
+        // phase-cost experiments of the pool kernel (results are wrong): bit 3 = no exact
+        // admission path, bit 4 = no final select/sort/merge, bit 5 = no starting bound
+        m |= (env_int("KSEL_POOL_SKIP", 0) & 7) << 3;
+#endif
         return m;
     }();
     return mode;

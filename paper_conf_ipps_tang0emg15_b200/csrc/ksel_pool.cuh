@@ -262,7 +262,10 @@ __device__ __noinline__ unsigned long long pool_narrow_regs(uint32_t* __restrict
             if (__reduce_add_sync(kFull, c) < need) vidx = cand;
         }
     }
-    // compaction in place: keep (key, idx) <= (vkey, vidx)
+    // compaction in place: keep (key, idx) <= (vkey, vidx); every lane's loads above
+    // precede any lane's stores below (the reductions already order them; the explicit
+    // warp barrier makes that visible to racecheck)
+    __syncwarp();
     const uint32_t lt = lanemask_lt();
     int w = 0;
 #pragma unroll
@@ -343,6 +346,7 @@ __device__ __noinline__ unsigned long long pool_narrow64(unsigned long long* __r
         }
     }
     const unsigned long long T = ((unsigned long long)vkey << 32) | vidx;
+    __syncwarp();  // all loads of the pool precede the in-place compaction
     const uint32_t lt = lanemask_lt();
     int w = 0;
 #pragma unroll

@@ -323,7 +323,7 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads)
     // (key, largest index) bounds the k-th pair -- the stream then admits a few
     // times k candidates instead of everything until the pool first fills.
     constexpr int NB = Cfg::NB;
-    if (nmine >= NB && k <= NB * CH / 2) {
+    if (nmine >= NB && k <= NB * CH / 2 && !(order_mode & 32)) {
         uint32_t keys[NB * CH / 128 * 4];
         uint32_t nreal = 0;
 #pragma unroll
@@ -428,13 +428,17 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads)
                 for (int u = 1; u < G; ++u) mn = fminf(mn, gm[u]);
                 go = __any_sync(kFull, col0 >= Ti ? mn < tv : mn <= tv);
             }
-            if (go) exact(srcf, (uint32_t)g, len, col0, x);
+            if (go && !(order_mode & 8)) exact(srcf, (uint32_t)g, len, col0, x);
         }
         __syncwarp();
         if (lane == 0 && li + S < nmine) issue(li + S);
     }
 
     // ---- finish: exact top-k of this warp's share, sorted -----------------------------------
+    if (order_mode & 16) {  // (phase-cost experiment: no final phase)
+        if (lane == 0 && n == 0x7fffffff) out_val[row] = 0.f;
+        return;
+    }
     if (n > k) {
         const unsigned long long t = pool_kth(pk, pi, n, (uint32_t)k, hist);
         n = pool_compact(pk, pi, n, (uint32_t)(t >> 32), (uint32_t)t);
