@@ -27,9 +27,12 @@ import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libksel.so")
-# tools/ timing experiments only: load the -DKSEL_EXPERIMENTS build (libksel_exp.so)
+# tools/ timing experiments only: load the -DKSEL_EXPERIMENTS build (libksel_exp.so), or
+# an A/B build of another revision (KSEL_AB_LIB=<file name next to this one>)
 if os.environ.get("KSEL_EXPERIMENTS_LIB") == "1":
     LIB_PATH = os.path.join(_HERE, "libksel_exp.so")
+elif os.environ.get("KSEL_AB_LIB"):
+    LIB_PATH = os.path.join(_HERE, os.path.basename(os.environ["KSEL_AB_LIB"]))
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(

@@ -81,7 +81,7 @@ int chunk_order_mode() {
 #ifdef KSEL_EXPERIMENTS
         // phase-cost experiments of the pool kernel (results are wrong): bit 3 = no exact
         // admission path, bit 4 = no final select/sort/merge, bit 5 = no starting bound
-        m |= (env_int("KSEL_POOL_SKIP", 0) & 7) << 3;
+        m |= env_int("KSEL_POOL_SKIP", 0) & (8 | 16 | 32);
 #endif
         return m;
     }();
@@ -195,6 +195,7 @@ int ksel_select_config(const float* dist, int64_t Q, int64_t N, int k, float* ou
     cudaError_t e;
     if (algo == KSEL_ALGO_RADIX) {
         e = launch_select_radix(dist, Q, N, k, out_val, out_idx, (cudaStream_t)stream);
+
     } else if (algo == KSEL_ALGO_QUEUE) {
         const int wpr = warps_per_row ? warps_per_row : stream_warps_per_row(Q, N, di.sms);
         e = launch_select_stream(dist, Q, N, k, out_val, out_idx, wpr, (cudaStream_t)stream);

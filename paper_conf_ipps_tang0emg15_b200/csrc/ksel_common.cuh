@@ -180,6 +180,20 @@ __device__ __forceinline__ void warr_merge(WArr<R>& q, const WArr<RB>& b, uint32
     warr_clean<R>(q, lane);
 }
 
+// x[j] for a runtime j in [0, 16): a 4-level select tree (registers cannot be indexed
+// dynamically without a local-memory copy).
+__device__ __forceinline__ float sel16(const float (&x)[16], int j) {
+    const bool b0 = j & 1, b1 = j & 2, b2 = j & 4, b3 = j & 8;
+    float l1[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) l1[i] = b0 ? x[2 * i + 1] : x[2 * i];
+    float l2[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) l2[i] = b1 ? l1[2 * i + 1] : l1[2 * i];
+    const float l3a = b2 ? l2[1] : l2[0], l3b = b2 ? l2[3] : l2[2];
+    return b3 ? l3b : l3a;
+}
+
 // Pair at (0-based) position pos of a warp array, broadcast to all lanes.
 template <int R>
 __device__ __forceinline__ void warr_get(const WArr<R>& a, int pos, uint32_t& k, uint32_t& i) {

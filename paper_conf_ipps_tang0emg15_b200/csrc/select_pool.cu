@@ -45,7 +45,7 @@ struct PoolCfg {
                                      ? kQueue + 512
                                      : ((2 * kQueue > kQueue + 512) ? 2 * kQueue : kQueue + 512);
     static constexpr int CH = 512;         // floats per staged chunk (2 KB bulk copy)
-    static constexpr int NB = (2048 / CH < SD) ? 2048 / CH : SD;  // chunks feeding the starting bound
+    static constexpr int NB = (3 < SD) ? 3 : SD;  // chunks feeding the starting bound (1536 values)
     static constexpr int S = SD;           // ring stages per warp (3, or 6 when few warps run per SM)
     static constexpr int G = 4;            // float4 per lane per sub-step (512 elements per warp)
     static constexpr int NS = 4 * G;       // element slots per lane per sub-step
@@ -109,7 +109,7 @@ __device__ __noinline__ void pool_merge_sorted(uint32_t* __restrict__ qk, uint32
 }
 
 template <int R, int WPR, int RPC, int SD>
-__global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads)
+__global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 && WPR * RPC <= 16) ? 16 / (WPR * RPC) : 1)
     ksel_pool_kernel(const float* __restrict__ dist, int64_t Q, int64_t N, int k, float* __restrict__ out_val,
                      int32_t* __restrict__ out_idx, int order_mode, SegMap seg) {
     using Cfg = PoolCfg<R, WPR, RPC, SD>;
@@ -196,18 +196,15 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads)
         }
         return it_tail++;
     };
-    auto chunk_len = [&](uint64_t c) -> uint32_t {
-        const uint64_t s0 = a0 + c * CH;
-        const uint64_t s1 = (s0 + CH < a1) ? s0 + CH : a1;
-        return (uint32_t)(s1 - s0);
-    };
+    const uint32_t body_len = (uint32_t)(a1 - a0);  // < 2^31
+    auto chunk_len = [&](uint32_t c) -> uint32_t { return min((uint32_t)CH, body_len - c * (uint32_t)CH); };
     auto issue = [&](int li) {
-        const uint64_t c = c_begin + next_chunk();
+        const uint32_t c = (uint32_t)c_begin + next_chunk();
         const int st = li % S;
-        cid[st] = (uint32_t)c;
+        cid[st] = c;
         const uint32_t bytes = chunk_len(c) * 4u;
         mbar_arrive_expect_tx(&mbar[st], bytes);
-        bulk_g2s(ring + st * CH, dist + a0 + c * CH, bytes, &mbar[st]);
+        bulk_g2s(ring + st * CH, dist + a0 + (uint64_t)c * CH, bytes, &mbar[st]);
     };
 
     if (lane == 0) {
@@ -382,10 +379,12 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads)
             const unsigned long long sh = *reinterpret_cast<volatile unsigned long long*>(grp_thr);
             tighten((uint32_t)(sh >> 32), (uint32_t)sh);
         }
-        mbar_wait(&mbar[st], (uint32_t)(li / S) & 1u);
-        const uint64_t c = cid[st];
+        // (a suspended wait: a warp whose data has not landed leaves its issue slots to
+        // the other warps of the SM sub-partition instead of polling)
+        mbar_wait_sleep(&mbar[st], (uint32_t)(li / S) & 1u);
+        const uint32_t c = cid[st];
         const uint32_t len = chunk_len(c);
-        const uint32_t col0 = (uint32_t)(a0 + c * CH - g0);
+        const uint32_t col0 = (uint32_t)(a0 - g0) + c * (uint32_t)CH;
         const float* srcf = ring + st * CH;
         const float4* src = reinterpret_cast<const float4*>(srcf);
 #pragma unroll 1
@@ -428,10 +427,17 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads)
                 for (int u = 1; u < G; ++u) mn = fminf(mn, gm[u]);
                 go = __any_sync(kFull, col0 >= Ti ? mn < tv : mn <= tv);
             }
+            // The stage is refilled as soon as nothing reads it any more: right after the
+            // vote when no lane has a candidate (the common case once the bound is tight:
+            // every stage of the ring then stays in flight while the chunk is filtered),
+            // else after the exact path, which re-reads admitted values from the stage.
+            const bool last = g + G >= CH / 128;
             if (go && !(order_mode & 8)) exact(srcf, (uint32_t)g, len, col0, x);
+            if (last) {
+                __syncwarp();
+                if (lane == 0 && li + S < nmine) issue(li + S);
+            }
         }
-        __syncwarp();
-        if (lane == 0 && li + S < nmine) issue(li + S);
     }
 
     // ---- finish: exact top-k of this warp's share, sorted -----------------------------------

@@ -145,14 +145,16 @@ def test_special_rows(K, oracle_mod):
 
 
 @pytest.mark.parametrize("k", [1, 8, 32, 128, 256, 1024])
-@pytest.mark.parametrize("dist", ["U", "G", "SA", "SD", "T"])
+@pytest.mark.parametrize("dist", ["U", "G", "DG", "SA", "SD", "T"])
 def test_config2_full_size(K, oracle_mod, dist, k):
-    # configs[1]: Q=1024, N=65536, the k sweep, all distributions -- all rows
+    # configs[1]: Q=1024, N=65536, the k sweep, all distributions -- all rows, with the
+    # launch bench.py times (auto) and the streaming kernel variants forced
     x = synth.rows(dist, synth.seed_for(2, dist), 0, 1024, 65536, device="cuda")
-    gv, gi = K.ksel_select(x, k)
-    torch.cuda.synchronize()
     ev, ei = oracle_mod.select(x.cpu().numpy(), k)
-    assert_same(ev, ei, gv, gi, "C2 %s k=%d" % (dist, k))
+    for algo in (0, 1, 2):
+        gv, gi = K.ksel_select(x, k, algo=algo)
+        torch.cuda.synchronize()
+        assert_same(ev, ei, gv, gi, "C2 %s k=%d algo=%d" % (dist, k, algo))
 
 
 @pytest.mark.slow

@@ -1,0 +1,7 @@
+cd $GRAFT_REPO_ROOT; mkdir -p gpurun_out
+timeout 900 python -m pytest tests/test_ksel_gpu.py -x -q -m gpu -k "k_sweep_all or special or unaligned or config2_full or fuzz_shapes or forced" > gpurun_out/pytest_g.log 2>&1; echo "pytest=$?"
+for a in 0 4; do for d in U T SD; do for k in 1 32 256 1024; do
+  printf "C2 %-2s k=%-4d algo=%d " $d $k $a; timeout 60 python tools/run_select.py --Q 1024 --N 65536 --k $k --dist $d --reps 3 --inner 20 --algo $a | tail -1
+done; done; done > gpurun_out/c2_g.txt 2>&1
+timeout 300 python tools/run_select.py --Q 16384 --N 1048576 --k 256 --dist U --reps 3 > gpurun_out/c3_g.txt 2>&1
+timeout 300 python tools/run_select.py --Q 16384 --N 1048576 --k 256 --dist U --reps 3 --algo 4 >> gpurun_out/c3_g.txt 2>&1
