@@ -141,13 +141,20 @@ KSEL_API int ksel_merge(const float* cand_val, const int32_t* cand_idx, int64_t 
  *   ref   [N][D] fp32, query [Q][D] fp32, device, 4-byte aligned, row-major.
  *   1 <= D <= 256 (D > 256 -> KSEL_ERR_UNSUPPORTED); 1 <= k <= min(N, KSEL_MAX_K);
  *   N + idx_offset <= 2^31 - 1, idx_offset >= 0.
- *   out_dist [Q][k] fp32: squared L2 distance (no sqrt), clamped at >= 0,
- *            computed as |q|^2 + |r|^2 - 2 q.r with fp32 accumulation (error
- *            bound: DESIGN.md "knn tolerance");
+ *   out_dist [Q][k] fp32: squared L2 distance (no sqrt, reading R9) computed
+ *            EXACTLY as the oracle does: (float) sum_t (q_t - r_t)^2 with the
+ *            differences, squares and the index-ordered sum in double;
  *   out_idx  [Q][k] int32: idx_offset + reference row, ascending by
- *            (distance, index).
+ *            (distance, index) -- bit-identical to the CPU oracle.
  *   d_work   device workspace of >= knn_search_workspace(N, Q, D, k) bytes
- *            (norms and split operand copies); NULL allowed when that is 0.
+ *            (fp16 operand images, per-query candidate pools; queries are
+ *            processed in chunks so that the pools stay below 2 GiB).
+ * Method: a one-pass fp16 tcgen05 GEMM (|q|^2 + |r|^2 - 2 q.r, TMEM accumulator)
+ * FILTERS the references with a rigorous error bound eps_q (R21),
+ * keeping every reference whose filter distance is within 2 eps_q of a k-th
+ * value; the survivors are rescored exactly and selected.  Queries whose band of
+ * near-equal filter distances overflows a pool (or with non-finite inputs) are
+ * solved by an exact brute-force fallback on the device.
  * The Q x N distance matrix is never written to memory. */
 KSEL_API size_t knn_search_workspace(int64_t N, int64_t Q, int D, int k);
 KSEL_API int knn_search(const float* ref, const float* query, int64_t N, int64_t Q, int D, int k,
@@ -171,14 +178,16 @@ KSEL_API size_t knn_graph_workspace(int64_t N, int D, int k);
 KSEL_API int knn_graph(const float* points, int64_t N, int D, int k, float* out_dist, int32_t* out_idx,
                        void* d_work, size_t work_bytes, void* stream);
 
-/* knn_distances -- DIAGNOSTIC (not the hot path): the same tcgen05 distance
- * computation as knn_search, but every d(q, r) is written to out[Q][N] (device,
- * fp32) instead of being selected.  Lets tests pin the tensor-core distance
- * against the oracle's definition independently of selection.
+/* knn_distances -- DIAGNOSTIC (not the hot path): the filter distances d~(q, r) of
+ * knn_search's tensor-core pass (fp16 operands, fp32 accumulation, clamped at 0)
+ * written to out[Q][N] (device, fp32) instead of being filtered, and, if out_eps
+ * (device, [Q]) is not NULL, the bound eps_q with |d~(q, r) - d(q, r)| <= eps_q
+ * for every r that knn_search relies on.  Lets tests pin the tensor-core
+ * distance and its error bound against the oracle's definition.
  * Workspace from knn_distances_workspace(N, Q, D). */
 KSEL_API size_t knn_distances_workspace(int64_t N, int64_t Q, int D);
 KSEL_API int knn_distances(const float* ref, const float* query, int64_t N, int64_t Q, int D, float* out,
-                           void* d_work, size_t work_bytes, void* stream);
+                           float* out_eps, void* d_work, size_t work_bytes, void* stream);
 
 /* ksel_select_paper -- ABLATION, not the hot path: the
  * paper's own per-thread designs, one thread per query, on B200.

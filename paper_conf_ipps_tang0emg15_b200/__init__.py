@@ -60,7 +60,7 @@ _lib.knn_graph.argtypes = [_p, _i64, _i32, _i32, _p, _p, _p, _sz, _p]
 _lib.knn_graph.restype = ctypes.c_int
 _lib.knn_distances_workspace.argtypes = [_i64, _i64, _i32]
 _lib.knn_distances_workspace.restype = _sz
-_lib.knn_distances.argtypes = [_p, _p, _i64, _i64, _i32, _p, _p, _sz, _p]
+_lib.knn_distances.argtypes = [_p, _p, _i64, _i64, _i32, _p, _p, _p, _sz, _p]
 _lib.knn_distances.restype = ctypes.c_int
 _lib.ksel_timing_enable.argtypes = [_i32]
 _lib.ksel_timing_enable.restype = ctypes.c_int
@@ -329,8 +329,9 @@ def knn_graph(points: torch.Tensor, k: int, out_dist: torch.Tensor | None = None
     return out_dist, out_idx
 
 
-def knn_distances(ref: torch.Tensor, query: torch.Tensor, out: torch.Tensor | None = None):
-    """DIAGNOSTIC: the tensor-core squared distances [Q, N] (materialised)."""
+def knn_distances(ref: torch.Tensor, query: torch.Tensor, out: torch.Tensor | None = None, with_eps: bool = False):
+    """DIAGNOSTIC: the tensor-core filter distances d~ [Q, N] (materialised); with_eps
+    also returns the per-query bound eps [Q] with |d~ - d| <= eps."""
     _dev_f32(ref, "ref", 2)
     _dev_f32(query, "query", 2)
     N, D = ref.shape
@@ -339,11 +340,13 @@ def knn_distances(ref: torch.Tensor, query: torch.Tensor, out: torch.Tensor | No
     if out is None:
         out = torch.empty((Q, N), dtype=torch.float32, device=ref.device)
     _out(out, "out", (Q, N), torch.float32, ref.device)
+    eps = torch.empty(Q, dtype=torch.float32, device=ref.device) if with_eps else None
     ws = torch.empty(max(1, int(_lib.knn_distances_workspace(N, Q, D))), dtype=torch.uint8, device=ref.device)
     with torch.cuda.device(ref.device):
         _check("knn_distances", _lib.knn_distances(ref.data_ptr(), query.data_ptr(), N, Q, D, out.data_ptr(),
-                                                   ws.data_ptr(), ws.numel(), _stream(ref.device)))
-    return out
+                                                   eps.data_ptr() if with_eps else None, ws.data_ptr(),
+                                                   ws.numel(), _stream(ref.device)))
+    return (out, eps) if with_eps else out
 
 
 # ---- collective-free exchange (ksel_ipc_*, ksel_flag_*, ksel_merge_lists) ----

@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 
 #include "ksel_internal.h"
+#include "knn_common.cuh"
 
 namespace ksel {
 
@@ -60,10 +61,13 @@ cudaError_t launch_merge(const MergeLists& L, int64_t Q, int S, int kin, int k, 
     KSEL_DISPATCH_R(launch_merge_r, queue_regs(k), L, Q, S, kin, k, ov, oi, stream)
 }
 
-cudaError_t launch_merge_pools(const unsigned long long* pools, int64_t P, const int32_t* cnt, int S, int64_t Q,
-                               const unsigned long long* thr, int k, int64_t idx_offset, float* ov, int32_t* oi,
-                               cudaStream_t stream) {
-    KSEL_DISPATCH_R(launch_merge_pools_r, queue_regs(k), pools, P, cnt, S, Q, thr, k, idx_offset, ov, oi, stream)
+cudaError_t launch_knn_rescore(const KnnRescoreArgs& a, cudaStream_t stream) {
+    KSEL_DISPATCH_R(launch_knn_rescore_r, queue_regs(a.k), a, stream)
 }
+
+cudaError_t launch_knn_fallback(const KnnRescoreArgs& a, cudaStream_t stream) {
+    KSEL_DISPATCH_R(launch_knn_fallback_r, queue_regs(a.k), a, stream)
+}
+
 
 }  // namespace ksel

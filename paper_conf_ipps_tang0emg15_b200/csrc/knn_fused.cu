@@ -1,38 +1,42 @@
-// knn_fused.cu -- knn_search: tcgen05/TMEM distance GEMM fused with k-selection.
+// knn_fused.cu -- knn_search: tcgen05/TMEM distance FILTER fused with k-selection,
+// followed by exact rescoring of the survivors (knn_rescore.cu).
 //
 // The k-NN of the paper has two phases (Sec. II.A): Euclidean
 // distances between every query and reference, then k-selection over each
 // query's row of N distances.  The paper computes the Q x N matrix with "the
 // method of [3]" and stores it in global memory (L243); here the matrix never
-// exists.  d(q, r) = |q|^2 + |r|^2 - 2 q.r (reading R9: squared L2), with the dot
+// exists.  d~(q, r) = |q|^2 + |r|^2 - 2 q.r (reading R9: squared L2), with the dot
 // products on the 5th-gen tensor cores:
 //
 //   * operands split once into bf16 hi/lo pairs (x ~ hi + lo, hi = bf16(x),
 //     lo = bf16(x - hi)); q.r ~ qh.rh + qh.rl + ql.rh -- three kind::f16 MMAs
-//     into one fp32 TMEM accumulator (the dropped ql.rl term is ~2^-16 relative;
-//     SURVEY 7.3 emulation: 8.8e-6 max relative error vs the 1e-4 bar).
-//     Integer data in [0,255] is exact (lo = 0).
+//     into one fp32 TMEM accumulator (the dropped ql.rl term is ~2^-16 relative).
 //   * the norms ride in the same accumulation: A holds -2q and one extra
 //     16-wide K block [n1, n2, n3, 1, 1, 1, 0...] with |q|^2 = n1+n2+n3 split
 //     three ways in bf16 (24 significant bits), B holds [1, 1, 1, m1, m2, m3, 0...]
-//     for |r|^2 -- so the accumulator IS d(q, r) and the epilogue touches each
+//     for |r|^2 -- so the accumulator IS d~(q, r) and the epilogue touches each
 //     distance once (no per-element norm adds).
+//   * d~ only FILTERS: |d~ - d| <= eps_q (a rigorous bound, knn_common.cuh knn_eps,
+//     DESIGN.md reading R21, ~1e-3 of the distance on the paper's workload), so a
+//     reference can be in the exact top-k only if d~ <= T + 2 eps_q for any k-th
+//     value T of d~ over k references; the epilogue admits exactly those, pools keep
+//     that band above their k-th d~, and knn_rescore.cu recomputes every survivor in
+//     the oracle's own arithmetic and selects the exact top-k -- bit-identical to the
+//     CPU oracle.  A query whose band overflows its pool (massive ties of d~, or
+//     non-finite input) is flagged and solved by an exact brute-force fallback.
 //   * CTA = one tile of 128 queries (TMEM lanes, A operand resident in shared
 //     memory) x a contiguous range of 256-reference tiles (TMEM columns, B
 //     operand streamed by 1-D TMA bulk copies from a pre-tiled image);
 //     warp 0 = producer, warp 1 = TMEM allocator + single-thread MMA issuer,
 //     warps 2-5 = epilogue (one thread per query: the paper's thread-per-query
 //     layout, L243), double-buffered 2 x 256-column accumulators.
-//   * epilogue: tcgen05.ld 64 columns at a time (the accumulator already is the
-//     distance), an fp32 min/vote pre-filter against the running bound, a rare
-//     path that appends packed (key << 32 | index) pairs to a per-query pool in
-//     global memory, warp-cooperative narrowing (register bisection, radix
-//     select for large pools) when a pool fills; the k-th pair of every
-//     narrowing is published per query (atomicMin) so all splits share bounds.
-//   * each CTA leaves its per-query pools (a superset of its reference range's
-//     share of the top-k); launch_merge_pools (merge.cu) gathers the pairs below
-//     the final shared bound and selects and sorts the exact top-k -- the
-//     divide-and-merge of L243.
+//   * epilogue: tcgen05.ld 32 columns at a time, an fp32 min/vote pre-filter against
+//     the running bound plus the band, a rare path that appends packed
+//     (key(d~) << 32 | index) pairs to a per-query pool in global memory,
+//     warp-cooperative narrowing (register bisection, radix select for large pools)
+//     when a pool fills; the k-th pair of every narrowing is published per query
+//     (atomicMin) so all splits share bounds.
+//   * queries are processed in chunks so that the pools stay below 2 GiB.
 #include <algorithm>
 #include <cstdint>
 #include <cstdlib>
@@ -45,6 +49,7 @@
 #include "ksel_common.cuh"
 #include "ksel_internal.h"
 #include "ksel_pool.cuh"
+#include "knn_common.cuh"
 
 namespace ksel {
 
@@ -58,7 +63,6 @@ constexpr int KNN_MAX_EW = 8;
 __host__ __device__ constexpr int knn_threads(int ew) { return 64 + 32 * ew; }
 constexpr int KNN_SB = 32;                                // sampling histogram buckets
 constexpr int KNN_CW = 64;                                // accumulator columns per epilogue step
-constexpr int KNN_MAX_D = 256;
 constexpr int kNarrowRegs = 40;  // register-resident narrowing: pools of <= 1280 pairs
 constexpr unsigned long long kSentPair = ((unsigned long long)kSentKey << 32) | kSentIdx;
 
@@ -123,11 +127,15 @@ __device__ __forceinline__ uint32_t bf2(float a, float b) {
 constexpr int KNN_PREP_THREADS = 256;
 
 __global__ void __launch_bounds__(KNN_PREP_THREADS)
-    knn_prep_kernel(const float* __restrict__ ref, const float* __restrict__ qry, KnnGeom g,
-                    uint4* __restrict__ ref_img, uint4* __restrict__ q_img) {
+    knn_prep_kernel(const float* __restrict__ ref, const float* __restrict__ qry, KnnGeom g, int nt,
+                    uint4* __restrict__ ref_img, uint4* __restrict__ q_img, float4* __restrict__ qstat,
+                    KnnStats* __restrict__ st) {
+    // blocks [0, nt): reference tiles (nt = NT on a call's first query chunk, else 0)
     __shared__ float tile[KNN_BN][KNN_KS + 1];
-    const bool is_q = blockIdx.x >= (unsigned)g.NT;
-    const int64_t t = is_q ? (int64_t)blockIdx.x - g.NT : (int64_t)blockIdx.x;
+    __shared__ uint32_t smax;  // max |r|^2 of this block's references (one global atomic per block)
+    if (threadIdx.x == 0) smax = 0u;
+    const bool is_q = blockIdx.x >= (unsigned)nt;
+    const int64_t t = is_q ? (int64_t)blockIdx.x - nt : (int64_t)blockIdx.x;
     const int rows = is_q ? KNN_BM : g.BN;
     const int64_t n = is_q ? g.Q : g.N;
     const float* x = is_q ? qry : ref;
@@ -174,6 +182,12 @@ __global__ void __launch_bounds__(KNN_PREP_THREADS)
         __syncthreads();
     }
     if (tid < rows) {
+        // the filter's error bound needs |q|^2 per query and max |r|^2 (rounded up)
+        const float sr = __double2float_ru(s);
+        if (row < n) {
+            if (is_q) qstat[row] = make_float4(0.f, 0.f, 0.f, sr);
+            else atomicMax(&smax, __float_as_uint(sr == sr ? sr : __int_as_float(0x7f800000)));  // block max
+        }
         const float n1 = __bfloat162float(__float2bfloat16_rn((float)s));
         const float n2 = __bfloat162float(__float2bfloat16_rn((float)(s - (double)n1)));
         const float n3 = __bfloat162float(__float2bfloat16_rn((float)(s - (double)n1 - (double)n2)));
@@ -189,6 +203,10 @@ __global__ void __launch_bounds__(KNN_PREP_THREADS)
         }
         blk[tid] = c0;
         blk[rows + tid] = make_uint4(0u, 0u, 0u, 0u);
+    }
+    if (!is_q) {  // (uniform per block)
+        __syncthreads();
+        if (tid == 0 && smax) atomicMax(&st->R2, smax);
     }
 }
 
@@ -323,8 +341,9 @@ struct KnnSmem {
 template <int MODE, int EW, int BN, int QPC>
 __global__ void __launch_bounds__(knn_threads(EW), 1)
     knn_fused_kernel(KnnGeom g, const uint8_t* __restrict__ ref_img, const uint8_t* __restrict__ q_img,
+                     const float4* __restrict__ qstat, const KnnStats* __restrict__ st,
                      unsigned long long* __restrict__ pool64, int32_t* __restrict__ cnt_out,
-                     unsigned long long* __restrict__ qthr, float* __restrict__ dump) {
+                     unsigned long long* __restrict__ qthr, int32_t* __restrict__ qfail, float* __restrict__ dump) {
     constexpr int HALVES = (QPC == 1) ? EW / 4 : 1;
     constexpr int WCOLS = BN / HALVES;  // columns of each tile this epilogue warp scans
     constexpr int SB = 2 * KNN_KS * BN * 2;   // bytes of one reference stage
@@ -485,38 +504,51 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
         // (each (split, half) keeps its own pools: S * HALVES lists per query for the merge)
         const size_t list = (size_t)split * HALVES + half;
         unsigned long long* pool = pool64 + (list * g.Q + (qvalid ? q : 0)) * g.P;
-        unsigned long long T = kSentPair;  // running bound on the k-th pair
-        float tv = 0.f;
-        bool fast = false;                 // T below +Inf: the fp32 compare d <= tv pre-filters
+        unsigned long long T = kSentPair;  // running bound on the k-th (d~, index) pair
+        // the band: 2 eps_q above the k-th d~ (every reference that can be in the exact top-k)
+        const float band = (qvalid && !DUMP) ? __fmul_ru(2.f, knn_eps(qstat[q], *st, g.D)) : 0.f;
+        float tv = 0.f;                    // filter value: value(T) + band, rounded up
+        bool fast = false;                 // finite filter value: the fp32 compare d~ <= tv pre-filters
+        bool failed = !(band < __int_as_float(0x7f800000));  // no finite band: exact fallback
+        if (qvalid && !DUMP && !PIPE_ONLY && failed) qfail[q] = 1;
         int n = 0;
 
         auto adopt = [&](unsigned long long t) {
             if (t < T) {
                 T = t;
-                fast = (uint32_t)(T >> 32) < 0xff800000u;
-                tv = __uint_as_float(bits_of_key((uint32_t)(T >> 32)));
+                const uint32_t tk = (uint32_t)(T >> 32);
+                tv = (tk < 0xff800000u) ? __fadd_ru(__uint_as_float(bits_of_key(tk)), band) : 0.f;
+                fast = tk < 0xff800000u && tv < __int_as_float(0x7f800000);
             }
         };
-        // warp-cooperative narrowing of every lane whose pool cannot take `room` more pairs
-        auto narrow_lanes = [&](int room, int target, int cap) {
-            uint32_t need = __ballot_sync(kFull, qvalid && n + room > cap);
+        // warp-cooperative narrowing of every lane whose pool cannot take `room` more pairs:
+        // the exact k-th pair of the pool becomes the bound and the pool keeps the band
+        // above it; mid-stream, a band that alone leaves no room fails the query
+        auto narrow_lanes = [&](int room, int target, int cap, bool final_pass) {
+            uint32_t need = __ballot_sync(kFull, qvalid && !failed && n + room > cap && n > target);
             while (need) {
                 if (PROF) prof_nnarrow++;
                 const int j = __ffs(need) - 1;
                 need &= need - 1u;
                 unsigned long long* jp = (unsigned long long*)__shfl_sync(kFull, (unsigned long long)pool, j);
                 const int jn = __shfl_sync(kFull, n, j);
+                const float jb = __shfl_sync(kFull, band, j);
                 int nn;
-                const unsigned long long t = (jn <= 256)   ? pool_narrow64<8>(jp, jn, (uint32_t)target, &nn)
-                                             : (jn <= 512) ? pool_narrow64<16>(jp, jn, (uint32_t)target, &nn)
+                const unsigned long long t = (jn <= 256)   ? pool_narrow64<8>(jp, jn, (uint32_t)target, &nn, jb)
+                                             : (jn <= 512) ? pool_narrow64<16>(jp, jn, (uint32_t)target, &nn, jb)
                                              : (jn <= 32 * kNarrowRegs)
-                                                 ? pool_narrow64<kNarrowRegs>(jp, jn, (uint32_t)target, &nn)
-                                                 : pool_select64(jp, jn, (uint32_t)target, hist, &nn);
+                                                 ? pool_narrow64<kNarrowRegs>(jp, jn, (uint32_t)target, &nn, jb)
+                                                 : pool_select64(jp, jn, (uint32_t)target, hist, &nn, jb);
                 if ((int)lane == j) {
                     n = nn;
                     adopt(t);
                     // publish: the k-th pair of this split's part bounds the whole row
                     if (target == g.k && (uint32_t)(t >> 32) != kSentKey) atomicMin(&qthr[q], t);
+                    if (!final_pass && n + room > cap) {  // the band alone fills the pool
+                        failed = true;
+                        n = 0;
+                        qfail[q] = 1;
+                    }
                 }
             }
             __syncwarp();
@@ -537,7 +569,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                 adopt(thr_next);
                 if (qvalid) thr_next = __ldcg(&qthr[q]);
                 const unsigned long long c0 = PROF ? clock64() : 0;
-                narrow_lanes(WCOLS, g.k, g.pcap);
+                narrow_lanes(WCOLS, g.k, g.pcap, false);
                 if (PROF) prof_narrow += clock64() - c0;
             }
             const unsigned long long cw0 = PROF ? clock64() : 0;
@@ -635,6 +667,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                 // lane needs are visited (candidates appended, predicated, from registers).
                 const uint32_t colt = (uint32_t)t * BN;  // N < 2^31
                 const int nlim = (int)min((int64_t)BN, g.N - (int64_t)colt);  // valid columns of the tile
+                const bool live = qvalid && !failed;
                 auto scan32 = [&](const uint32_t(&v)[32], int c0) {
                     float gmn[8];
 #pragma unroll
@@ -643,7 +676,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                                        fminf(__uint_as_float(v[4 * j + 2]), __uint_as_float(v[4 * j + 3])));
                     const float mn = fminf(fminf(fminf(gmn[0], gmn[1]), fminf(gmn[2], gmn[3])),
                                            fminf(fminf(gmn[4], gmn[5]), fminf(gmn[6], gmn[7])));
-                    if (!__any_sync(kFull, qvalid && (!fast || mn <= tv))) return;
+                    if (!__any_sync(kFull, live && (!fast || mn <= tv))) return;
                     const unsigned long long cr0 = PROF ? clock64() : 0;
                     // rare path: each lane visits only its own candidate groups (a divergent
                     // loop of max-over-lanes length); the group's 4 values are picked from the
@@ -653,7 +686,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                     uint32_t gm = 0;
 #pragma unroll
                     for (int u = 0; u < 8; ++u) gm |= (uint32_t)(!fast || gmn[u] <= tv) << u;
-                    if (!qvalid) gm = 0;
+                    if (!live) gm = 0;
                     while (gm) {
                         const int u = __ffs(gm) - 1;
                         gm &= gm - 1u;
@@ -717,8 +750,8 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
             // pair of this split in the row's top-k (all pairs <= any bound; narrowing keeps
             // the pool's k smallest); launch_merge_pools gathers the pools' pairs <= the
             // final published bound and selects the exact top-k of the row.
-            narrow_lanes(g.P - g.k, g.k, g.P);  // n > k  <=>  n + (P - k) > P
-            if (qvalid) cnt_out[list * g.Q + q] = n;
+            narrow_lanes(g.P - g.k, g.k, g.P, true);  // n > k  <=>  n + (P - k) > P
+            if (qvalid) cnt_out[list * g.Q + q] = failed ? 0 : n;
         }
         if (PROF) {
             __syncwarp();
@@ -744,10 +777,18 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
 static size_t al256(size_t x) { return (x + 255u) & ~(size_t)255u; }
 
 struct KnnWork {
-    size_t ref_img, q_img, pool, cnt, qthr, prof, total;
+    size_t ref_img, stats, q_img, qstat, pool, cnt, qthr, qfail, fb, prof, total;
 };
 
-static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int64_t idx_offset) {
+// Queries are processed in chunks (multiples of 128 queries) so that the pools,
+// lists * Qc * P * 8 bytes, stay below kPoolBudget (a k-NN graph of 10^6
+// points would otherwise need tens of GB of workspace).
+constexpr size_t kPoolBudget = 2ull << 30;
+
+// max_lists > 0: cap the split count so that S * halves * Q <= max_lists (a later query
+// chunk must fit the workspace laid out for the first)
+static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int64_t idx_offset,
+                            int64_t max_lists = 0) {
     KnnGeom g{};
     g.N = N;
     g.Q = Q;
@@ -825,6 +866,7 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     double best_cost = 1e30;
     const int smax = (int)((g.NT < 64) ? g.NT : 64);
     for (int s = 1; s <= smax; ++s) {
+        if (max_lists > 0 && s > 1 && (int64_t)s * g.halves * Q > max_lists) break;
         const double ctas = (double)g.QTp * s;
         const double waves = ctas / num_sms;
         const double cost = (double)((int64_t)((ctas + num_sms - 1) / num_sms)) / waves  // tail efficiency
@@ -836,7 +878,10 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     static const int coldw_env = env_int("KSEL_KNN_COLDW", 1000);  // experiments: first-wave split weight (per mille)
     g.cold_w = (coldw_env > 0 && coldw_env <= 1000) ? coldw_env : 1000;
     static const int splits_env = env_int("KSEL_KNN_SPLITS", 0);  // experiments: force the split count
-    if (splits_env > 0) g.S = std::min(splits_env, smax);
+    if (splits_env > 0) {
+        g.S = std::min(splits_env, smax);
+        if (max_lists > 0) g.S = (int)std::max<int64_t>(1, std::min<int64_t>(g.S, max_lists / (g.halves * Q)));
+    }
     g.cold_splits = std::min(g.S, (num_sms + g.QTp - 1) / g.QTp);
     return g;
 }
@@ -845,13 +890,31 @@ static KnnWork knn_work_layout(const KnnGeom& g) {
     KnnWork w{};
     size_t off = 0;
     w.ref_img = off; off += al256((size_t)g.NT * g.tile_bytes());
-    w.q_img = off;   off += al256((size_t)g.QT * g.a_bytes());
-    w.pool = off;    off += al256((size_t)2 * g.S * g.Q * g.P * 8);  // 2 lists (column halves) per split
-    w.cnt = off;     off += al256((size_t)2 * g.S * g.Q * 4);
+    w.stats = off;   off += al256(sizeof(KnnStats));
+    w.q_img = off;   off += al256((size_t)g.QTp * g.QPC * g.a_bytes());
+    w.qstat = off;   off += al256((size_t)g.Q * 16);
+    w.pool = off;    off += al256((size_t)g.halves * g.S * g.Q * g.P * 8);
+    w.cnt = off;     off += al256((size_t)g.halves * g.S * g.Q * 4);
     w.qthr = off;    off += al256((size_t)g.Q * 8);
+    w.qfail = off;   off += al256((size_t)g.Q * 4);
+    w.fb = off;      off += al256(knn_fallback_bytes(g.k));
     w.prof = off;    off += al256((size_t)g.QTp * g.S * KNN_MAX_EW * 16 * 8);  // MODE 3 counters
     w.total = off;
     return w;
+}
+
+// queries per chunk (a multiple of 128, or Q), so that the pools fit kPoolBudget
+static int64_t knn_query_chunk(int64_t N, int64_t Q, int D, int k, int sms) {
+    int64_t qc = Q;
+    for (;;) {
+        const KnnGeom g = knn_geometry(N, qc, D, k, sms, 0);
+        if ((size_t)g.halves * g.S * (size_t)qc * (size_t)g.P * 8u <= kPoolBudget || qc <= KNN_BM) return qc;
+        qc = std::max<int64_t>(KNN_BM, (qc / 2 + KNN_BM - 1) / KNN_BM * KNN_BM);
+    }
+}
+
+static size_t knn_workspace_bytes(int64_t N, int64_t Q, int D, int k, int sms) {
+    return knn_work_layout(knn_geometry(N, knn_query_chunk(N, Q, D, k, sms), D, k, sms, 0)).total;
 }
 
 static int knn_device_sms() {
@@ -859,71 +922,123 @@ static int knn_device_sms() {
     return current_device_info(&di) == KSEL_OK ? di.sms : 148;
 }
 
-static cudaError_t knn_run(const float* ref, const float* query, const KnnGeom& g, uint8_t* work,
-                           float* out_dist, int32_t* out_idx, float* dump, cudaStream_t stream) {
-    const KnnWork w = knn_work_layout(g);
+// knn_distances: the bound eps_q of every query (diagnostic output)
+__global__ void knn_eps_kernel(const float4* __restrict__ qstat, const KnnStats* __restrict__ st, int D, int64_t Q,
+                               float* __restrict__ out) {
+    const int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (q < Q) out[q] = knn_eps(qstat[q], *st, D);
+}
+
+// The reference image is built once per call (with the first query chunk); queries go
+// in chunks of Qc, the workspace laid out for a full chunk (gq).
+static cudaError_t knn_run(const float* ref, const float* query, int64_t N, int64_t Q, int D, int k,
+                           int64_t idx_offset, uint8_t* work, float* out_dist, int32_t* out_idx, float* dump,
+                           float* dump_eps, int sms, cudaStream_t stream) {
+    const int64_t Qc = knn_query_chunk(N, Q, D, k, sms);
+    const KnnGeom gq = knn_geometry(N, Qc, D, k, sms, idx_offset);
+    const KnnWork w = knn_work_layout(gq);
     uint4* ref_img = reinterpret_cast<uint4*>(work + w.ref_img);
     uint4* q_img = reinterpret_cast<uint4*>(work + w.q_img);
-
-    knn_prep_kernel<<<(unsigned)(g.NT + g.QT), KNN_PREP_THREADS, 0, stream>>>(ref, query, g, ref_img, q_img);
-    note_launch();
-    cudaError_t e = cudaGetLastError();
+    float4* qstat = reinterpret_cast<float4*>(work + w.qstat);
+    KnnStats* stats = reinterpret_cast<KnnStats*>(work + w.stats);
+    cudaError_t e = cudaMemsetAsync(stats, 0, sizeof(KnnStats), stream);
     if (e != cudaSuccess) return e;
-
-    e = cudaMemsetAsync(work + w.qthr, 0xff, (size_t)g.Q * 8, stream);  // "no bound yet"
-    if (e != cudaSuccess) return e;
-    const int smem = KnnSmem::total(g);
+    for (int64_t q0 = 0; q0 < Q; q0 += Qc) {
+        const int64_t nq = std::min(Qc, Q - q0);
+        const KnnGeom g = knn_geometry(N, nq, D, k, sms, idx_offset, (int64_t)gq.halves * gq.S * Qc);
+        const int nt = (q0 == 0) ? g.NT : 0;  // reference tiles: first chunk only
+        knn_prep_kernel<<<(unsigned)(nt + g.QT), KNN_PREP_THREADS, 0, stream>>>(
+            ref, query + q0 * (int64_t)D, g, nt, ref_img, q_img, qstat, stats);
+        note_launch();
+        e = cudaGetLastError();
+        if (e == cudaSuccess) e = cudaMemsetAsync(work + w.qthr, 0xff, (size_t)nq * 8, stream);  // "no bound yet"
+        if (e == cudaSuccess) e = cudaMemsetAsync(work + w.qfail, 0, (size_t)nq * 4, stream);
+        if (e != cudaSuccess) return e;
+        const int smem = KnnSmem::total(g);
+        float* kdump = dump ? dump + q0 * N : nullptr;
 #ifdef KSEL_EXPERIMENTS
-    // Timing experiments only (a -DKSEL_EXPERIMENTS build; the product library has none of
-    // these): 2 pipeline only, 3 counters, 4 no TMEM reads -- modes 2 and 4 return no result.
-    static const int mode_env = [] {
-        const int m = env_int("KSEL_KNN_MODE", 0);
-        return (m >= 2 && m <= 4) ? m : 0;
-    }();
-    const bool ew8 = g.halves == 2;
-    auto kern = (g.QPC == 2)
-                    ? (dump ? knn_fused_kernel<1, 8, 128, 2>
-                       : mode_env == 2 ? knn_fused_kernel<2, 8, 128, 2>
-                       : mode_env == 3 ? knn_fused_kernel<3, 8, 128, 2>
-                       : mode_env == 4 ? knn_fused_kernel<4, 8, 128, 2>
-                                       : knn_fused_kernel<0, 8, 128, 2>)
-                : dump ? (ew8 ? knn_fused_kernel<1, 8, 256, 1> : knn_fused_kernel<1, 4, 256, 1>)
-                : mode_env == 2 ? (ew8 ? knn_fused_kernel<2, 8, 256, 1> : knn_fused_kernel<2, 4, 256, 1>)
-                : mode_env == 3 ? (ew8 ? knn_fused_kernel<3, 8, 256, 1> : knn_fused_kernel<3, 4, 256, 1>)
-                : mode_env == 4 ? knn_fused_kernel<4, 4, 256, 1>
-                                : (ew8 ? knn_fused_kernel<0, 8, 256, 1> : knn_fused_kernel<0, 4, 256, 1>);
+        // Timing experiments only (a -DKSEL_EXPERIMENTS build; the product library has none of
+        // these): 2 pipeline only, 3 counters, 4 no TMEM reads -- modes 2 and 4 return no result.
+        static const int mode_env = [] {
+            const int m = env_int("KSEL_KNN_MODE", 0);
+            return (m >= 2 && m <= 4) ? m : 0;
+        }();
+        const bool ew8 = g.halves == 2;
+        auto kern = (g.QPC == 2)
+                        ? (dump ? knn_fused_kernel<1, 8, 128, 2>
+                           : mode_env == 2 ? knn_fused_kernel<2, 8, 128, 2>
+                           : mode_env == 3 ? knn_fused_kernel<3, 8, 128, 2>
+                           : mode_env == 4 ? knn_fused_kernel<4, 8, 128, 2>
+                                           : knn_fused_kernel<0, 8, 128, 2>)
+                    : dump ? (ew8 ? knn_fused_kernel<1, 8, 256, 1> : knn_fused_kernel<1, 4, 256, 1>)
+                    : mode_env == 2 ? (ew8 ? knn_fused_kernel<2, 8, 256, 1> : knn_fused_kernel<2, 4, 256, 1>)
+                    : mode_env == 3 ? (ew8 ? knn_fused_kernel<3, 8, 256, 1> : knn_fused_kernel<3, 4, 256, 1>)
+                    : mode_env == 4 ? knn_fused_kernel<4, 4, 256, 1>
+                                    : (ew8 ? knn_fused_kernel<0, 8, 256, 1> : knn_fused_kernel<0, 4, 256, 1>);
+        if (!dump && mode_env == 3) kdump = reinterpret_cast<float*>(work + w.prof);
 #else
-    constexpr int mode_env = 0;
-    auto kern = dump ? knn_fused_kernel<1, 4, 256, 1> : knn_fused_kernel<0, 4, 256, 1>;
+        constexpr int mode_env = 0;
+        auto kern = dump ? knn_fused_kernel<1, 4, 256, 1> : knn_fused_kernel<0, 4, 256, 1>;
 #endif
-    if (!dump && mode_env == 3) dump = reinterpret_cast<float*>(work + w.prof);
-    e = ensure_smem_attr(reinterpret_cast<const void*>(kern), smem);
-    if (e != cudaSuccess) return e;
-    const int slot = dump ? -1 : timing_begin(stream);
-    cudaLaunchConfig_t cfg{};
-    cudaLaunchAttribute attr[1];
-    cfg.gridDim = dim3((unsigned)(g.QTp * g.S));
-    cfg.blockDim = dim3((unsigned)knn_threads(g.EW));
-    cfg.dynamicSmemBytes = (size_t)smem;
-    cfg.stream = stream;
-    attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = (unsigned)g.cs;
-    attr[0].val.clusterDim.y = 1;
-    attr[0].val.clusterDim.z = 1;
-    cfg.attrs = attr;
-    cfg.numAttrs = 1;
-    e = cudaLaunchKernelEx(&cfg, kern, g, reinterpret_cast<const uint8_t*>(ref_img),
-                           reinterpret_cast<const uint8_t*>(q_img), reinterpret_cast<unsigned long long*>(work + w.pool),
-                           reinterpret_cast<int32_t*>(work + w.cnt), reinterpret_cast<unsigned long long*>(work + w.qthr),
-                           dump);
-    note_launch();
-    timing_end(slot, stream);
-    if (e == cudaSuccess) e = cudaGetLastError();
-    if (e != cudaSuccess || (dump && mode_env != 3)) return e;
-    return launch_merge_pools(reinterpret_cast<const unsigned long long*>(work + w.pool), g.P,
-                              reinterpret_cast<const int32_t*>(work + w.cnt), g.halves * g.S, g.Q,
-                              reinterpret_cast<const unsigned long long*>(work + w.qthr), g.k, g.idx_offset, out_dist,
-                              out_idx, stream);
+        e = ensure_smem_attr(reinterpret_cast<const void*>(kern), smem);
+        if (e != cudaSuccess) return e;
+        const int slot = dump ? -1 : timing_begin(stream);
+        cudaLaunchConfig_t cfg{};
+        cudaLaunchAttribute attr[1];
+        cfg.gridDim = dim3((unsigned)(g.QTp * g.S));
+        cfg.blockDim = dim3((unsigned)knn_threads(g.EW));
+        cfg.dynamicSmemBytes = (size_t)smem;
+        cfg.stream = stream;
+        attr[0].id = cudaLaunchAttributeClusterDimension;
+        attr[0].val.clusterDim.x = (unsigned)g.cs;
+        attr[0].val.clusterDim.y = 1;
+        attr[0].val.clusterDim.z = 1;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
+        e = cudaLaunchKernelEx(&cfg, kern, g, reinterpret_cast<const uint8_t*>(ref_img),
+                               reinterpret_cast<const uint8_t*>(q_img), static_cast<const float4*>(qstat),
+                               static_cast<const KnnStats*>(stats), reinterpret_cast<unsigned long long*>(work + w.pool),
+                               reinterpret_cast<int32_t*>(work + w.cnt),
+                               reinterpret_cast<unsigned long long*>(work + w.qthr),
+                               reinterpret_cast<int32_t*>(work + w.qfail), kdump);
+        note_launch();
+        timing_end(slot, stream);
+        if (e == cudaSuccess) e = cudaGetLastError();
+        if (e != cudaSuccess) return e;
+        if (dump) {
+            if (dump_eps) {
+                knn_eps_kernel<<<(unsigned)((nq + 255) / 256), 256, 0, stream>>>(qstat, stats, D, nq, dump_eps + q0);
+                note_launch();
+                e = cudaGetLastError();
+                if (e != cudaSuccess) return e;
+            }
+            continue;
+        }
+        if (mode_env == 3) continue;
+        KnnRescoreArgs a{};
+        a.ref = ref;
+        a.query = query + q0 * (int64_t)D;
+        a.N = N;
+        a.Q = nq;
+        a.D = D;
+        a.k = k;
+        a.idx_offset = idx_offset;
+        a.pools = reinterpret_cast<const unsigned long long*>(work + w.pool);
+        a.P = g.P;
+        a.cnt = reinterpret_cast<const int32_t*>(work + w.cnt);
+        a.S = g.halves * g.S;
+        a.thr = reinterpret_cast<const unsigned long long*>(work + w.qthr);
+        a.qfail = reinterpret_cast<const int32_t*>(work + w.qfail);
+        a.qstat = qstat;
+        a.stats = stats;
+        a.fb = work + w.fb;
+        a.out_val = out_dist + q0 * k;
+        a.out_idx = out_idx + q0 * k;
+        e = launch_knn_rescore(a, stream);
+        if (e == cudaSuccess) e = launch_knn_fallback(a, stream);
+        if (e != cudaSuccess) return e;
+    }
+    return cudaSuccess;
 }
 
 static int knn_check(const float* ref, const float* query, int64_t N, int64_t Q, int D, int k, int64_t idx_offset) {
@@ -968,8 +1083,7 @@ extern "C" {
 
 size_t knn_search_workspace(int64_t N, int64_t Q, int D, int k) {
     if (N < 1 || Q < 1 || D < 1 || D > KNN_MAX_D || k < 1 || k > KSEL_MAX_K) return 0;
-    const KnnGeom g = knn_geometry(N, Q, D, k, knn_device_sms(), 0);
-    return knn_work_layout(g).total;
+    return knn_workspace_bytes(N, Q, D, k, knn_device_sms());
 }
 
 int knn_search(const float* ref, const float* query, int64_t N, int64_t Q, int D, int k, float* out_dist,
@@ -980,10 +1094,9 @@ int knn_search(const float* ref, const float* query, int64_t N, int64_t Q, int D
     DevInfo di;
     st = current_device_info(&di);
     if (st) return st;
-    const KnnGeom g = knn_geometry(N, Q, D, k, di.sms, idx_offset);
-    if (work_bytes < knn_work_layout(g).total) return KSEL_ERR_INVALID_ARG;
-    cudaError_t e = knn_run(ref, query, g, static_cast<uint8_t*>(d_work), out_dist, out_idx, nullptr,
-                            (cudaStream_t)stream);
+    if (work_bytes < knn_workspace_bytes(N, Q, D, k, di.sms)) return KSEL_ERR_INVALID_ARG;
+    cudaError_t e = knn_run(ref, query, N, Q, D, k, idx_offset, static_cast<uint8_t*>(d_work), out_dist, out_idx,
+                            nullptr, nullptr, di.sms, (cudaStream_t)stream);
     return e == cudaSuccess ? KSEL_OK : KSEL_ERR_CUDA;
 }
 
@@ -1003,14 +1116,14 @@ int knn_graph(const float* points, int64_t N, int D, int k, float* out_dist, int
     DevInfo di;
     st = current_device_info(&di);
     if (st) return st;
-    const KnnGeom g = knn_geometry(N, N, D, k + 1, di.sms, 0);
-    const size_t base = al256(knn_work_layout(g).total);
+    const size_t base = al256(knn_workspace_bytes(N, N, D, k + 1, di.sms));
     const size_t tmp = al256((size_t)N * (k + 1) * 4);
     if (work_bytes < base + 2 * tmp) return KSEL_ERR_INVALID_ARG;
     uint8_t* w = static_cast<uint8_t*>(d_work);
     float* tv = reinterpret_cast<float*>(w + base);
     int32_t* ti = reinterpret_cast<int32_t*>(w + base + tmp);
-    cudaError_t e = knn_run(points, points, g, w, tv, ti, nullptr, (cudaStream_t)stream);
+    cudaError_t e = knn_run(points, points, N, N, D, k + 1, 0, w, tv, ti, nullptr, nullptr, di.sms,
+                            (cudaStream_t)stream);
     if (e != cudaSuccess) return KSEL_ERR_CUDA;
     knn_drop_self_kernel<<<(unsigned)((N + 7) / 8), 256, 0, (cudaStream_t)stream>>>(tv, ti, N, k, out_dist, out_idx);
     note_launch();
@@ -1019,17 +1132,17 @@ int knn_graph(const float* points, int64_t N, int D, int k, float* out_dist, int
 
 size_t knn_distances_workspace(int64_t N, int64_t Q, int D) { return knn_search_workspace(N, Q, D, 1); }
 
-int knn_distances(const float* ref, const float* query, int64_t N, int64_t Q, int D, float* out, void* d_work,
-                  size_t work_bytes, void* stream) {
+int knn_distances(const float* ref, const float* query, int64_t N, int64_t Q, int D, float* out, float* out_eps,
+                  void* d_work, size_t work_bytes, void* stream) {
     int st = knn_check(ref, query, N, Q, D, 1, 0);
     if (st) return st;
     if (!out || !d_work) return KSEL_ERR_INVALID_ARG;
     DevInfo di;
     st = current_device_info(&di);
     if (st) return st;
-    const KnnGeom g = knn_geometry(N, Q, D, 1, di.sms, 0);
-    if (work_bytes < knn_work_layout(g).total) return KSEL_ERR_INVALID_ARG;
-    cudaError_t e = knn_run(ref, query, g, static_cast<uint8_t*>(d_work), nullptr, nullptr, out, (cudaStream_t)stream);
+    if (work_bytes < knn_workspace_bytes(N, Q, D, 1, di.sms)) return KSEL_ERR_INVALID_ARG;
+    cudaError_t e = knn_run(ref, query, N, Q, D, 1, 0, static_cast<uint8_t*>(d_work), nullptr, nullptr, out, out_eps,
+                            di.sms, (cudaStream_t)stream);
     return e == cudaSuccess ? KSEL_OK : KSEL_ERR_CUDA;
 }
 

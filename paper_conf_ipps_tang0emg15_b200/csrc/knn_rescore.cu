@@ -1,0 +1,327 @@
+// KSEL_SPLIT_R
+// knn_rescore.cu -- the exact end of knn_search (knn_fused.cu): rescoring of the
+// candidates the fp16 tensor-core filter left, and an exact brute-force fallback.
+//
+// Every candidate's distance is recomputed in the oracle's own arithmetic (reading
+// R9, the CPU definition in DESIGN.md section 2): d = (float) sum_{t < D} (q_t - r_t)^2
+// with each difference and square in double and the sum taken in index order, one
+// rounding to fp32 at the end (the differences and squares of fp32 inputs are exact
+// in double, so only the additions round -- in the same order as the oracle).  The
+// top-k by (d, index) of the exact pairs is then the oracle's result bit for bit
+// (PAPER.md L13 distance phase, L11/L19 selection, L637 sorted output).
+//
+// knn_rescore_kernel: one warp per query.  The filter kernel left, per reference
+// split, a pool of (d~, row) pairs holding every row with d~ <= T + 2 eps_q (T: any
+// k-th d~).  The warp gathers the pools' pairs into a shared-memory buffer, narrowing
+// it to the band above ITS k-th d~ (the k-th over all splits: tighter than any one
+// split's), rescores the band (one lane per candidate) and keeps the exact top-k; if
+// the band itself does not fit the buffer (k near 1024 with a wide band), candidates
+// are rescored as they are gathered against the running exact k-th instead.
+//
+// knn_fallback_kernel: queries flagged by the filter (a band of tied d~ larger than
+// the pool, or non-finite inputs) are solved by brute force: one CTA per query, every
+// reference rescored exactly, per-warp pools of exact pairs narrowed by radix select,
+// merged, sorted.  Slow (a full exact pass over N) but exact; it does nothing when no
+// query is flagged.
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "ksel_common.cuh"
+#include "ksel_internal.h"
+#include "ksel_pool.cuh"
+#include "knn_common.cuh"
+
+#ifndef KSEL_ONLY_R
+#error "compile once per queue size with -DKSEL_ONLY_R=1|2|4|8|16|32"
+#endif
+
+namespace ksel {
+
+constexpr int kRsWarps = 4;
+constexpr int kRsRegs = 36;              // exact-pair buffer of 1152 per warp (>= k' + 32 for k' <= 1024)
+constexpr int kRsCap = 32 * kRsRegs;
+
+// The oracle's distance of one reference row (r: D floats, global) to the query held in
+// double (qd, shared memory): differences and squares in double, summed in index order.
+__device__ __forceinline__ float exact_dist(const float* __restrict__ r, const double* __restrict__ qd, int D) {
+    double acc = 0.0;
+    if ((D & 3) == 0 && (reinterpret_cast<uintptr_t>(r) & 15u) == 0) {
+        // 8 independent 16-byte loads in flight before any use (the row is a gather from
+        // HBM / L2; a load-use chain per float4 would serialise on memory latency)
+        const float4* r4 = reinterpret_cast<const float4*>(r);
+        for (int t4 = 0; t4 < D / 4; t4 += 8) {
+            float4 v[8];
+#pragma unroll
+            for (int j = 0; j < 8; ++j) v[j] = (t4 + j < D / 4) ? __ldg(r4 + t4 + j) : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+                if (t4 + j < D / 4) {
+                    const int t = 4 * (t4 + j);
+                    double d = __dsub_rn(qd[t], (double)v[j].x);
+                    acc = __dadd_rn(acc, __dmul_rn(d, d));
+                    d = __dsub_rn(qd[t + 1], (double)v[j].y);
+                    acc = __dadd_rn(acc, __dmul_rn(d, d));
+                    d = __dsub_rn(qd[t + 2], (double)v[j].z);
+                    acc = __dadd_rn(acc, __dmul_rn(d, d));
+                    d = __dsub_rn(qd[t + 3], (double)v[j].w);
+                    acc = __dadd_rn(acc, __dmul_rn(d, d));
+                }
+            }
+        }
+    } else {
+        for (int t = 0; t < D; ++t) {
+            const double d = __dsub_rn(qd[t], (double)__ldg(r + t));
+            acc = __dadd_rn(acc, __dmul_rn(d, d));
+        }
+    }
+    return __double2float_rn(acc);
+}
+
+__device__ __forceinline__ float key_value(uint32_t key) { return __uint_as_float(bits_of_key(key)); }
+
+template <int R>
+__device__ __forceinline__ void emit_sorted(const unsigned long long* buf, int c, int k, int64_t idx_offset,
+                                            float* __restrict__ ov, int32_t* __restrict__ oi, uint32_t lane) {
+    WArr<R> a;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const int e = r * 32 + (int)lane;
+        const unsigned long long pr = (e < c) ? buf[e] : ~0ull;
+        a.k[r] = (e < c) ? (uint32_t)(pr >> 32) : kSentKey;
+        a.i[r] = (e < c) ? (uint32_t)pr : kSentIdx;
+    }
+    warr_sort<R>(a, lane);
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const int e = r * 32 + (int)lane;
+        if (e < k) {
+            // exact distances are >= +0 or NaN: the key inverts exactly except NaN payloads
+            ov[e] = __uint_as_float(a.k[r] == 0xffffffffu ? 0x7fc00000u : bits_of_key(a.k[r]));
+            oi[e] = (a.i[r] == kSentIdx) ? (int32_t)kSentIdx : (int32_t)((int64_t)a.i[r] + idx_offset);
+        }
+    }
+}
+
+template <int R>
+__global__ void __launch_bounds__(32 * kRsWarps) knn_rescore_kernel(const KnnRescoreArgs a) {
+    __shared__ unsigned long long buf_all[kRsWarps][kRsCap];
+    __shared__ double qd_all[kRsWarps][KNN_MAX_D];
+    const uint32_t lane = lane_id();
+    const int w = threadIdx.x >> 5;
+    const int64_t q = (int64_t)blockIdx.x * kRsWarps + w;
+    if (q >= a.Q || a.qfail[q]) return;
+    unsigned long long* buf = buf_all[w];
+    double* qd = qd_all[w];
+    for (int t = (int)lane; t < a.D; t += 32) qd[t] = (double)a.query[q * a.D + t];
+    __syncwarp();
+    const float eps = knn_eps(a.qstat[q], *a.stats, a.D);
+    const float band = __fmul_ru(2.f, eps);
+    unsigned long long Kb = band_bound(a.thr[q], band);  // candidates: pair <= Kb
+    const uint32_t lt = lanemask_lt();
+    // Phase A: gather the approximate pairs of all splits below the band, narrowing the
+    // buffer to (its k-th d~ + the band) when it fills -- afterwards it holds exactly the
+    // references that can be in the top-k.  Phase B (only if that band alone does not fit
+    // the buffer): rescore what is there, keep the exact top-k, and from then on rescore
+    // each gathered candidate at once, skipping those with d~ - eps_q above the exact k-th.
+    bool exact_mode = false;
+    unsigned long long Tx = ~0ull;            // exact bound (phase B)
+    float txv = __int_as_float(0x7f800000);   // its value
+    int c = 0;
+    auto rescore_buffer = [&]() {
+        for (int e = (int)lane; e < c; e += 32) {
+            const uint32_t row = (uint32_t)buf[e];
+            buf[e] = ((unsigned long long)key_of(exact_dist(a.ref + (int64_t)row * a.D, qd, a.D)) << 32) | row;
+        }
+        __syncwarp();
+    };
+#pragma unroll 1
+    for (int s = 0; s < a.S; ++s) {
+        const int ns = a.cnt[(int64_t)s * a.Q + q];
+        const unsigned long long* pr = a.pools + ((int64_t)s * a.Q + q) * a.P;
+#pragma unroll 1
+        for (int base = 0; base < ns; base += 32) {
+            const int x = base + (int)lane;
+            const unsigned long long v = (x < ns) ? __ldcg(pr + x) : ~0ull;
+            if (!exact_mode) {
+                bool keep = x < ns && v <= Kb;
+                uint32_t bal = __ballot_sync(kFull, keep);
+                if (c + __popc(bal) > kRsCap) {
+                    int nn;
+                    const unsigned long long Ta = pool_narrow64<kRsRegs, false>(buf, c, (uint32_t)a.k, &nn, band);
+                    c = nn;
+                    const unsigned long long Kn = band_bound(Ta, band);
+                    Kb = Kn < Kb ? Kn : Kb;
+                    keep = keep && v <= Kb;
+                    bal = __ballot_sync(kFull, keep);
+                    if (c + __popc(bal) > kRsCap) {  // the band alone overflows: phase B
+                        rescore_buffer();
+                        Tx = pool_narrow64<kRsRegs, false>(buf, c, (uint32_t)a.k, &nn);
+                        c = nn;
+                        txv = key_value((uint32_t)(Tx >> 32));
+                        exact_mode = true;
+                    }
+                }
+                if (!exact_mode) {
+                    if (keep) buf[c + __popc(bal & lt)] = v;
+                    c += __popc(bal);
+                    __syncwarp();
+                    continue;
+                }
+            }
+            // phase B: a candidate whose d~ - eps_q exceeds the exact k-th so far cannot win
+            const bool cand = x < ns && v <= Kb && __fsub_rd(key_value((uint32_t)(v >> 32)), eps) <= txv;
+            unsigned long long ex = ~0ull;
+            if (cand) {
+                const uint32_t row = (uint32_t)v;
+                ex = ((unsigned long long)key_of(exact_dist(a.ref + (int64_t)row * a.D, qd, a.D)) << 32) | row;
+            }
+            bool keep = cand && ex <= Tx;
+            uint32_t bal = __ballot_sync(kFull, keep);
+            if (c + __popc(bal) > kRsCap) {  // full: narrow to the exact k-th pair
+                int nn;
+                Tx = pool_narrow64<kRsRegs, false>(buf, c, (uint32_t)a.k, &nn);
+                c = nn;
+                txv = key_value((uint32_t)(Tx >> 32));
+                keep = keep && ex <= Tx;
+                bal = __ballot_sync(kFull, keep);
+            }
+            if (keep) buf[c + __popc(bal & lt)] = ex;
+            c += __popc(bal);
+            __syncwarp();
+        }
+    }
+    if (!exact_mode) {  // phase A ended: the band set, rescored exactly
+        if (c > a.k) {
+            int nn;
+            pool_narrow64<kRsRegs, false>(buf, c, (uint32_t)a.k, &nn, band);
+            c = nn;
+        }
+        rescore_buffer();
+    }
+    if (c > a.k) {
+        int nn;
+        pool_narrow64<kRsRegs, false>(buf, c, (uint32_t)a.k, &nn);
+        c = nn;
+    }
+    emit_sorted<R>(buf, c, a.k, a.idx_offset, a.out_val + q * a.k, a.out_idx + q * a.k, lane);
+}
+
+template <int R>
+__global__ void __launch_bounds__(32 * kFbWarps) knn_fallback_kernel(const KnnRescoreArgs a) {
+    __shared__ double qd[KNN_MAX_D];
+    __shared__ uint32_t hist_all[kFbWarps][256];
+    __shared__ int cnt_s[kFbWarps];
+    constexpr int kp = 32 * R;
+    constexpr int PW = kp + 256;  // per-warp pool
+    const uint32_t lane = lane_id();
+    const int w = threadIdx.x >> 5;
+    const uint32_t lt = lanemask_lt();
+    unsigned long long* cta = reinterpret_cast<unsigned long long*>(a.fb) +
+                              (size_t)blockIdx.x * kFbWarps * (size_t)(2 * kp + 256);
+    unsigned long long* wpool = cta + (size_t)w * PW;
+    unsigned long long* merge = cta + (size_t)kFbWarps * PW;  // kFbWarps * kp pairs
+    __shared__ int flagged[32 * kFbWarps];
+    __shared__ int nflag;
+    // scan the failure flags 256 at a time (one load per thread); solve the flagged queries
+    for (int64_t q0 = (int64_t)blockIdx.x * 256; q0 < a.Q; q0 += (int64_t)gridDim.x * 256) {
+        if (threadIdx.x == 0) nflag = 0;
+        __syncthreads();
+        const int64_t qq = q0 + threadIdx.x;
+        if (qq < a.Q && a.qfail[qq]) flagged[atomicAdd(&nflag, 1)] = (int)threadIdx.x;
+        __syncthreads();
+        const int nf = nflag;
+    for (int f = 0; f < nf; ++f) {
+        const int64_t q = q0 + flagged[f];
+        __syncthreads();
+        for (int t = threadIdx.x; t < a.D; t += blockDim.x) qd[t] = (double)a.query[q * a.D + t];
+        __syncthreads();
+        unsigned long long Tw = ~0ull;
+        int c = 0;
+#pragma unroll 1
+        for (int64_t i0 = (int64_t)w * 32; i0 < a.N; i0 += 32 * kFbWarps) {
+            const int64_t i = i0 + lane;
+            unsigned long long ex = ~0ull;
+            if (i < a.N) ex = ((unsigned long long)key_of(exact_dist(a.ref + i * a.D, qd, a.D)) << 32) | (uint32_t)i;
+            bool keep = i < a.N && ex <= Tw;
+            uint32_t bal = __ballot_sync(kFull, keep);
+            if (c + __popc(bal) > PW) {
+                int nn;
+                Tw = pool_select64(wpool, c, (uint32_t)a.k, hist_all[w], &nn);
+                c = nn;
+                keep = keep && ex <= Tw;
+                bal = __ballot_sync(kFull, keep);
+            }
+            if (keep) wpool[c + __popc(bal & lt)] = ex;
+            c += __popc(bal);
+            __syncwarp();
+        }
+        if (c > a.k) {
+            int nn;
+            pool_select64(wpool, c, (uint32_t)a.k, hist_all[w], &nn);
+            c = nn;
+        }
+        if (lane == 0) cnt_s[w] = c;
+        __syncthreads();
+        if (w == 0) {
+            int m = 0;
+            for (int v = 0; v < kFbWarps; ++v) {
+                const int cv = cnt_s[v];
+                const unsigned long long* src = cta + (size_t)v * PW;
+                for (int e = (int)lane; e < cv; e += 32) merge[m + e] = __ldcg(src + e);
+                m += cv;
+            }
+            __syncwarp();
+            if (m > a.k) {
+                int nn;
+                pool_select64(merge, m, (uint32_t)a.k, hist_all[0], &nn);
+                m = nn;
+            }
+            __syncwarp();
+            // (merge is global memory: read it back through L2)
+            WArr<R> s;
+#pragma unroll
+            for (int r = 0; r < R; ++r) {
+                const int e = r * 32 + (int)lane;
+                const unsigned long long pr = (e < m) ? __ldcg(merge + e) : ~0ull;
+                s.k[r] = (e < m) ? (uint32_t)(pr >> 32) : kSentKey;
+                s.i[r] = (e < m) ? (uint32_t)pr : kSentIdx;
+            }
+            warr_sort<R>(s, lane);
+            float* ov = a.out_val + q * a.k;
+            int32_t* oi = a.out_idx + q * a.k;
+#pragma unroll
+            for (int r = 0; r < R; ++r) {
+                const int e = r * 32 + (int)lane;
+                if (e < a.k) {
+                    ov[e] = __uint_as_float(s.k[r] == 0xffffffffu ? 0x7fc00000u : bits_of_key(s.k[r]));
+                    oi[e] = (int32_t)((int64_t)s.i[r] + a.idx_offset);
+                }
+            }
+        }
+        __syncthreads();
+    }
+    __syncthreads();
+    }
+}
+
+template <int R>
+cudaError_t launch_knn_rescore_r(const KnnRescoreArgs& a, cudaStream_t stream) {
+    const int64_t grid = (a.Q + kRsWarps - 1) / kRsWarps;
+    knn_rescore_kernel<R><<<(unsigned)grid, 32 * kRsWarps, 0, stream>>>(a);
+    note_launch();
+    return cudaGetLastError();
+}
+
+template <int R>
+cudaError_t launch_knn_fallback_r(const KnnRescoreArgs& a, cudaStream_t stream) {
+    const int64_t blocks = (a.Q + 255) / 256;
+    const int grid = (int)(blocks < kFbCtas ? blocks : kFbCtas);
+    knn_fallback_kernel<R><<<grid, 32 * kFbWarps, 0, stream>>>(a);
+    note_launch();
+    return cudaGetLastError();
+}
+
+template cudaError_t launch_knn_rescore_r<KSEL_ONLY_R>(const KnnRescoreArgs&, cudaStream_t);
+template cudaError_t launch_knn_fallback_r<KSEL_ONLY_R>(const KnnRescoreArgs&, cudaStream_t);
+
+}  // namespace ksel

@@ -84,10 +84,6 @@ uint64_t flag_timeout_ns();
 cudaError_t launch_merge(const MergeLists& L, int64_t Q, int S, int kin, int k, float* out_val, int32_t* out_idx,
                          cudaStream_t stream);
 
-// Top-k per query of the S split pools of the fused k-NN (merge.cu).
-cudaError_t launch_merge_pools(const unsigned long long* pools, int64_t P, const int32_t* cnt, int S, int64_t Q,
-                               const unsigned long long* thr, int k, int64_t idx_offset, float* out_val,
-                               int32_t* out_idx, cudaStream_t stream);
 
 // Per-queue-size entry points (explicitly instantiated, one object per R).
 template <int R>
@@ -99,9 +95,5 @@ cudaError_t launch_pool_r(const float* dist, int64_t Q, int64_t N, int k, float*
 template <int R>
 cudaError_t launch_merge_r(const MergeLists& L, int64_t Q, int S, int kin, int k, float* ov, int32_t* oi,
                            cudaStream_t stream);
-template <int R>
-cudaError_t launch_merge_pools_r(const unsigned long long* pools, int64_t P, const int32_t* cnt, int S, int64_t Q,
-                                 const unsigned long long* thr, int k, int64_t idx_offset, float* ov, int32_t* oi,
-                                 cudaStream_t stream);
 
 }  // namespace ksel

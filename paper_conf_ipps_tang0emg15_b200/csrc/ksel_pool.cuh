@@ -288,9 +288,23 @@ __device__ __noinline__ unsigned long long pool_narrow_regs(uint32_t* __restrict
 // u64 array; the key bisection starts below the common prefix of the pool's
 // smallest and largest key.  GLOBAL: the pool is in global memory (L2 loads,
 // __ldcg: other lanes wrote it); otherwise generic loads (shared memory).
+// Compaction bound of a narrowing to the want-th pair T: T itself, or -- for pools of
+// approximate keys (the fused k-NN's filter distances) -- every pair whose value is
+// <= value(T) + band (band >= 0, rounded up; no finite bound keeps everything).
+__device__ __forceinline__ unsigned long long band_bound(unsigned long long T, float band) {
+    if (band < 0.f) return T;
+    const uint32_t tk = (uint32_t)(T >> 32);
+    if (tk >= 0xff800000u) return ~0ull;
+    const float v = __fadd_ru(__uint_as_float(bits_of_key(tk)), band);
+    if (!(v < __int_as_float(0x7f800000))) return ~0ull;
+    const unsigned long long K = ((unsigned long long)key_of(v) << 32) | 0xffffffffull;
+    return K > T ? K : T;
+}
+
+// band >= 0: keep the band above the want-th pair (band_bound); the want-th pair is returned.
 template <int NR, bool GLOBAL = true>
 __device__ __noinline__ unsigned long long pool_narrow64(unsigned long long* __restrict__ pool, int n, uint32_t want,
-                                                         int* n_out) {
+                                                         int* n_out, float band = -1.f) {
     const uint32_t lane = lane_id();
     unsigned long long r[NR];
     uint32_t kmin = 0xffffffffu, kmax = 0u;
@@ -346,12 +360,13 @@ __device__ __noinline__ unsigned long long pool_narrow64(unsigned long long* __r
         }
     }
     const unsigned long long T = ((unsigned long long)vkey << 32) | vidx;
+    const unsigned long long K = band_bound(T, band);
     __syncwarp();  // all loads of the pool precede the in-place compaction
     const uint32_t lt = lanemask_lt();
     int w = 0;
 #pragma unroll
     for (int u = 0; u < NR; ++u) {
-        const bool keep = (u * 32 + (int)lane < n) && r[u] <= T;
+        const bool keep = (u * 32 + (int)lane < n) && r[u] <= K;
         const uint32_t bal = __ballot_sync(kFull, keep);
         if (keep) pool[w + __popc(bal & lt)] = r[u];
         w += __popc(bal);
@@ -388,7 +403,7 @@ __device__ __forceinline__ void pool_scan64(const unsigned long long* __restrict
 // transposed layout).  The pool is then compacted in place to the pairs <= it.
 __device__ __noinline__ static unsigned long long pool_select64(unsigned long long* __restrict__ pool, int n,
                                                                uint32_t want, uint32_t* __restrict__ hist,
-                                                               int* n_out) {
+                                                               int* n_out, float band = -1.f) {
     const uint32_t lane = lane_id();
     uint32_t kmin = 0xffffffffu, kmax = 0u;
     pool_scan64(pool, n, lane, [&](unsigned long long v) {
@@ -449,6 +464,7 @@ __device__ __noinline__ static unsigned long long pool_select64(unsigned long lo
         vidx = ip;
     }
     const unsigned long long T = ((unsigned long long)vkey << 32) | vidx;
+    const unsigned long long K = band_bound(T, band);
     // in-place compaction, 8 slabs of 32 per batch: every read of a batch precedes its
     // writes, and writes never pass the batch's first slab (w <= base)
     const uint32_t lt = lanemask_lt();
@@ -464,7 +480,7 @@ __device__ __noinline__ static unsigned long long pool_select64(unsigned long lo
         __syncwarp();
 #pragma unroll
         for (int j = 0; j < 8; ++j) {
-            const bool keep = base + j * 32 + (int)lane < n && v[j] <= T;
+            const bool keep = base + j * 32 + (int)lane < n && v[j] <= K;
             const uint32_t bal = __ballot_sync(kFull, keep);
             if (keep) pool[w + __popc(bal & lt)] = v[j];
             w += __popc(bal);

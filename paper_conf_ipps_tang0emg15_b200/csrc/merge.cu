@@ -194,100 +194,6 @@ cudaError_t launch_merge_r(const MergeLists& L, int64_t Q, int S, int kin, int k
     return cudaErrorInvalidValue;
 }
 
-// Final step of the fused k-NN (knn_fused.cu): each of the S reference splits
-// left, per query, a pool of cnt[s][q] packed pairs (key << 32 | local index)
-// that contains every pair of its split in the row's top-k; thr[q] is the
-// tightest bound on the row's k-th pair any split published.  One warp per
-// query gathers the pairs <= thr[q] from the S pools into shared memory
-// (coalesced, ballot compaction; if the buffer would overflow it is narrowed to
-// its exact top-k first, by register bisection), narrows to exactly k, sorts the
-// k pairs in registers and emits them with the index offset added.  Pairs are
-// distinct, so the result is the exact top-k of the row.
-constexpr int kPoolRegs = 40;
-constexpr int kGatherCap = 32 * kPoolRegs;
-
-template <int R>
-__global__ void __launch_bounds__(32 * kMergeWarps)
-    ksel_merge_pools_kernel(const unsigned long long* __restrict__ pools, int64_t P, const int32_t* __restrict__ cnt,
-                            int S, int64_t Q, const unsigned long long* __restrict__ thr, int k, int64_t idx_offset,
-                            float* __restrict__ out_val, int32_t* __restrict__ out_idx) {
-    __shared__ unsigned long long buf_all[kMergeWarps][kGatherCap];
-    const uint32_t lane = lane_id();
-    const int w = threadIdx.x >> 5;
-    const int64_t q = (int64_t)blockIdx.x * kMergeWarps + w;
-    if (q >= Q) return;
-    unsigned long long* buf = buf_all[w];
-    unsigned long long T = thr[q];
-    const uint32_t lt = lanemask_lt();
-    int c = 0;
-#pragma unroll 1
-    for (int s = 0; s < S; ++s) {
-        const int ns = cnt[(int64_t)s * Q + q];
-        const unsigned long long* pr = pools + ((int64_t)s * Q + q) * P;
-#pragma unroll 1
-        for (int base = 0; base < ns; base += 64) {  // two loads in flight per lane
-            const int x0 = base + (int)lane, x1 = x0 + 32;
-            const unsigned long long v0 = (x0 < ns) ? __ldcg(pr + x0) : ~0ull;
-            const unsigned long long v1 = (x1 < ns) ? __ldcg(pr + x1) : ~0ull;
-#pragma unroll
-            for (int h = 0; h < 2; ++h) {
-                const unsigned long long v = h ? v1 : v0;
-                bool keep = ((h ? x1 : x0) < ns) && v <= T;
-                uint32_t bal = __ballot_sync(kFull, keep);
-                if (c + __popc(bal) > kGatherCap) {  // rare: tighten to the buffer's k-th pair
-                    int nn;
-                    T = pool_narrow64<kPoolRegs, false>(buf, c, (uint32_t)k, &nn);
-                    c = nn;
-                    keep = keep && v <= T;
-                    bal = __ballot_sync(kFull, keep);
-                }
-                if (keep) buf[c + __popc(bal & lt)] = v;
-                c += __popc(bal);
-            }
-        }
-    }
-    __syncwarp();
-    if (c > k) {
-        int nn;
-        pool_narrow64<kPoolRegs, false>(buf, c, (uint32_t)k, &nn);
-        c = nn;
-    }
-    WArr<R> a;
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-        const int e = r * 32 + (int)lane;
-        const unsigned long long pr = (e < c) ? buf[e] : ~0ull;
-        a.k[r] = (e < c) ? (uint32_t)(pr >> 32) : kSentKey;
-        a.i[r] = (e < c) ? (uint32_t)pr : kSentIdx;
-    }
-    warr_sort<R>(a, lane);
-    float* ov = out_val + q * (int64_t)k;
-    int32_t* oi = out_idx + q * (int64_t)k;
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-        const int e = r * 32 + (int)lane;
-        if (e < k) {
-            ov[e] = __uint_as_float(bits_of_key(a.k[r]));
-            oi[e] = (a.i[r] == kSentIdx) ? (int32_t)kSentIdx : (int32_t)((int64_t)a.i[r] + idx_offset);
-        }
-    }
-}
-
-template <int R>
-cudaError_t launch_merge_pools_r(const unsigned long long* pools, int64_t P, const int32_t* cnt, int S, int64_t Q,
-                                 const unsigned long long* thr, int k, int64_t idx_offset, float* ov, int32_t* oi,
-                                 cudaStream_t stream) {
-    const int64_t grid = (Q + kMergeWarps - 1) / kMergeWarps;
-    ksel_merge_pools_kernel<R><<<(unsigned)grid, 32 * kMergeWarps, 0, stream>>>(pools, P, cnt, S, Q, thr, k,
-                                                                                idx_offset, ov, oi);
-    note_launch();
-    return cudaGetLastError();
-}
-
-template cudaError_t launch_merge_pools_r<KSEL_ONLY_R>(const unsigned long long*, int64_t, const int32_t*, int,
-                                                       int64_t, const unsigned long long*, int, int64_t, float*,
-                                                       int32_t*, cudaStream_t);
-
 template cudaError_t launch_merge_r<KSEL_ONLY_R>(const MergeLists&, int64_t, int, int, int, float*, int32_t*,
                                                  cudaStream_t);
 
