@@ -102,10 +102,64 @@ __device__ __forceinline__ void emit_sorted(const unsigned long long* buf, int c
     }
 }
 
+// The want-th smallest KEY (d~) over the union of a query's S pools (global memory):
+// MSD radix select on the 32-bit key below the union's common prefix, one warp, the
+// per-warp histogram in shared memory (hist_find: ksel_pool.cuh).  Returns the key v
+// with #{key < v} < want <= #{key <= v}.
+static __device__ __noinline__ uint32_t lists_kth_key(const unsigned long long* __restrict__ pools, const int32_t* __restrict__ cnt,
+                                              int S, int64_t Q, int64_t q, int64_t P, uint32_t want,
+                                              uint32_t* __restrict__ hist) {
+    const uint32_t lane = lane_id();
+    auto scan = [&](auto f) {
+        for (int s = 0; s < S; ++s) {
+            const int ns = cnt[(int64_t)s * Q + q];
+            const unsigned long long* pr = pools + ((int64_t)s * Q + q) * P;
+            for (int base = 0; base < ns; base += 128) {
+                unsigned long long v[4];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const int x = base + j * 32 + (int)lane;
+                    v[j] = (x < ns) ? __ldcg(pr + x) : ~0ull;
+                }
+#pragma unroll
+                for (int j = 0; j < 4; ++j)
+                    if (base + j * 32 + (int)lane < ns) f((uint32_t)(v[j] >> 32));
+            }
+        }
+    };
+    uint32_t kmin = 0xffffffffu, kmax = 0u;
+    scan([&](uint32_t kk) {
+        kmin = min(kmin, kk);
+        kmax = max(kmax, kk);
+    });
+    kmin = __reduce_min_sync(kFull, kmin);
+    kmax = __reduce_max_sync(kFull, kmax);
+    int hi = (kmin == kmax) ? -1 : 31 - __clz(kmin ^ kmax);
+    uint32_t prefix = (hi < 0) ? kmin : (kmin & ~((2u << hi) - 1u));
+    uint32_t cnt_b;
+    while (hi >= 0) {
+        const int lo = hi >= 7 ? hi - 7 : 0;
+        const uint32_t dmask = (2u << (hi - lo)) - 1u;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) hist[j * 32 + lane] = 0u;
+        __syncwarp();
+        scan([&](uint32_t kk) {
+            if (hi == 31 || ((kk ^ prefix) >> (hi + 1)) == 0u) atomicAdd(&hist[hist_slot((kk >> lo) & dmask)], 1u);
+        });
+        __syncwarp();
+        const uint32_t d = hist_find(hist, lane, want, cnt_b);
+        prefix |= d << lo;
+        __syncwarp();
+        hi = lo - 1;
+    }
+    return prefix;
+}
+
 template <int R>
 __global__ void __launch_bounds__(32 * kRsWarps) knn_rescore_kernel(const KnnRescoreArgs a) {
     __shared__ unsigned long long buf_all[kRsWarps][kRsCap];
     __shared__ double qd_all[kRsWarps][KNN_MAX_D];
+    __shared__ uint32_t hist_all[kRsWarps][256];
     const uint32_t lane = lane_id();
     const int w = threadIdx.x >> 5;
     const int64_t q = (int64_t)blockIdx.x * kRsWarps + w;
@@ -116,7 +170,20 @@ __global__ void __launch_bounds__(32 * kRsWarps) knn_rescore_kernel(const KnnRes
     __syncwarp();
     const float eps = knn_eps(a.qstat[q], *a.stats, a.D);
     const float band = __fmul_ru(2.f, eps);
-    unsigned long long Kb = band_bound(a.thr[q], band);  // candidates: pair <= Kb
+    // the k-th d~ over ALL of the query's pools (at least k references have a d~ <= it):
+    // only the band above it can hold the exact top-k
+    unsigned long long T0 = a.thr[q];
+    {
+        int tot = 0;
+        for (int s = (int)lane; s < a.S; s += 32) tot += a.cnt[(int64_t)s * a.Q + q];
+        tot = __reduce_add_sync(kFull, tot);
+        if (tot > kRsCap && tot >= a.k) {  // (a union that fits the buffer is band-narrowed there)
+            const uint32_t kk = lists_kth_key(a.pools, a.cnt, a.S, a.Q, q, a.P, (uint32_t)a.k, hist_all[w]);
+            const unsigned long long t = ((unsigned long long)kk << 32) | 0xffffffffull;
+            T0 = t < T0 ? t : T0;
+        }
+    }
+    unsigned long long Kb = band_bound(T0, band);  // candidates: pair <= Kb
     const uint32_t lt = lanemask_lt();
     // Phase A: gather the approximate pairs of all splits below the band, narrowing the
     // buffer to (its k-th d~ + the band) when it fills -- afterwards it holds exactly the
