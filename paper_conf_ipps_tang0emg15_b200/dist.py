@@ -7,19 +7,20 @@ Two modes:
   owns rows [r*Q/g, (r+1)*Q/g) -- no collective at all (:func:`query_rows`).
 * ``knn_search`` shards the reference set by rows: rank r holds references
   [r*N/g, (r+1)*N/g), computes the per-query top-k of its shard with global
-  indices (idx_offset), the candidates are exchanged with one NCCL
-  all-gather over NVLink and ``ksel_merge`` (divide-and-merge)
-  produces the exact global top-k.  Each rank merges only its own slice of
-  queries, so the merge work also scales with g (:func:`knn_search_sharded`).
+  indices (idx_offset), the candidates are exchanged with NCCL all-gathers over
+  NVLink -- one per query chunk, overlapping the next chunk's search -- and the
+  merge (divide-and-merge) reads the gathered lists in place and
+  produces the exact global top-k.  Each rank merges only its own slice of every
+  chunk, so the merge work also scales with g (:func:`knn_search_sharded`).
 
 Exactness: each shard's lexicographic (value, index) order is the global one
 (indices are offset monotonically), every global top-k element is in its
 shard's top-k, so the merge of the shard lists is the global top-k --
 bit-identical to the unsharded result.
 
-The local kernels and the collective are parameters so that the host-side
-logic (partitioning, offsets, packing, slicing) can be exercised with gloo on
-CPU in tests; the defaults are the CUDA library and NCCL.
+The local kernels are parameters so that the host-side logic (partitioning,
+offsets, chunking, the in-place buffers, slicing) can be exercised with gloo on
+CPU in tests; the defaults are the CUDA library (and NCCL under torchrun).
 """
 from __future__ import annotations
 
@@ -37,33 +38,48 @@ def query_rows(Q: int, world: int, rank: int) -> tuple[int, int]:
     return shard_range(Q, world, rank)
 
 
-def _default_knn(ref, query, k, idx_offset):
+def _default_knn(ref, query, k, idx_offset, out_val, out_idx):
     from . import knn_search
-    return knn_search(ref, query, k, idx_offset=idx_offset)
+    knn_search(ref, query, k, idx_offset=idx_offset, out_dist=out_val, out_idx=out_idx)
 
 
-def _default_merge(cand_val, cand_idx, k):
-    from . import ksel_merge
-    return ksel_merge(cand_val, cand_idx, k)
+def _default_merge(vals, idxs, k, out_val, out_idx):
+    """Top-k of the union of the lists vals[s] / idxs[s] ([nq, kin] views, possibly inside
+    one gathered buffer): ksel_merge_lists reads them in place through a pointer table."""
+    from . import ksel_merge_lists
+    nq, kin = vals[0].shape
+    ksel_merge_lists([v.data_ptr() for v in vals], [i.data_ptr() for i in idxs], nq, kin, k, out_val, out_idx)
 
 
-def _all_gather(out: torch.Tensor, inp: torch.Tensor, group=None):
+def _all_gather(out: torch.Tensor, inp: torch.Tensor, group=None, async_op=False):
     """all_gather_into_tensor, with a list fallback for backends without it."""
     try:
-        tdist.all_gather_into_tensor(out, inp, group=group)
+        return tdist.all_gather_into_tensor(out, inp, group=group, async_op=async_op)
     except (RuntimeError, AttributeError, NotImplementedError):
         world = tdist.get_world_size(group)
         parts = list(out.chunk(world, dim=0))
-        tdist.all_gather(parts, inp, group=group)
+        return tdist.all_gather(parts, inp, group=group, async_op=async_op)
+
+
+def chunk_ranges(Q: int, chunks: int) -> list:
+    """Contiguous query chunks [a, b) of the exchange pipeline."""
+    c = max(1, min(int(chunks), Q))
+    return [shard_range(Q, c, i) for i in range(c)]
 
 
 def knn_search_sharded(ref_shard: torch.Tensor, query: torch.Tensor, k: int, n_total: int, group=None,
-                       local_knn=None, merge=None):
-    """Row-sharded k-NN: local top-k with global indices, all-gather, merge.
+                       chunks: int = 4, local_knn=None, merge=None):
+    """Row-sharded k-NN: local top-k with global indices, all-gather, merge -- pipelined
+    over query chunks.
 
     ``ref_shard`` holds this rank's references (rows shard_range(n_total, g, r)),
-    ``query`` all Q queries (replicated).  Returns (values, indices, (q0, q1)):
-    the exact global top-k of queries [q0, q1) -- this rank's slice.
+    ``query`` all Q queries (replicated).  Queries go in ``chunks`` contiguous chunks; for
+    chunk c the local search writes its (value bits, index) lists straight into one
+    [2][qc][k] send buffer, ONE all-gather (async, NCCL over NVLink) moves them into a
+    [g][2][qc][k] receive buffer while the search of chunk c + 1 runs, and this rank then
+    merges its slice of chunk c's queries reading the g lists in place (pointer tables:
+    no stacking, no copies).  Returns (values, indices, qids): the exact global top-k of
+    the queries qids (this rank's slice of every chunk, ascending).
     """
     world = tdist.get_world_size(group)
     rank = tdist.get_rank(group)
@@ -72,39 +88,61 @@ def knn_search_sharded(ref_shard: torch.Tensor, query: torch.Tensor, k: int, n_t
     r0, r1 = shard_range(n_total, world, rank)
     assert ref_shard.shape[0] == r1 - r0, "ref_shard must hold rows [%d, %d)" % (r0, r1)
     Q = query.shape[0]
-    v, i = local_knn(ref_shard, query, k, r0)
-    # one collective: (value bits, index) packed as int32 pairs
-    packed = torch.stack([v.contiguous().view(torch.int32), i.contiguous()], dim=-1)  # [Q, k, 2]
-    flat = torch.empty((world * Q,) + tuple(packed.shape[1:]), dtype=packed.dtype, device=packed.device)
-    _all_gather(flat, packed, group)
-    gathered = flat.view((world,) + tuple(packed.shape))
-    q0, q1 = shard_range(Q, world, rank)
-    cand = gathered[:, q0:q1]
-    cand_val = cand[..., 0].contiguous().view(torch.float32)  # [world, q1-q0, k]
-    cand_idx = cand[..., 1].contiguous()
-    mv, mi = merge(cand_val, cand_idx, k)
-    return mv, mi, (q0, q1)
+    dev = query.device
+    spans = chunk_ranges(Q, chunks)
+    slices = [(qa + shard_range(qb - qa, world, rank)[0], qa + shard_range(qb - qa, world, rank)[1])
+              for qa, qb in spans]
+    qids = torch.cat([torch.arange(a, b, dtype=torch.int64) for a, b in slices])
+    out_v = torch.empty((qids.numel(), k), dtype=torch.float32, device=dev)
+    out_i = torch.empty((qids.numel(), k), dtype=torch.int32, device=dev)
+    pending = []  # (work, recv, slice in the chunk, output row offset)
+
+    def finish(item):
+        work, recv, (s0, s1), off = item
+        if work is not None:
+            work.wait()
+        if s1 > s0:
+            vals = [recv[s, 0, s0:s1].view(torch.float32) for s in range(world)]
+            idxs = [recv[s, 1, s0:s1] for s in range(world)]
+            merge(vals, idxs, k, out_v[off:off + s1 - s0], out_i[off:off + s1 - s0])
+
+    off = 0
+    for (qa, qb), (sa, sb) in zip(spans, slices):
+        qc = qb - qa
+        send = torch.empty((2, qc, k), dtype=torch.int32, device=dev)
+        local_knn(ref_shard, query[qa:qb], k, r0, send[0].view(torch.float32), send[1])
+        recv = torch.empty((world, 2, qc, k), dtype=torch.int32, device=dev)
+        work = _all_gather(recv.view(-1), send.view(-1), group, async_op=True)
+        # the previous chunk's exchange overlapped this chunk's search: merge it now
+        if pending:
+            finish(pending.pop())
+        pending.append((work, recv, (sa - qa, sb - qa), off))
+        off += sb - sa
+    while pending:
+        finish(pending.pop())
+    return out_v, out_i, qids
 
 
 # ---------------------------------------------------------------------------
 # Collective-free exchange: the merge reads peers' lists
 # ---------------------------------------------------------------------------
 
-_P2P_HDR = 512  # bytes: ready[2] u32 at 0, consumed[world <= 64] u32 at 64
+_P2P_HDR = 512  # bytes: ready[2][8] u32 at 0, consumed[world <= 64] u32 at 64
+P2P_MAX_CHUNKS = 8
 
 
 def p2p_layout(Q: int, k: int, world: int) -> dict:
     """Byte offsets inside each rank's exchange buffer.
 
-    ``ready(b)``: u32 epoch flag of double buffer b (written by the owner);
-    ``consumed(s)``: u32 epoch flag written by rank s once it merged the owner's
-    lists; ``val(b)`` / ``idx(b)``: the owner's [Q][k] fp32 / int32 top-k lists.
+    ``ready(b, c)``: u32 epoch flag of query chunk c of double buffer b (written by
+    the owner); ``consumed(s)``: u32 epoch flag written by rank s once it merged the
+    owner's lists; ``val(b)`` / ``idx(b)``: the owner's [Q][k] fp32 / int32 top-k lists.
     """
     if not 1 <= world <= 64:
         raise ValueError("world size must be in [1, 64]")
     lst = Q * k * 4
     return {
-        "ready": lambda b: 4 * b,
+        "ready": lambda b, c=0: 4 * (b * P2P_MAX_CHUNKS + c),
         "consumed": lambda s: 64 + 4 * s,
         "val": lambda b: _P2P_HDR + b * 2 * lst,
         "idx": lambda b: _P2P_HDR + b * 2 * lst + lst,
@@ -119,19 +157,22 @@ class KnnP2P:
     [Q][k] candidate lists plus flags; handles are exchanged once over the
     process group and mapped with CUDA IPC (NVLink / NVSwitch peer memory; on a
     single GPU, several processes share it the same way).  Per call (epoch e,
-    buffer b = e % 2), all stream-ordered on the current stream, no host sync:
+    buffer b = e % 2), all stream-ordered on the current stream, no host sync,
+    pipelined over ``chunks`` query chunks:
 
     1. (e >= 2) wait until every rank consumed epoch e - 2 of this buffer;
-    2. ``knn_search`` of the local shard (global indices) into buffer b;
-    3. signal ready[b] = e + 1;
-    4. ``ksel_merge_lists`` over the g lists of this rank's query slice,
-       straight from the peers' buffers, each list waited for (ready >= e + 1);
-    5. signal consumed[rank] = e + 1 in every peer's buffer.
+    2. for each chunk c: ``knn_search`` of the local shard (global indices) for
+       chunk c's queries straight into buffer b, then signal ready[b][c] = e + 1;
+       after chunk c's search, ``ksel_merge_lists`` of chunk c - 1 -- this rank's
+       slice of it, read in place from the peers' buffers, each list waited for
+       (ready >= e + 1) -- so the peers' chunk c - 1 is normally complete while
+       the next search is queued behind the merge;
+    3. signal consumed[rank] = e + 1 in every peer's buffer.
 
     Same result as :func:`knn_search_sharded` (bit-identical to unsharded).
     """
 
-    def __init__(self, Q: int, k: int, n_total: int, group=None, local_knn=None):
+    def __init__(self, Q: int, k: int, n_total: int, group=None, local_knn=None, chunks: int = 4):
         from . import ipc_alloc, ipc_open
         self.group = group
         self.world = tdist.get_world_size(group)
@@ -145,6 +186,7 @@ class KnnP2P:
         tdist.all_gather_object(handles, handle, group=group)
         self.peer = [self.base if s == self.rank else ipc_open(handles[s]) for s in range(self.world)]
         tdist.barrier(group=group)
+        self.chunks = max(1, min(int(chunks), P2P_MAX_CHUNKS, Q))
         self.epoch = 0
         self.warm = False
 
@@ -178,25 +220,40 @@ class KnnP2P:
         own = device_bytes(self.base, L["bytes"])
         ov = own[L["val"](b): L["val"](b) + Q * k * 4].view(torch.float32).view(Q, k)
         oi = own[L["idx"](b): L["idx"](b) + Q * k * 4].view(torch.int32).view(Q, k)
-        if self.local_knn is None:  # the library writes straight into the exchange buffer
-            from . import knn_search
-            knn_search(ref_shard, query, k, idx_offset=r0, out_dist=ov, out_idx=oi)
-        else:
-            v, i = self.local_knn(ref_shard, query, k, r0)
-            ov.copy_(v)
-            oi.copy_(i)
-        flag_signal(self.base + L["ready"](b), e + 1)
-        q0, q1 = shard_range(Q, self.world, self.rank)
-        mv = torch.empty((q1 - q0, k), dtype=torch.float32, device=query.device)
-        mi = torch.empty((q1 - q0, k), dtype=torch.int32, device=query.device)
-        if q1 > q0:
-            ksel_merge_lists([p + L["val"](b) + q0 * k * 4 for p in self.peer],
-                             [p + L["idx"](b) + q0 * k * 4 for p in self.peer], q1 - q0, k, k, mv, mi,
-                             ready_ptrs=[p + L["ready"](b) for p in self.peer], epoch=e + 1)
+        spans = chunk_ranges(Q, self.chunks)
+        slices = [(qa + shard_range(qb - qa, self.world, self.rank)[0],
+                   qa + shard_range(qb - qa, self.world, self.rank)[1]) for qa, qb in spans]
+        qids = torch.cat([torch.arange(a_, b_, dtype=torch.int64) for a_, b_ in slices])
+        mv = torch.empty((qids.numel(), k), dtype=torch.float32, device=query.device)
+        mi = torch.empty((qids.numel(), k), dtype=torch.int32, device=query.device)
+        offs = [0]
+        for a_, b_ in slices:
+            offs.append(offs[-1] + b_ - a_)
+
+        def merge(c):
+            s0, s1 = slices[c]
+            if s1 > s0:
+                ksel_merge_lists([p + L["val"](b) + s0 * k * 4 for p in self.peer],
+                                 [p + L["idx"](b) + s0 * k * 4 for p in self.peer], s1 - s0, k, k,
+                                 mv[offs[c]:offs[c + 1]], mi[offs[c]:offs[c + 1]],
+                                 ready_ptrs=[p + L["ready"](b, c) for p in self.peer], epoch=e + 1)
+
+        for c, (qa, qb) in enumerate(spans):
+            if self.local_knn is None:  # the library writes straight into the exchange buffer
+                from . import knn_search
+                knn_search(ref_shard, query[qa:qb], k, idx_offset=r0, out_dist=ov[qa:qb], out_idx=oi[qa:qb])
+            else:
+                v, i = self.local_knn(ref_shard, query[qa:qb], k, r0)
+                ov[qa:qb].copy_(v)
+                oi[qa:qb].copy_(i)
+            flag_signal(self.base + L["ready"](b, c), e + 1)
+            if c > 0:
+                merge(c - 1)
+        merge(len(spans) - 1)
         for p in self.peer:
             flag_signal(p + L["consumed"](self.rank), e + 1)
         self.epoch += 1
-        return mv, mi, (q0, q1)
+        return mv, mi, qids
 
     def check(self):
         """Synchronise and raise if a device-side flag wait of the exchange timed out

@@ -2,10 +2,12 @@
 
 The local kernels are replaced by CPU stand-ins built on the oracle (test
 infrastructure) so that the host-side plumbing of the multi-GPU paths --
-partitioning, global index offsets, (value, index) packing, the all-gather and
-the per-rank query slice of the merge -- is checked end to end against the
-unsharded oracle result, bit for bit.  On a GPU box the same functions run
-with the CUDA library and NCCL (bench.py / tests/test_dist_gpu.py).
+partitioning, global index offsets, the query-chunk pipeline, the in-place
+[2][qc][k] send / [g][2][qc][k] receive buffers, the async all-gathers and the
+per-rank query slices of the merge -- is checked end to end against the
+unsharded oracle result, bit for bit.  tests/test_dist_gpu.py runs the same
+function with the CUDA kernels (several processes sharing one GPU); bench.py
+runs it with NCCL under torchrun.
 """
 import os
 import socket
@@ -27,19 +29,21 @@ def _free_port():
     return p
 
 
-def _cpu_knn(ref, query, k, idx_offset):
+def _cpu_knn(ref, query, k, idx_offset, out_v, out_i):
     import oracle
     v, i = oracle.knn(ref.numpy(), query.numpy(), k, idx_offset=idx_offset)
-    return torch.from_numpy(v), torch.from_numpy(i)
+    out_v.copy_(torch.from_numpy(v))
+    out_i.copy_(torch.from_numpy(i))
 
 
-def _cpu_merge(cv, ci, k):
+def _cpu_merge(vals, idxs, k, out_v, out_i):
     import oracle
-    v, i = oracle.merge(cv.numpy(), ci.numpy(), k)
-    return torch.from_numpy(v), torch.from_numpy(i)
+    v, i = oracle.merge(torch.stack(vals).numpy(), torch.stack(idxs).numpy(), k)
+    out_v.copy_(torch.from_numpy(v))
+    out_i.copy_(torch.from_numpy(i))
 
 
-def _worker(rank, world, port, kind, N, Q, D, k, out_dir):
+def _worker(rank, world, port, kind, N, Q, D, k, chunks, out_dir):
     import sys
     sys.path.insert(0, ROOT)
     os.environ["MASTER_ADDR"] = "127.0.0.1"
@@ -50,34 +54,43 @@ def _worker(rank, world, port, kind, N, Q, D, k, out_dir):
     ref = synth.knn_points(kind, 11, 0, N, D)
     qry = synth.knn_points(kind, 12, 0, Q, D)
     r0, r1 = kd.shard_range(N, world, rank)
-    v, i, (q0, q1) = kd.knn_search_sharded(ref[r0:r1].contiguous(), qry, k, N, local_knn=_cpu_knn,
-                                           merge=_cpu_merge)
+    v, i, qids = kd.knn_search_sharded(ref[r0:r1].contiguous(), qry, k, N, chunks=chunks, local_knn=_cpu_knn,
+                                       merge=_cpu_merge)
     np.save(os.path.join(out_dir, "v%d.npy" % rank), v.numpy())
     np.save(os.path.join(out_dir, "i%d.npy" % rank), i.numpy())
-    np.save(os.path.join(out_dir, "q%d.npy" % rank), np.array([q0, q1]))
+    np.save(os.path.join(out_dir, "q%d.npy" % rank), qids.numpy())
     tdist.barrier()
     tdist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world", [2, 3])
+@pytest.mark.parametrize("world,chunks", [(2, 1), (2, 3), (3, 4)])
 @pytest.mark.parametrize("kind", ["knn-S", "knn-U"])
-def test_row_sharded_knn_equals_unsharded(tmp_path, oracle_mod, world, kind):
+def test_row_sharded_knn_equals_unsharded(tmp_path, oracle_mod, world, chunks, kind):
     N, Q, D, k = 1003, 37, 16, 25
-    mp.start_processes(_worker, args=(world, _free_port(), kind, N, Q, D, k, str(tmp_path)), nprocs=world,
-                       join=True, start_method="spawn")
+    mp.start_processes(_worker, args=(world, _free_port(), kind, N, Q, D, k, chunks, str(tmp_path)),
+                       nprocs=world, join=True, start_method="spawn")
     import synth
     ref = synth.knn_points(kind, 11, 0, N, D).numpy()
     qry = synth.knn_points(kind, 12, 0, Q, D).numpy()
     ev, ei = oracle_mod.knn(ref, qry, k)
-    covered = 0
+    seen = []
     for r in range(world):
-        q0, q1 = np.load(tmp_path / ("q%d.npy" % r))
+        qids = np.load(tmp_path / ("q%d.npy" % r))
         v = np.load(tmp_path / ("v%d.npy" % r))
         i = np.load(tmp_path / ("i%d.npy" % r))
-        assert np.array_equal(i, ei[q0:q1])
-        assert np.array_equal(v.view(np.uint32), ev[q0:q1].view(np.uint32))
-        covered += q1 - q0
-    assert covered == Q
+        assert np.array_equal(i, ei[qids])
+        assert np.array_equal(v.view(np.uint32), ev[qids].view(np.uint32))
+        seen += qids.tolist()
+    assert sorted(seen) == list(range(Q))  # every query merged by exactly one rank
+
+
+def test_chunk_ranges_partition():
+    from paper_conf_ipps_tang0emg15_b200 import dist as kd
+    for Q in (1, 5, 37, 10000):
+        for c in (1, 3, 4, 8, 100):
+            spans = kd.chunk_ranges(Q, c)
+            assert spans[0][0] == 0 and spans[-1][1] == Q and len(spans) == min(c, Q)
+            assert all(spans[j][1] == spans[j + 1][0] for j in range(len(spans) - 1))
 
 
 def test_query_rows_partition():
@@ -94,7 +107,8 @@ def test_p2p_layout_regions_disjoint():
     from paper_conf_ipps_tang0emg15_b200 import dist
     for Q, k, world in [(1, 1, 1), (1000, 100, 8), (10000, 1024, 64), (7, 3, 5)]:
         L = dist.p2p_layout(Q, k, world)
-        spans = [(L["ready"](b), 4) for b in range(2)] + [(L["consumed"](s), 4) for s in range(world)]
+        spans = [(L["ready"](b, c), 4) for b in range(2) for c in range(dist.P2P_MAX_CHUNKS)]
+        spans += [(L["consumed"](s), 4) for s in range(world)]
         spans += [(L["val"](b), Q * k * 4) for b in range(2)] + [(L["idx"](b), Q * k * 4) for b in range(2)]
         spans.sort()
         for (a, n), (b_, _) in zip(spans, spans[1:]):

@@ -139,16 +139,17 @@ from paper_conf_ipps_tang0emg15_b200 import dist
 torch.cuda.set_device(0)
 tdist.init_process_group("gloo", init_method="tcp://127.0.0.1:" + port, rank=rank, world_size=world)
 N, Q, D, k = 20000, 1000, 128, 100
-p2p = dist.KnnP2P(Q, k, N)
+p2p = dist.KnnP2P(Q, k, N, chunks=3)
 r0, r1 = dist.shard_range(N, world, rank)
 for ep in range(4):
     kind = "knn-S" if ep % 2 else "knn-U"
     ref = synth.knn_points(kind, 70 + ep, 0, N, D, device="cuda")
     qry = synth.knn_points(kind, 80 + ep, 0, Q, D, device="cuda")
-    mv, mi, (q0, q1) = p2p(ref[r0:r1].contiguous(), qry)
+    mv, mi, qids = p2p(ref[r0:r1].contiguous(), qry)
     torch.cuda.synchronize()
     np.save(out + "/v_%d_%d.npy" % (ep, rank), mv.cpu().numpy())
     np.save(out + "/i_%d_%d.npy" % (ep, rank), mi.cpu().numpy())
+    np.save(out + "/q_%d_%d.npy" % (ep, rank), qids.numpy())
 p2p.check()
 p2p.close()
 tdist.destroy_process_group()
@@ -180,14 +181,16 @@ def test_knn_p2p_processes_on_one_gpu(K, oracle_mod, tmp_path, world):
         qry = synth.knn_points(kind, 80 + ep, 0, Q, D, device="cuda")
         ev, ei = K.knn_search(ref, qry, k)
         ev, ei = ev.cpu().numpy(), ei.cpu().numpy()
+        qids = np.concatenate([np.load(tmp_path / ("q_%d_%d.npy" % (ep, r))) for r in range(world)])
         gv = np.concatenate([np.load(tmp_path / ("v_%d_%d.npy" % (ep, r))) for r in range(world)])
         gi = np.concatenate([np.load(tmp_path / ("i_%d_%d.npy" % (ep, r))) for r in range(world)])
-        # against the oracle (all Q queries of all ranks' slices, in rank order)
+        assert sorted(qids.tolist()) == list(range(Q))  # every query merged by exactly one rank
+        order = np.argsort(qids)
+        gv, gi = gv[order], gi[order]
+        # against the oracle (all Q queries), and bit-identical to the unsharded knn_search
         check_knn(oracle_mod, ref.cpu(), qry.cpu(), k, gv, gi)
-        for r in range(world):
-            q0, q1 = dist.shard_range(Q, world, r)
-            assert np.array_equal(gi[q0:q1], ei[q0:q1]), (ep, r)
-            assert np.array_equal(gv[q0:q1].view(np.uint32), ev[q0:q1].view(np.uint32)), (ep, r)
+        assert np.array_equal(gi, ei), ep
+        assert np.array_equal(gv.view(np.uint32), ev.view(np.uint32)), ep
 
 
 def test_flag_wait_timeout_reports_without_killing_the_context(K):

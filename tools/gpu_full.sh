@@ -1,0 +1,3 @@
+cd $GRAFT_REPO_ROOT; mkdir -p gpurun_out
+timeout 300 python __graft_entry__.py smoke > gpurun_out/smoke.log 2>&1; echo "smoke=$?"
+timeout 2400 python -m pytest tests -m gpu -q -rf -x > gpurun_out/pytest_full.log 2>&1; echo "pytest=$?"
