@@ -23,12 +23,15 @@ struct KnnStats {
 //     off by <= 6.1 2^-16 |q_i r_i|, and sum |q_i r_i| <= |q| |r| <= sqrt(|q|^2 R2);
 //   * fp32 accumulation of 3D products and 6 norm terms, each rounding <= 2^-24 of the
 //     absolute sum <= 2.02 (|q|^2 + |r|^2), and the 24-bit norm splits:
-//     (3D + 16) 2^-23 (|q|^2 + R2);
+//     (3D + 16) 2^-23 (|q|^2 + R2), plus (3D + 16) 2^-124 for underflow;
 // times 2 for safety.  Returned rounded up; +Inf if an input is not finite (the query
 // then takes the exact fallback).
 __device__ __forceinline__ float knn_eps(float4 qs, const KnnStats& st, int D) {
     const double R2 = (double)__uint_as_float(st.R2), nq = (double)qs.w;
-    const double e = 2.0 * (6.1 * 0x1p-16 * sqrt(nq * R2) + (double)(3 * D + 16) * 0x1p-23 * (nq + R2));
+    // (+ (3D + 16) 2^-124: products and partial sums that underflow the fp32 range -- flushed
+    // or denormal in the tensor core -- each lose less than 2^-126)
+    const double e = 2.0 * (6.1 * 0x1p-16 * sqrt(nq * R2) + (double)(3 * D + 16) * 0x1p-23 * (nq + R2) +
+                            (double)(3 * D + 16) * 0x1p-124);
     const float f = __double2float_ru(e);
     return (f == f) ? f : __int_as_float(0x7f800000);
 }
