@@ -322,11 +322,16 @@ __device__ __forceinline__ void umma_commit_mc(uint64_t* bar, uint16_t mask) {
 // ---------------------------------------------------------------------------
 struct KnnSmem {
     static constexpr int kHistWarp = 256 * 4;                  // per epilogue warp: radix histogram (pool_select64)
-    static constexpr int kWarpScratch = KNN_SB * 32 * 4;      // per epilogue warp: sampling histogram, one per lane
+    static constexpr int kWarpScratch = KNN_SB * 32 * 4;      // per query group of 32: sampling histogram, one per lane
     // scratch of `ew` epilogue warps (sized for the launch: every KB left goes to the ring)
-    __host__ __device__ static int scratch(int ew) { return ew * (kHistWarp + kWarpScratch); }
+    // EW warps' radix histograms, one sampling histogram per query group (a TMEM lane
+    // quadrant of a query tile: the EW / 4 warps scanning its column parts share it), and
+    // the per-query state those warps share: pool fill, failure flag, bound pair
+    __host__ __device__ static int scratch(int ew, int qpc) {
+        return ew * kHistWarp + 4 * qpc * kWarpScratch + qpc * 128 * 16;
+    }
     __host__ __device__ static int total(const KnnGeom& g) {
-        return 1024 /*align slack*/ + g.QPC * g.a_bytes() + g.NS * g.stage_bytes() + scratch(g.EW) +
+        return 1024 /*align slack*/ + g.QPC * g.a_bytes() + g.NS * g.stage_bytes() + scratch(g.EW, g.QPC) +
                (2 * g.NS + 5) * 8 + 16;
     }
 };
@@ -361,7 +366,11 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
     uint8_t* sB = sA + QPC * g.a_bytes();
     uint32_t* hist_all = reinterpret_cast<uint32_t*>(sB + NS * SB);
     float* dstage_all = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(hist_all) + EW * KnnSmem::kHistWarp);
-    uint64_t* bars = reinterpret_cast<uint64_t*>(reinterpret_cast<uint8_t*>(dstage_all) + EW * KnnSmem::kWarpScratch);
+    unsigned long long* qs_T = reinterpret_cast<unsigned long long*>(reinterpret_cast<uint8_t*>(dstage_all) +
+                                                                     4 * QPC * KnnSmem::kWarpScratch);  // [QPC*128]
+    int* qs_n = reinterpret_cast<int*>(qs_T + QPC * 128);                                              // [QPC*128]
+    int* qs_f = qs_n + QPC * 128;                                                                      // [QPC*128]
+    uint64_t* bars = reinterpret_cast<uint64_t*>(qs_f + QPC * 128);
     uint64_t* full = bars;
     uint64_t* empty = bars + NS;
     uint64_t* accf = bars + 2 * NS;
@@ -499,10 +508,22 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
         const int64_t q = (int64_t)qt * KNN_BM + row;
         const bool qvalid = q < g.Q;
         uint32_t* hist = hist_all + e * 256;
-        uint8_t* wscratch = reinterpret_cast<uint8_t*>(dstage_all) + e * KnnSmem::kWarpScratch;
-        // this query's candidate pool: packed pairs (key << 32 | reference row)
-        // (each (split, half) keeps its own pools: S * HALVES lists per query for the merge)
-        const size_t list = (size_t)split * HALVES + half;
+        // The PAIR = EW / 4 warps on one query group (same TMEM lanes, different column
+        // parts) share the query's pool, its fill counter and its bound (shared memory);
+        // they meet at a named barrier before and after every narrowing phase.
+        constexpr int PAIR = HALVES;
+        const int qgrp = hq * 4 + quad;
+        const int qidx = hq * 128 + row;
+        uint8_t* wscratch = reinterpret_cast<uint8_t*>(dstage_all) + qgrp * KnnSmem::kWarpScratch;
+        int* np = qs_n + qidx;
+        int* fp = qs_f + qidx;
+        unsigned long long* Tp = qs_T + qidx;
+        auto pair_bar = [&]() {
+            if constexpr (PAIR > 1) asm volatile("bar.sync %0, %1;" ::"r"(1 + qgrp), "r"(32 * PAIR) : "memory");
+            else __syncwarp();
+        };
+        // this query's candidate pool: packed pairs (key << 32 | reference row), one per split
+        const size_t list = (size_t)split;
         unsigned long long* pool = pool64 + (list * g.Q + (qvalid ? q : 0)) * g.P;
         unsigned long long T = kSentPair;  // running bound on the k-th (d~, index) pair
         // the band: 2 eps_q above the k-th d~ (every reference that can be in the exact top-k)
@@ -510,26 +531,49 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
         float tv = 0.f;                    // filter value: value(T) + band, rounded up
         bool fast = false;                 // finite filter value: the fp32 compare d~ <= tv pre-filters
         bool failed = !(band < __int_as_float(0x7f800000));  // no finite band: exact fallback
-        if (qvalid && !DUMP && !PIPE_ONLY && failed) qfail[q] = 1;
-        int n = 0;
+        if (qvalid && !DUMP && !PIPE_ONLY && failed && half == 0) qfail[q] = 1;
+        if (half == 0) {
+            *np = 0;
+            *fp = failed ? 1 : 0;
+            *Tp = kSentPair;
+        }
+        pair_bar();
 
+        auto set_T = [&](unsigned long long t) {
+            T = t;
+            const uint32_t tk = (uint32_t)(T >> 32);
+            tv = (tk < 0xff800000u) ? __fadd_ru(__uint_as_float(bits_of_key(tk)), band) : 0.f;
+            fast = tk < 0xff800000u && tv < __int_as_float(0x7f800000);
+        };
         auto adopt = [&](unsigned long long t) {
             if (t < T) {
-                T = t;
-                const uint32_t tk = (uint32_t)(T >> 32);
-                tv = (tk < 0xff800000u) ? __fadd_ru(__uint_as_float(bits_of_key(tk)), band) : 0.f;
-                fast = tk < 0xff800000u && tv < __int_as_float(0x7f800000);
+                set_T(t);
+                if (PAIR > 1) atomicMin(Tp, t);
+            }
+        };
+        // after a pair barrier: the pair's shared bound and failure flag
+        auto refresh = [&]() {
+            if constexpr (PAIR > 1) {
+                const unsigned long long t = *reinterpret_cast<volatile unsigned long long*>(Tp);
+                if (t < T) set_T(t);
+                failed = *reinterpret_cast<volatile int*>(fp) != 0;
             }
         };
         // warp-cooperative narrowing of every lane whose pool cannot take `room` more pairs:
         // the exact k-th pair of the pool becomes the bound and the pool keeps the band
         // above it; mid-stream, a band that alone leaves no room fails the query
+        // (the PAIR warps of a query group split the narrowings of its lanes between them)
         auto narrow_lanes = [&](int room, int target, int cap, bool final_pass) {
+            pair_bar();
+            refresh();
+            const int n = *reinterpret_cast<volatile int*>(np);
             uint32_t need = __ballot_sync(kFull, qvalid && !failed && n + room > cap && n > target);
+            int turn = 0;
             while (need) {
                 if (PROF) prof_nnarrow++;
                 const int j = __ffs(need) - 1;
                 need &= need - 1u;
+                if ((turn++ % PAIR) != half) continue;
                 unsigned long long* jp = (unsigned long long*)__shfl_sync(kFull, (unsigned long long)pool, j);
                 const int jn = __shfl_sync(kFull, n, j);
                 const float jb = __shfl_sync(kFull, band, j);
@@ -540,18 +584,21 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                                                  ? pool_narrow64<kNarrowRegs>(jp, jn, (uint32_t)target, &nn, jb)
                                                  : pool_select64(jp, jn, (uint32_t)target, hist, &nn, jb);
                 if ((int)lane == j) {
-                    n = nn;
+                    *np = nn;
                     adopt(t);
                     // publish: the k-th pair of this split's part bounds the whole row
                     if (target == g.k && (uint32_t)(t >> 32) != kSentKey) atomicMin(&qthr[q], t);
-                    if (!final_pass && n + room > cap) {  // the band alone fills the pool
+                    if (!final_pass && nn + room > cap) {  // the band alone fills the pool
                         failed = true;
-                        n = 0;
+                        *np = 0;
+                        *fp = 1;
                         qfail[q] = 1;
                     }
                 }
             }
             __syncwarp();
+            pair_bar();
+            refresh();
         };
 
         // sample histogram of this lane's query: 64 buckets [lo, hi) in the warp scratch
@@ -569,7 +616,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                 adopt(thr_next);
                 if (qvalid) thr_next = __ldcg(&qthr[q]);
                 const unsigned long long c0 = PROF ? clock64() : 0;
-                narrow_lanes(WCOLS, g.k, g.pcap, false);
+                narrow_lanes(BN, g.k, g.pcap, false);  // room: both column parts of a tile
                 if (PROF) prof_narrow += clock64() - c0;
             }
             const unsigned long long cw0 = PROF ? clock64() : 0;
@@ -619,8 +666,11 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                     // spare bucket for rounding); otherwise no histogram for this query
                     if (!(s_hi < __int_as_float(0x7f800000)) || !(s_hi - s_lo > s_hi * 0x1p-10f)) s_hi = -1.f;
                     s_inv = (s_hi > 0.f) ? (float)KNN_SB / (s_hi - s_lo) : 0.f;
+                    if (half == 0) {
 #pragma unroll 8
-                    for (int j = 0; j < KNN_SB; ++j) shist[j * 32] = 0u;
+                        for (int j = 0; j < KNN_SB; ++j) shist[j * 32] = 0u;
+                    }
+                    pair_bar();  // the shared histogram is clear before either warp counts
                 }
             }
             if (sampling) {
@@ -638,8 +688,9 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                         }
                     }
                 }
-                if (lt == Fs - 1 && qvalid && s_hi > 0.f) {
-                    // >= k of this warp's sampled distances lie in buckets <= j, i.e. below lo + (j + 1) w;
+                if (lt == Fs - 1) pair_bar();  // both column parts counted
+                if (lt == Fs - 1 && qvalid && s_hi > 0.f && half == 0) {
+                    // >= k of the sampled distances lie in buckets <= j, i.e. below lo + (j + 1) w;
                     // one spare bucket absorbs the rounding of the bucket index
                     uint32_t cum = 0;
                     int j = 0;
@@ -700,7 +751,8 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                             const float x = __uint_as_float(b2 ? c23 : c01);
                             if (cu + i < nlim && (!fast || x <= tv)) {
                                 const float dc = (x < 0.f) ? 0.f : x;  // clamp, NaN propagates
-                                pool[n++] = ((unsigned long long)key_of(dc) << 32) | (colt + (uint32_t)(cu + i));
+                                const int slot = (PAIR > 1) ? atomicAdd(np, 1) : (*np)++;
+                                pool[slot] = ((unsigned long long)key_of(dc) << 32) | (colt + (uint32_t)(cu + i));
                                 if (PROF) prof_app++;
                             }
                         }
@@ -726,7 +778,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                 uint32_t v[KNN_CW];
                 tmem_ld64(taddr + (uint32_t)(c * KNN_CW), v);
                 if (PIPE_ONLY) {
-                    if (v[0] == 0x7fc00001u && v[KNN_CW - 1] == 0x7fc00001u) n++;  // keep the load alive
+                    if (v[0] == 0x7fc00001u && v[KNN_CW - 1] == 0x7fc00001u) (*np)++;  // keep the load alive
                     continue;
                 }
                 const int64_t col0 = (int64_t)t * BN + c * KNN_CW;
@@ -751,7 +803,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
             // the pool's k smallest); launch_merge_pools gathers the pools' pairs <= the
             // final published bound and selects the exact top-k of the row.
             narrow_lanes(g.P - g.k, g.k, g.P, true);  // n > k  <=>  n + (P - k) > P
-            if (qvalid) cnt_out[list * g.Q + q] = failed ? 0 : n;
+            if (qvalid && half == 0) cnt_out[list * g.Q + q] = failed ? 0 : *np;
         }
         if (PROF) {
             __syncwarp();
@@ -840,13 +892,13 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
 #ifdef KSEL_EXPERIMENTS
     static const int ew_env = env_int("KSEL_KNN_EW", 4) == 8 ? 8 : 4;  // experiments: 4 or 8 epilogue warps
 #else
-    constexpr int ew_env = 4;
+    constexpr int ew_env = 8;
 #endif
     g.halves = (g.QPC == 2) ? 1 : ew_env / 4;
     g.EW = (g.QPC == 2) ? 8 : 4 * g.halves;
     // ring depth: as many stages as fit next to the resident query tile(s)
     const int fixed =
-        1024 + g.QPC * (g.Dp * 512 + KNN_NORM_A_BYTES) + KnnSmem::scratch(g.EW) + 512;
+        1024 + g.QPC * (g.Dp * 512 + KNN_NORM_A_BYTES) + KnnSmem::scratch(g.EW, g.QPC) + 512;
     g.NS = (kMaxSmemPerBlock - fixed) / g.stage_bytes();
     if (g.NS > 6) g.NS = 6;
     g.idx_offset = idx_offset;
@@ -854,7 +906,7 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     // narrow before a pool reaches P when queues are small: the bound then tracks the
     // k-th of what has been seen more closely in cold CTAs (measured: 512 for k <= 128)
     const int cap = cap_env > 0 ? cap_env : (kk <= 128 ? 512 : g.P);
-    g.pcap = std::max(kk + 32 + g.BN / g.halves, std::min(g.P, cap));
+    g.pcap = std::max(kk + 32 + g.BN, std::min(g.P, cap));
     g.ntiles = g.NT;
     g.tstride = 1;
     // first-wave CTAs sample 16 tiles (4096 references) for their starting bound
@@ -866,7 +918,7 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     double best_cost = 1e30;
     const int smax = (int)((g.NT < 64) ? g.NT : 64);
     for (int s = 1; s <= smax; ++s) {
-        if (max_lists > 0 && s > 1 && (int64_t)s * g.halves * Q > max_lists) break;
+        if (max_lists > 0 && s > 1 && (int64_t)s * Q > max_lists) break;
         const double ctas = (double)g.QTp * s;
         const double waves = ctas / num_sms;
         const double cost = (double)((int64_t)((ctas + num_sms - 1) / num_sms)) / waves  // tail efficiency
@@ -880,7 +932,7 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     static const int splits_env = env_int("KSEL_KNN_SPLITS", 0);  // experiments: force the split count
     if (splits_env > 0) {
         g.S = std::min(splits_env, smax);
-        if (max_lists > 0) g.S = (int)std::max<int64_t>(1, std::min<int64_t>(g.S, max_lists / (g.halves * Q)));
+        if (max_lists > 0) g.S = (int)std::max<int64_t>(1, std::min<int64_t>(g.S, max_lists / Q));
     }
     g.cold_splits = std::min(g.S, (num_sms + g.QTp - 1) / g.QTp);
     return g;
@@ -893,8 +945,8 @@ static KnnWork knn_work_layout(const KnnGeom& g) {
     w.stats = off;   off += al256(sizeof(KnnStats));
     w.q_img = off;   off += al256((size_t)g.QTp * g.QPC * g.a_bytes());
     w.qstat = off;   off += al256((size_t)g.Q * 16);
-    w.pool = off;    off += al256((size_t)g.halves * g.S * g.Q * g.P * 8);
-    w.cnt = off;     off += al256((size_t)g.halves * g.S * g.Q * 4);
+    w.pool = off;    off += al256((size_t)g.S * g.Q * g.P * 8);  // one pool per (split, query)
+    w.cnt = off;     off += al256((size_t)g.S * g.Q * 4);
     w.qthr = off;    off += al256((size_t)g.Q * 8);
     w.qfail = off;   off += al256((size_t)g.Q * 4);
     w.fb = off;      off += al256(knn_fallback_bytes(g.k));
@@ -908,7 +960,7 @@ static int64_t knn_query_chunk(int64_t N, int64_t Q, int D, int k, int sms) {
     int64_t qc = Q;
     for (;;) {
         const KnnGeom g = knn_geometry(N, qc, D, k, sms, 0);
-        if ((size_t)g.halves * g.S * (size_t)qc * (size_t)g.P * 8u <= kPoolBudget || qc <= KNN_BM) return qc;
+        if ((size_t)g.S * (size_t)qc * (size_t)g.P * 8u <= kPoolBudget || qc <= KNN_BM) return qc;
         qc = std::max<int64_t>(KNN_BM, (qc / 2 + KNN_BM - 1) / KNN_BM * KNN_BM);
     }
 }
@@ -945,7 +997,7 @@ static cudaError_t knn_run(const float* ref, const float* query, int64_t N, int6
     if (e != cudaSuccess) return e;
     for (int64_t q0 = 0; q0 < Q; q0 += Qc) {
         const int64_t nq = std::min(Qc, Q - q0);
-        const KnnGeom g = knn_geometry(N, nq, D, k, sms, idx_offset, (int64_t)gq.halves * gq.S * Qc);
+        const KnnGeom g = knn_geometry(N, nq, D, k, sms, idx_offset, (int64_t)gq.S * Qc);
         const int nt = (q0 == 0) ? g.NT : 0;  // reference tiles: first chunk only
         knn_prep_kernel<<<(unsigned)(nt + g.QT), KNN_PREP_THREADS, 0, stream>>>(
             ref, query + q0 * (int64_t)D, g, nt, ref_img, q_img, qstat, stats);
@@ -978,7 +1030,7 @@ static cudaError_t knn_run(const float* ref, const float* query, int64_t N, int6
         if (!dump && mode_env == 3) kdump = reinterpret_cast<float*>(work + w.prof);
 #else
         constexpr int mode_env = 0;
-        auto kern = dump ? knn_fused_kernel<1, 4, 256, 1> : knn_fused_kernel<0, 4, 256, 1>;
+        auto kern = dump ? knn_fused_kernel<1, 8, 256, 1> : knn_fused_kernel<0, 8, 256, 1>;
 #endif
         e = ensure_smem_attr(reinterpret_cast<const void*>(kern), smem);
         if (e != cudaSuccess) return e;
@@ -1026,7 +1078,7 @@ static cudaError_t knn_run(const float* ref, const float* query, int64_t N, int6
         a.pools = reinterpret_cast<const unsigned long long*>(work + w.pool);
         a.P = g.P;
         a.cnt = reinterpret_cast<const int32_t*>(work + w.cnt);
-        a.S = g.halves * g.S;
+        a.S = g.S;
         a.thr = reinterpret_cast<const unsigned long long*>(work + w.qthr);
         a.qfail = reinterpret_cast<const int32_t*>(work + w.qfail);
         a.qstat = qstat;
