@@ -57,6 +57,9 @@ def parse():
     ap.add_argument("--dist", default=None)
     ap.add_argument("--scaling", choices=["weak", "strong"], default="strong")
     ap.add_argument("--no-sweep", action="store_true", help="skip the k x distribution / kNN sweep (N = 1)")
+    ap.add_argument("--knn-sharded", choices=["auto", "on", "off"], default="auto",
+                    help="also time the row-sharded kNN (configs[4]) over the process group: "
+                         "auto = only when N > 1")
     ap.add_argument("--e2e-rows", type=int, default=0,
                     help="rows per end-to-end step per rank (host buffers); 0 = 2048 on one GPU, "
                          "512 per rank on several (pinned host memory: 4 MB per row)")
@@ -505,6 +508,65 @@ def run_sweep(dev, K, peak_hbm, peak_bf16):
     return out
 
 
+def run_knn_row_sharded(args, rank, world, dev, K, tdist):
+    """configs[4] over the process group: N = 8*10^6 references sharded by rows (10^6 per
+    rank at g = 8; N = 10^6 * g in total for g < 8 so every rank keeps the per-rank shape),
+    Q = 10^4, k = 1024, each rank's search writing into the chunked all-gather buffers and
+    merging its query slices in place (dist.knn_search_sharded; NCCL over NVLink).  Device
+    time between barriers, max over ranks; bit-exactness of this path is tested in
+    tests/test_dist_gpu.py (same function, real kernels)."""
+    import torch
+
+    import synth
+    from paper_conf_ipps_tang0emg15_b200 import dist as kd
+    N = 1000000 * world if world < 8 else 8000000
+    Q, D, k = 10000, 128, 1024
+    r0, r1 = kd.shard_range(N, world, rank)
+    ref = synth.knn_points("knn-U", 41, r0, r1 - r0, D, device=dev)
+    qry = synth.knn_points("knn-U", 42, 0, Q, D, device=dev)
+    ws = torch.empty(K.knn_search_workspace(r1 - r0, Q, D, k), dtype=torch.uint8, device=dev)
+
+    def local_knn(rs, qq, kk, off, out_v, out_i):
+        K.knn_search(rs, qq, kk, idx_offset=off, out_dist=out_v, out_idx=out_i, workspace=ws)
+
+    chunks = int(os.environ.get("KSEL_BENCH_CHUNKS", "0")) or kd.auto_chunks(Q)
+
+    def step():
+        return kd.knn_search_sharded(ref, qry, k, N, local_knn=local_knn, chunks=chunks)
+
+    for _ in range(2):
+        step()
+    torch.cuda.synchronize()
+    steps = 3
+    if world > 1:
+        tdist.barrier()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(steps):
+        v, i, qids = step()
+    e1.record()
+    torch.cuda.synchronize()
+    t = torch.tensor([e0.elapsed_time(e1) / steps], dtype=torch.float64, device=dev)
+    if world > 1:
+        tdist.barrier()
+        tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
+    ms = float(t.item())
+    # every query merged by exactly one rank, k ascending distances each
+    nq = torch.tensor([qids.numel()], dtype=torch.int64, device=dev)
+    if world > 1:
+        tdist.all_reduce(nq)
+    ok = int(nq.item()) == Q and bool((v[:, 1:] >= v[:, :-1]).all().item())
+    del ref, qry, ws
+    torch.cuda.empty_cache()
+    return {"workload": "knn_search N=%d (row-sharded x%d) Q=%d D=%d k=%d knn-U" % (N, world, Q, D, k),
+            "ms_per_step": ms, "queries_per_s": Q / (ms / 1e3), "chunks": chunks,
+            "exchange": "async all_gather_into_tensor per query chunk (%s) + in-place merge; chunks: "
+                        "dist.auto_chunks (1 at Q = 10^4: chunking the search costs more than the "
+                        "exchange it hides, profiles/r02_knn_sharded_chunks.txt)" % ("NCCL" if world > 1 else "single rank"),
+            "tflops_per_rank": 2.0 * Q * (r1 - r0) * D / (ms / 1e3) / 1e12, "queries_covered_sorted": ok}
+
+
 KNN_CONFIGS = {
     # name: (N total, Q, D, k, point kind, mode)
     "c4": (1000000, 10000, 128, 100, "knn-U", "replica"),
@@ -663,6 +725,10 @@ def main():
     dev = torch.device("cuda", local_rank)
     if world > 1:
         tdist.init_process_group("nccl", device_id=dev)
+    elif args.knn_sharded == "on":  # single-rank NCCL group: exercises the sharded path on one GPU
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29533")
+        tdist.init_process_group("nccl", rank=0, world_size=1, device_id=dev)
 
     import paper_conf_ipps_tang0emg15_b200 as K
 
@@ -680,9 +746,15 @@ def main():
             except Exception:
                 pass
             line["sweep"] = run_sweep(dev, K, line["roofline"]["peak"], peak_bf16)
+        if args.config == "c3" and (args.knn_sharded == "on" or (args.knn_sharded == "auto" and world > 1)):
+            import torch
+            torch.cuda.empty_cache()
+            ks = run_knn_row_sharded(args, rank, world, dev, K, tdist)
+            if rank == 0:
+                line["knn_row_sharded"] = ks
     if rank == 0:
         print(json.dumps(line), flush=True)
-    if world > 1:
+    if tdist.is_initialized():
         tdist.destroy_process_group()
 
 

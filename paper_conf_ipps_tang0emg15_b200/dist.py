@@ -61,6 +61,15 @@ def _all_gather(out: torch.Tensor, inp: torch.Tensor, group=None, async_op=False
         return tdist.all_gather(parts, inp, group=group, async_op=async_op)
 
 
+def auto_chunks(Q: int) -> int:
+    """Query chunks of the exchange pipeline.  Every extra knn_search call pays a cold
+    start (first-wave CTAs without a published bound) and a reference prologue; measured
+    on one B200 at configs[4]'s per-rank shape (10^6 references, Q = 10^4, k = 1024):
+    1 / 2 / 4 chunks = 18.4 / 23.6 / 36.8 ms per step against an all-gather of ~1 ms at
+    8 GPUs -- so the pipeline is used only for large query batches (>= 20000 per chunk)."""
+    return max(1, min(4, Q // 20000))
+
+
 def chunk_ranges(Q: int, chunks: int) -> list:
     """Contiguous query chunks [a, b) of the exchange pipeline."""
     c = max(1, min(int(chunks), Q))
@@ -68,7 +77,7 @@ def chunk_ranges(Q: int, chunks: int) -> list:
 
 
 def knn_search_sharded(ref_shard: torch.Tensor, query: torch.Tensor, k: int, n_total: int, group=None,
-                       chunks: int = 4, local_knn=None, merge=None):
+                       chunks: int | None = None, local_knn=None, merge=None):
     """Row-sharded k-NN: local top-k with global indices, all-gather, merge -- pipelined
     over query chunks.
 
@@ -89,7 +98,7 @@ def knn_search_sharded(ref_shard: torch.Tensor, query: torch.Tensor, k: int, n_t
     assert ref_shard.shape[0] == r1 - r0, "ref_shard must hold rows [%d, %d)" % (r0, r1)
     Q = query.shape[0]
     dev = query.device
-    spans = chunk_ranges(Q, chunks)
+    spans = chunk_ranges(Q, auto_chunks(Q) if chunks is None else chunks)
     slices = [(qa + shard_range(qb - qa, world, rank)[0], qa + shard_range(qb - qa, world, rank)[1])
               for qa, qb in spans]
     qids = torch.cat([torch.arange(a, b, dtype=torch.int64) for a, b in slices])
@@ -172,7 +181,7 @@ class KnnP2P:
     Same result as :func:`knn_search_sharded` (bit-identical to unsharded).
     """
 
-    def __init__(self, Q: int, k: int, n_total: int, group=None, local_knn=None, chunks: int = 4):
+    def __init__(self, Q: int, k: int, n_total: int, group=None, local_knn=None, chunks: int | None = None):
         from . import ipc_alloc, ipc_open
         self.group = group
         self.world = tdist.get_world_size(group)
@@ -186,7 +195,7 @@ class KnnP2P:
         tdist.all_gather_object(handles, handle, group=group)
         self.peer = [self.base if s == self.rank else ipc_open(handles[s]) for s in range(self.world)]
         tdist.barrier(group=group)
-        self.chunks = max(1, min(int(chunks), P2P_MAX_CHUNKS, Q))
+        self.chunks = max(1, min(int(auto_chunks(Q) if chunks is None else chunks), P2P_MAX_CHUNKS, Q))
         self.epoch = 0
         self.warm = False
 
