@@ -567,6 +567,9 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
             pair_bar();
             refresh();
             const int n = *reinterpret_cast<volatile int*>(np);
+            // both warps of the pair have read the shared fills and bounds before either
+            // narrows (and writes them): they derive the same `need` and split it consistently
+            pair_bar();
             uint32_t need = __ballot_sync(kFull, qvalid && !failed && n + room > cap && n > target);
             int turn = 0;
             while (need) {
