@@ -96,6 +96,9 @@ KSEL_API int ksel_select_ex(const float* dist, int64_t Q, int64_t N, int k, floa
  *                  a cluster of <= 8 CTAs holds the row in registers and narrows
  *                  the exact k-th key by four 8-bit radix passes over all of it
  *                  (HP's value buckets, L225), then sorts the k selected pairs.
+ *                  KSEL_ALGO_HIST (4): one CTA per row, a shared-memory pool narrowed
+ *                  by range-adaptive radix histograms -- built into the experiments
+ *                  library only (KSEL_BUILD_EXPERIMENTS=1); KSEL_ERR_UNSUPPORTED here.
  *   warps_per_row  0 = automatic, else 1, 2, 4 or 8 warps cooperating on each row
  *                  (ignored by KSEL_ALGO_RADIX).
  * Other arguments as ksel_select; invalid algo / warps_per_row -> INVALID_ARG. */
@@ -103,6 +106,7 @@ KSEL_API int ksel_select_ex(const float* dist, int64_t Q, int64_t N, int k, floa
 #define KSEL_ALGO_QUEUE 1
 #define KSEL_ALGO_POOL 2
 #define KSEL_ALGO_RADIX 3
+#define KSEL_ALGO_HIST 4
 KSEL_API int ksel_select_config(const float* dist, int64_t Q, int64_t N, int k, float* out_val,
                                 int32_t* out_idx, int algo, int warps_per_row, void* stream);
 

@@ -90,7 +90,7 @@ for _f in (_lib.ksel_select, _lib.ksel_select_config, _lib.ksel_select_host, _li
     _f.restype = ctypes.c_int
 
 KSEL_MAX_K = 1024
-ALGO_AUTO, ALGO_QUEUE, ALGO_POOL, ALGO_RADIX = 0, 1, 2, 3
+ALGO_AUTO, ALGO_QUEUE, ALGO_POOL, ALGO_RADIX, ALGO_HIST = 0, 1, 2, 3, 4
 PQ_INSERT, PQ_HEAP, PQ_MERGE, PQ_MERGE_ALIGNED = 0, 1, 2, 3
 PB_NONE, PB_BUFFER, PB_FULL, PB_FULL_SORTED = 0, 1, 2, 3
 EXPORTS = ("ksel_select", "ksel_select_workspace", "ksel_select_ex", "ksel_select_config", "ksel_select_host_workspace", "ksel_select_host", "ksel_merge",

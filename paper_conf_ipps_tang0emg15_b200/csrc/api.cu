@@ -179,8 +179,9 @@ int ksel_select_config(const float* dist, int64_t Q, int64_t N, int k, float* ou
                        int warps_per_row, void* stream) {
     int st = check_select_args(dist, Q, N, k, out_val, out_idx);
     if (st) return st;
-    if (algo < KSEL_ALGO_AUTO || algo > KSEL_ALGO_RADIX) return KSEL_ERR_INVALID_ARG;
+    if (algo < KSEL_ALGO_AUTO || algo > KSEL_ALGO_HIST) return KSEL_ERR_INVALID_ARG;
     if (algo == KSEL_ALGO_RADIX && !radix_supported(N, k)) return KSEL_ERR_UNSUPPORTED;
+    if (algo == KSEL_ALGO_HIST && !hist_supported(N, k)) return KSEL_ERR_UNSUPPORTED;  // (experiments build only)
     if (warps_per_row != 0 && warps_per_row != 1 && warps_per_row != 2 && warps_per_row != 4 && warps_per_row != 8)
         return KSEL_ERR_INVALID_ARG;
     const size_t in_bytes = (size_t)Q * (size_t)N * 4u, out_bytes = (size_t)Q * (size_t)k * 4u;
@@ -195,7 +196,8 @@ int ksel_select_config(const float* dist, int64_t Q, int64_t N, int k, float* ou
     cudaError_t e;
     if (algo == KSEL_ALGO_RADIX) {
         e = launch_select_radix(dist, Q, N, k, out_val, out_idx, (cudaStream_t)stream);
-
+    } else if (algo == KSEL_ALGO_HIST) {
+        e = launch_select_hist(dist, Q, N, k, out_val, out_idx, di.sms, (cudaStream_t)stream);
     } else if (algo == KSEL_ALGO_QUEUE) {
         const int wpr = warps_per_row ? warps_per_row : stream_warps_per_row(Q, N, di.sms);
         e = launch_select_stream(dist, Q, N, k, out_val, out_idx, wpr, (cudaStream_t)stream);

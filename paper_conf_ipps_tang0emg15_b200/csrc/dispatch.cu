@@ -3,6 +3,7 @@
 #include <cstdint>
 #include <cuda_runtime.h>
 
+#include "ksel.h"
 #include "ksel_internal.h"
 #include "knn_common.cuh"
 
@@ -60,6 +61,22 @@ cudaError_t launch_merge(const MergeLists& L, int64_t Q, int S, int kin, int k, 
                          cudaStream_t stream) {
     KSEL_DISPATCH_R(launch_merge_r, queue_regs(k), L, Q, S, kin, k, ov, oi, stream)
 }
+
+#ifdef KSEL_EXPERIMENTS
+bool hist_supported(int64_t N, int k) { return N <= ((int64_t)1 << 30) && k >= 1 && k <= KSEL_MAX_K; }
+
+cudaError_t launch_select_hist(const float* dist, int64_t Q, int64_t N, int k, float* ov, int32_t* oi, int sms,
+                               cudaStream_t stream) {
+    KSEL_DISPATCH_R(launch_hist_r, queue_regs(k), dist, Q, N, k, ov, oi, sms, stream)
+}
+#else
+// KSEL_ALGO_HIST (select_hist.cu) is built into the experiments library only: it lost to
+// the pool kernel on C2 (profiles/r02_c2_hist_kernel_exp.txt).
+bool hist_supported(int64_t, int) { return false; }
+cudaError_t launch_select_hist(const float*, int64_t, int64_t, int, float*, int32_t*, int, cudaStream_t) {
+    return cudaErrorNotSupported;
+}
+#endif
 
 cudaError_t launch_knn_rescore(const KnnRescoreArgs& a, cudaStream_t stream) {
     KSEL_DISPATCH_R(launch_knn_rescore_r, queue_regs(a.k), a, stream)

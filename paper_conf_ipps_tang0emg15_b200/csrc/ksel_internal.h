@@ -61,6 +61,14 @@ bool radix_supported(int64_t N, int k);
 cudaError_t launch_select_radix(const float* dist, int64_t Q, int64_t N, int k, float* out_val, int32_t* out_idx,
                                 cudaStream_t stream);
 
+// One-CTA-per-row histogram selection for rows of <= 2^17 values (select_hist.cu).
+bool hist_supported(int64_t N, int k);
+cudaError_t launch_select_hist(const float* dist, int64_t Q, int64_t N, int k, float* out_val, int32_t* out_idx,
+                               int sms, cudaStream_t stream);
+template <int R>
+cudaError_t launch_hist_r(const float* dist, int64_t Q, int64_t N, int k, float* ov, int32_t* oi, int sms,
+                          cudaStream_t stream);
+
 // Merge of S sorted candidate lists (merge.cu).  List s of query q is
 // v[s] + q * kin / i[s] + q * kin (lists may live in different allocations, e.g.
 // peers' memory); ready[s] (optional) is waited for (>= epoch, acquire at system
