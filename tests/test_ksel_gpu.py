@@ -194,7 +194,7 @@ def test_config3_rows_other_distributions(K, oracle_mod, dist, k):
 # ---- split rows (few long rows over the whole GPU) ----------------
 
 @pytest.mark.parametrize("Q,N", [(1, (1 << 18) + 13), (3, 1 << 20), (7, 3 * (1 << 19) + 1), (40, 1 << 18)])
-@pytest.mark.parametrize("dist", ["U", "SD", "T", "X"])
+@pytest.mark.parametrize("dist", ["U", "SA", "SD", "T", "X"])
 def test_split_rows_vs_oracle(K, oracle_mod, Q, N, dist):
     # Q below the SM count: ksel_select cuts rows into segments (one CTA each, row-global
     # indices) and merges the S lists; ragged N makes unaligned segment heads and a short
@@ -224,6 +224,34 @@ def test_split_rows_single_long_row(K, oracle_mod):
             torch.cuda.synchronize()
             ev, ei = oracle_mod.select(x.cpu().numpy(), k)
             assert_same(ev, ei, gv, gi, "one row %s k=%d" % (dist, k))
+
+
+def test_split_rows_shared_bound_edge_cases(K, oracle_mod):
+    # the segments of a row share a row-wide bound: segments that end up with fewer than k
+    # pairs below it pad with (NaN, -1), which the second level must never select; the
+    # bound is not shared while it is NaN (rows with fewer than k non-NaN values)
+    N = (1 << 20) + 7
+    rng = np.random.default_rng(77)
+    rows = []
+    a = np.full(N, np.nan, dtype=np.float32)  # 50 finite values, the rest NaN (k > 50 below)
+    a[rng.choice(N, 50, replace=False)] = rng.random(50, dtype=np.float32)
+    rows.append(a)
+    b = np.arange(N, dtype=np.float32)  # ascending: every later segment runs short
+    rows.append(b)
+    c = np.full(N, 2.0, dtype=np.float32)  # ties everywhere + a few smaller values late
+    c[-100:] = 1.0
+    rows.append(c)
+    d = rng.random(N, dtype=np.float32)  # NaNs mixed into random values
+    d[rng.choice(N, N // 3, replace=False)] = np.nan
+    rows.append(d)
+    x_cpu = torch.from_numpy(np.stack(rows))
+    x = x_cpu.cuda()
+    for k in (1, 64, 100, 1024):
+        gv, gi = K.ksel_select(x, k)
+        torch.cuda.synchronize()
+        ev, ei = oracle_mod.select(x_cpu.numpy(), k)
+        assert_same(ev, ei, gv, gi, "split shared-bound edge k=%d" % k)
+        assert int(gi.min()) >= 0
 
 
 def test_split_rows_workspace_errors(K):
