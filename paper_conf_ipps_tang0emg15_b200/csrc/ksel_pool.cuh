@@ -202,10 +202,16 @@ __device__ __forceinline__ uint32_t count_lt(const uint32_t (&rk)[NR], uint32_t 
 // when all keys share their top bits, e.g. distances), ties by a second
 // bisection on the index, and the pool is compacted in place to the pairs
 // <= that pair (exactly `want` of them).  Returns the pair; *n_out = want.
+//
+// slack > 0 (mid-stream narrowings): the bisection stops at the first candidate key c
+// with want <= #{key < c} <= want + slack and keeps exactly those pairs; the returned
+// bound (c - 1, 0x7ffffffe) -- "every index of key c - 1" -- still has >= want pairs at
+// or below it.  A looser but valid threshold, found in a few steps instead of ~32 (the
+// exact k-th is only needed at the end of a row).
 template <int NR>
 __device__ __noinline__ unsigned long long pool_narrow_regs(uint32_t* __restrict__ pk, uint32_t* __restrict__ pi,
                                                             int n, uint32_t want, int* n_out,
-                                                            uint32_t* ties_out = nullptr) {
+                                                            uint32_t* ties_out = nullptr, uint32_t slack = 0) {
     const uint32_t lane = lane_id();
     uint32_t rk[NR], ri[NR];
 #pragma unroll
@@ -229,37 +235,50 @@ __device__ __noinline__ unsigned long long pool_narrow_regs(uint32_t* __restrict
     kmax = __reduce_max_sync(kFull, kmax);
     const int top = (kmin == kmax) ? -1 : 31 - __clz(kmin ^ kmax);
     uint32_t vkey = (top < 0) ? kmin : (kmin & ~((2u << top) - 1u));
+    uint32_t early = 0;  // (slack) candidate key whose "below" set fits [want, want + slack]
 #pragma unroll 1
     for (int b = top; b >= 0; --b) {
         const uint32_t cand = vkey | (1u << b);
-        if (__reduce_add_sync(kFull, count_lt<NR>(rk, cand)) < want) vkey = cand;
+        const uint32_t c = __reduce_add_sync(kFull, count_lt<NR>(rk, cand));
+        if (c < want) {
+            vkey = cand;
+        } else if (c <= want + slack && slack) {
+            early = cand;
+            break;
+        }
     }
-    uint32_t less = 0, eq = 0, mx = 0;
-#pragma unroll
-    for (int u = 0; u < NR; ++u) {
-        const bool valid = u * 32 + (int)lane < n;
-        less += (rk[u] < vkey) ? 1u : 0u;
-        const bool e = valid && rk[u] == vkey;
-        eq += e ? 1u : 0u;
-        mx = e ? max(mx, ri[u]) : mx;
-    }
-    less = __reduce_add_sync(kFull, less);
-    eq = __reduce_add_sync(kFull, eq);
-    if (ties_out) *ties_out = eq;
-    const uint32_t need = want - less;  // ties of vkey to keep, in index order
     uint32_t vidx;
-    if (eq == need) {
-        vidx = __reduce_max_sync(kFull, mx);
+    if (early) {  // keep every pair with key < early
+        vkey = early - 1u;
+        vidx = 0xffffffffu;
+        if (ties_out) *ties_out = 0;
     } else {
-        vidx = 0;
-#pragma unroll 1
-        for (int b = 31; b >= 0; --b) {
-            const uint32_t cand = vidx | (1u << b);
-            uint32_t c = 0;
+        uint32_t less = 0, eq = 0, mx = 0;
 #pragma unroll
-            for (int u = 0; u < NR; ++u)
-                c += (u * 32 + (int)lane < n && rk[u] == vkey && ri[u] < cand) ? 1u : 0u;
-            if (__reduce_add_sync(kFull, c) < need) vidx = cand;
+        for (int u = 0; u < NR; ++u) {
+            const bool valid = u * 32 + (int)lane < n;
+            less += (rk[u] < vkey) ? 1u : 0u;
+            const bool e = valid && rk[u] == vkey;
+            eq += e ? 1u : 0u;
+            mx = e ? max(mx, ri[u]) : mx;
+        }
+        less = __reduce_add_sync(kFull, less);
+        eq = __reduce_add_sync(kFull, eq);
+        if (ties_out) *ties_out = eq;
+        const uint32_t need = want - less;  // ties of vkey to keep, in index order
+        if (eq == need) {
+            vidx = __reduce_max_sync(kFull, mx);
+        } else {
+            vidx = 0;
+#pragma unroll 1
+            for (int b = 31; b >= 0; --b) {
+                const uint32_t cand = vidx | (1u << b);
+                uint32_t c = 0;
+#pragma unroll
+                for (int u = 0; u < NR; ++u)
+                    c += (u * 32 + (int)lane < n && rk[u] == vkey && ri[u] < cand) ? 1u : 0u;
+                if (__reduce_add_sync(kFull, c) < need) vidx = cand;
+            }
         }
     }
     // compaction in place: keep (key, idx) <= (vkey, vidx); every lane's loads above
@@ -281,7 +300,7 @@ __device__ __noinline__ unsigned long long pool_narrow_regs(uint32_t* __restrict
     }
     __syncwarp();
     *n_out = w;
-    return ((unsigned long long)vkey << 32) | vidx;
+    return ((unsigned long long)vkey << 32) | (early ? 0x7ffffffeu : vidx);
 }
 
 // Same as pool_narrow_regs for a pool of packed pairs (key << 32 | idx) in one

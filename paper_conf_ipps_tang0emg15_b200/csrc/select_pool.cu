@@ -233,13 +233,13 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
     // warp uses the exact lexicographic test, which keeps tied rows (few distinct
     // values) from filling the pool with equal keys.
     bool exact_ties = (order_mode & 4) != 0;  // KSEL_LOOSE=1 experiment: exact from the start
-    auto narrow = [&]() {
+    auto narrow = [&](uint32_t slack) {
         unsigned long long t;
         uint32_t ties = 0;
         if constexpr (Cfg::kPool <= 32 * 24) {
             // small pools: register-resident bisection (no histogram atomics)
             int nn;
-            t = pool_narrow_regs<Cfg::kPool / 32>(pk, pi, n, (uint32_t)k, &nn, &ties);
+            t = pool_narrow_regs<Cfg::kPool / 32>(pk, pi, n, (uint32_t)k, &nn, &ties, slack);
             n = nn;
         } else {
             t = pool_kth(pk, pi, n, (uint32_t)k, hist, &ties);
@@ -285,7 +285,12 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
         uint32_t total;
         const uint32_t excl = warp_excl_scan(__popc(adm), lane, total);
         if (total == 0) return;
-        if (n + (int)total > Cfg::kPool) narrow();
+        if (n + (int)total > Cfg::kPool) {
+            // stop the narrowing anywhere in [k, k + slack] pairs as long as this sub-step
+            // still fits behind them (slack <= a quarter of the pool's spare room)
+            const int room = Cfg::kPool - k - (int)total;
+            narrow(room > 0 ? (uint32_t)min(room, (Cfg::kPool - k) / 4) : 0u);
+        }
         int pos = n + (int)excl;
         for (uint32_t t = adm; t; t &= t - 1u) {
             const uint32_t e = elem(__ffs(t) - 1);
