@@ -571,6 +571,9 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
             // narrows (and writes them): they derive the same `need` and split it consistently
             pair_bar();
             uint32_t need = __ballot_sync(kFull, qvalid && !failed && n + room > cap && n > target);
+            // mid-stream, any bound with k..k + slack pairs at or below it will do (the
+            // exact k-th is only needed by the final pass): the narrowing stops early
+            const uint32_t slk = final_pass ? 0u : (uint32_t)max(0, (cap - target - room) / 4);
             int turn = 0;
             while (need) {
                 if (PROF) prof_nnarrow++;
@@ -581,11 +584,11 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                 const int jn = __shfl_sync(kFull, n, j);
                 const float jb = __shfl_sync(kFull, band, j);
                 int nn;
-                const unsigned long long t = (jn <= 256)   ? pool_narrow64<8>(jp, jn, (uint32_t)target, &nn, jb)
-                                             : (jn <= 512) ? pool_narrow64<16>(jp, jn, (uint32_t)target, &nn, jb)
-                                             : (jn <= 32 * kNarrowRegs)
-                                                 ? pool_narrow64<kNarrowRegs>(jp, jn, (uint32_t)target, &nn, jb)
-                                                 : pool_select64(jp, jn, (uint32_t)target, hist, &nn, jb);
+                const unsigned long long t =
+                    (jn <= 256)   ? pool_narrow64<8>(jp, jn, (uint32_t)target, &nn, jb, slk)
+                    : (jn <= 512) ? pool_narrow64<16>(jp, jn, (uint32_t)target, &nn, jb, slk)
+                    : (jn <= 32 * kNarrowRegs) ? pool_narrow64<kNarrowRegs>(jp, jn, (uint32_t)target, &nn, jb, slk)
+                                               : pool_select64(jp, jn, (uint32_t)target, hist, &nn, jb, slk);
                 if ((int)lane == j) {
                     *np = nn;
                     adopt(t);

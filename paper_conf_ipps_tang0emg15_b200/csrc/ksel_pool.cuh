@@ -322,8 +322,10 @@ __device__ __forceinline__ unsigned long long band_bound(unsigned long long T, f
 
 // band >= 0: keep the band above the want-th pair (band_bound); the want-th pair is returned.
 template <int NR, bool GLOBAL = true>
+// slack > 0: stop at the first candidate key c with want <= #{key < c} <= want + slack
+// (as pool_narrow_regs) and return the key-level bound (c - 1, 0x7ffffffe).
 __device__ __noinline__ unsigned long long pool_narrow64(unsigned long long* __restrict__ pool, int n, uint32_t want,
-                                                         int* n_out, float band = -1.f) {
+                                                         int* n_out, float band = -1.f, uint32_t slack = 0) {
     const uint32_t lane = lane_id();
     unsigned long long r[NR];
     uint32_t kmin = 0xffffffffu, kmax = 0u;
@@ -345,37 +347,49 @@ __device__ __noinline__ unsigned long long pool_narrow64(unsigned long long* __r
     uint32_t hk[NR];  // the key halves (pads: 0xffffffff, never below)
 #pragma unroll
     for (int u = 0; u < NR; ++u) hk[u] = (uint32_t)(r[u] >> 32);
+    uint32_t early = 0;
 #pragma unroll 1
     for (int b = top; b >= 0; --b) {
         const uint32_t cand = vkey | (1u << b);
-        if (__reduce_add_sync(kFull, count_lt<NR>(hk, cand)) < want) vkey = cand;
+        const uint32_t c = __reduce_add_sync(kFull, count_lt<NR>(hk, cand));
+        if (c < want) {
+            vkey = cand;
+        } else if (c <= want + slack && slack) {
+            early = cand;
+            break;
+        }
     }
-    uint32_t less = 0, eq = 0, mx = 0;
-#pragma unroll
-    for (int u = 0; u < NR; ++u) {
-        const bool valid = u * 32 + (int)lane < n;
-        const uint32_t kk = (uint32_t)(r[u] >> 32);
-        less += (valid && kk < vkey) ? 1u : 0u;
-        const bool e = valid && kk == vkey;
-        eq += e ? 1u : 0u;
-        mx = e ? max(mx, (uint32_t)r[u]) : mx;
-    }
-    less = __reduce_add_sync(kFull, less);
-    eq = __reduce_add_sync(kFull, eq);
-    const uint32_t need = want - less;
     uint32_t vidx;
-    if (eq == need) {
-        vidx = __reduce_max_sync(kFull, mx);
+    if (early) {
+        vkey = early - 1u;
+        vidx = 0x7ffffffeu;
     } else {
-        vidx = 0;
-#pragma unroll 1
-        for (int b = 31; b >= 0; --b) {
-            const uint32_t cand = vidx | (1u << b);
-            uint32_t c = 0;
+        uint32_t less = 0, eq = 0, mx = 0;
 #pragma unroll
-            for (int u = 0; u < NR; ++u)
-                c += (u * 32 + (int)lane < n && (uint32_t)(r[u] >> 32) == vkey && (uint32_t)r[u] < cand) ? 1u : 0u;
-            if (__reduce_add_sync(kFull, c) < need) vidx = cand;
+        for (int u = 0; u < NR; ++u) {
+            const bool valid = u * 32 + (int)lane < n;
+            const uint32_t kk = (uint32_t)(r[u] >> 32);
+            less += (valid && kk < vkey) ? 1u : 0u;
+            const bool e = valid && kk == vkey;
+            eq += e ? 1u : 0u;
+            mx = e ? max(mx, (uint32_t)r[u]) : mx;
+        }
+        less = __reduce_add_sync(kFull, less);
+        eq = __reduce_add_sync(kFull, eq);
+        const uint32_t need = want - less;
+        if (eq == need) {
+            vidx = __reduce_max_sync(kFull, mx);
+        } else {
+            vidx = 0;
+#pragma unroll 1
+            for (int b = 31; b >= 0; --b) {
+                const uint32_t cand = vidx | (1u << b);
+                uint32_t c = 0;
+#pragma unroll
+                for (int u = 0; u < NR; ++u)
+                    c += (u * 32 + (int)lane < n && (uint32_t)(r[u] >> 32) == vkey && (uint32_t)r[u] < cand) ? 1u : 0u;
+                if (__reduce_add_sync(kFull, c) < need) vidx = cand;
+            }
         }
     }
     const unsigned long long T = ((unsigned long long)vkey << 32) | vidx;
@@ -420,9 +434,13 @@ __device__ __forceinline__ void pool_scan64(const unsigned long long* __restrict
 // common prefix of the pool's smallest and largest key (distances share their
 // top bits), then of the index for ties; shared-memory histogram `hist` (256 u32,
 // transposed layout).  The pool is then compacted in place to the pairs <= it.
+// slack > 0: stop after the first key digit whose bucket, with everything below it,
+// holds at most want + slack pairs; the bound is then (bucket's last key, 0x7ffffffe).
 __device__ __noinline__ static unsigned long long pool_select64(unsigned long long* __restrict__ pool, int n,
                                                                uint32_t want, uint32_t* __restrict__ hist,
-                                                               int* n_out, float band = -1.f) {
+                                                               int* n_out, float band = -1.f, uint32_t slack = 0) {
+    const uint32_t want0 = want;
+    bool early = false;
     const uint32_t lane = lane_id();
     uint32_t kmin = 0xffffffffu, kmax = 0u;
     pool_scan64(pool, n, lane, [&](unsigned long long v) {
@@ -451,11 +469,18 @@ __device__ __noinline__ static unsigned long long pool_select64(unsigned long lo
         const uint32_t d = hist_find(hist, lane, want, cnt);
         prefix |= d << lo;
         __syncwarp();
+        if (slack && (want0 - want) + cnt <= want0 + slack) {  // take the whole bucket
+            prefix |= (1u << lo) - 1u;
+            early = true;
+            break;
+        }
         hi = lo - 1;
     }
     const uint32_t vkey = prefix;
     uint32_t vidx;
-    if (cnt == want) {
+    if (early) {
+        vidx = 0x7ffffffeu;
+    } else if (cnt == want) {
         uint32_t m = 0;
         pool_scan64(pool, n, lane, [&](unsigned long long v) {
             if ((uint32_t)(v >> 32) == vkey) m = max(m, (uint32_t)v);

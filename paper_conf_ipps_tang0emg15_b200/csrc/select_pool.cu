@@ -364,15 +364,25 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
             kmax = __reduce_max_sync(kFull, kmax);
             const int top = (kmin == kmax) ? -1 : 31 - __clz(kmin ^ kmax);
             uint32_t vkey = (top < 0) ? kmin : (kmin & ~((2u << top) - 1u));
+            // (stops early at a candidate key with k..k + k/4 keys below it: any key with
+            // >= k keys at or below it is a valid starting bound)
+            uint32_t early = 0;
+            const uint32_t kslack = (uint32_t)k + max(8u, (uint32_t)k / 4u);
 #pragma unroll 1
             for (int bit = top; bit >= kLow; --bit) {
                 const uint32_t cand = vkey | (1u << bit);
                 uint32_t c = 0;
 #pragma unroll
                 for (int j = 0; j < NB * CH / 128 * 4; ++j) c += (keys[j] < cand) ? 1u : 0u;
-                if (__reduce_add_sync(kFull, c) < (uint32_t)k) vkey = cand;
+                c = __reduce_add_sync(kFull, c);
+                if (c < (uint32_t)k) {
+                    vkey = cand;
+                } else if (c <= kslack) {
+                    early = cand;
+                    break;
+                }
             }
-            const uint32_t bkey = (top >= kLow) ? (vkey | ((1u << kLow) - 1u)) : kmax;
+            const uint32_t bkey = early ? early - 1u : (top >= kLow) ? (vkey | ((1u << kLow) - 1u)) : kmax;
             tighten(bkey, 0x7ffffffeu);
             if (WPR > 1 && lane == 0) atomicMin(grp_thr, ((unsigned long long)bkey << 32) | 0x7ffffffeu);
         }
