@@ -71,10 +71,14 @@ __device__ __forceinline__ uint32_t hist_find(const uint32_t* hist, uint32_t lan
 // Exact want-th smallest (key, idx) pair among pool[0..n), want in [1, n].
 // MSD radix select, 8-bit digits: 4 passes over the key, then (only if the
 // k-th key value is tied beyond the rank needed) 4 passes over the index.
+// slack > 0: stop after the first key digit whose bucket, with everything below it, holds
+// at most want + slack pairs, and return (that bucket's last key, 0x7ffffffe): a valid
+// (>= want pairs at or below it) but not exact bound, for mid-stream narrowings.
 __device__ __noinline__ static unsigned long long pool_kth(const uint32_t* __restrict__ pk, const uint32_t* __restrict__ pi,
                                                     int n, uint32_t want, uint32_t* __restrict__ hist,
-                                                    uint32_t* ties_out = nullptr) {
+                                                    uint32_t* ties_out = nullptr, uint32_t slack = 0) {
     const uint32_t lane = lane_id();
+    const uint32_t want0 = want;
     // Digits above the highest bit where the pool's smallest and largest keys differ
     // are common to all keys: start at the pass holding that bit (pools of keys near
     // one bound usually share their top byte or two).
@@ -110,6 +114,10 @@ __device__ __noinline__ static unsigned long long pool_kth(const uint32_t* __res
         const uint32_t d = hist_find(hist, lane, want, cnt);
         prefix |= d << shift;
         __syncwarp();
+        if (slack && shift > 0 && (want0 - want) + cnt <= want0 + slack) {  // take the whole bucket
+            if (ties_out) *ties_out = 0;
+            return ((unsigned long long)(prefix | ((1u << shift) - 1u)) << 32) | 0x7ffffffeu;
+        }
     }
     const uint32_t vkey = prefix;
     if (ties_out) *ties_out = cnt;  // pool entries whose key equals the k-th key

@@ -242,7 +242,7 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
             t = pool_narrow_regs<Cfg::kPool / 32>(pk, pi, n, (uint32_t)k, &nn, &ties, slack);
             n = nn;
         } else {
-            t = pool_kth(pk, pi, n, (uint32_t)k, hist, &ties);
+            t = pool_kth(pk, pi, n, (uint32_t)k, hist, &ties, slack);
             n = pool_compact(pk, pi, n, (uint32_t)(t >> 32), (uint32_t)t);
         }
         if (ties > 16u) exact_ties = true;
