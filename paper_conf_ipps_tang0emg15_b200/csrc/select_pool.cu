@@ -367,7 +367,7 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
             // (stops early at a candidate key with k..k + k/4 keys below it: any key with
             // >= k keys at or below it is a valid starting bound)
             uint32_t early = 0;
-            const uint32_t kslack = (uint32_t)k + max(8u, (uint32_t)k / 4u);
+            const uint32_t kslack = (uint32_t)k + (uint32_t)k / 4u;
 #pragma unroll 1
             for (int bit = top; bit >= kLow; --bit) {
                 const uint32_t cand = vkey | (1u << bit);
