@@ -71,11 +71,11 @@ int env_int(const char* name, int dflt) {
 }
 
 int chunk_order_mode() {
-    // bits 0-1: chunk visit order (KSEL_ORDER, default 2); bit 2: loose admission
+    // bits 0-1: chunk visit order (KSEL_ORDER, default 3); bit 2: loose admission
     // experiment (KSEL_LOOSE=1).  Experiments only; the defaults are the product.
     static const int mode = [] {
         const char* e = std::getenv("KSEL_ORDER");
-        int m = (e && (e[0] == '0' || e[0] == '1' || e[0] == '2')) ? e[0] - '0' : 2;
+        int m = (e && e[0] >= '0' && e[0] <= '3') ? e[0] - '0' : 3;
         const char* l = std::getenv("KSEL_LOOSE");
         if (l && l[0] == '1') m |= 4;
 #ifdef KSEL_EXPERIMENTS

@@ -155,13 +155,16 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
     const uint64_t c_end = nch * (wig + 1) / WPR;
     const int nmine = (int)(c_end - c_begin);
 
-    // Visit order: first a "spread prologue" of NP chunks evenly spaced over the
-    // warp's range (c = i * step), then every other chunk in address order.  The
-    // prologue gives the running threshold a representative sample of the whole
-    // range early, so sorted or trending rows (which an in-order scan would
-    // admit entirely, e.g. descending rows) are filtered like random ones, while
-    // the bulk of the traffic stays sequential for DRAM locality.  The result
-    // does not depend on the order.  Only the issuing lane walks the order
+    // Visit order of the warp's chunks (KSEL_ORDER; the result does not depend on it).
+    // Default (3, r2): the first chunk, the last L = ceil(k / CH) + 1 chunks, then the
+    // rest in column order.  The first and the last chunks feed the starting bound
+    // (an ascending row's smallest values come first, a descending row's last; L covers
+    // k of them), and the column-order remainder meets a tied row's smallest indices
+    // first, so the exact (key, index) bound settles at once.  Measured against mode 2
+    // (first, last, then a golden-ratio stride permutation, round 1's default): C2 tied
+    // rows T/X -15..26 % at k >= 256, sorted rows -27 % at k = 1024, U/G/DG -1..4 %,
+    // C3 -2.6 %.  Mode 1: a spread prologue of 16 evenly spaced chunks, then column
+    // order; mode 0: column order.  Only the issuing lane walks the order
     // (incrementally, no divisions); the chunk id travels with the stage.
     const uint32_t nm = (uint32_t)nmine;
     uint32_t np = (nm >= 64u) ? 16u : nm / 4u;
@@ -174,7 +177,16 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
         while (gcd(pstride, nm) != 1u) pstride += 2;
     }
     uint32_t it_i = 0, it_blk = 0, it_off = 1, it_tail = np * step, it_p = 0;
+    const uint32_t tailL = (uint32_t)(k + CH - 1) / CH + 1u;
     auto next_chunk = [&]() -> uint32_t {  // lane 0 only; chunk index relative to c_begin
+        if ((order_mode & 3) == 3) {
+            // the first chunk, the last L (enough for k: a descending row's smallest values),
+            // then the rest in column order -- tied rows meet their smallest indices first
+            if (nm <= tailL + 1u) return it_i++;
+            if (it_i == 0u) return it_i++;
+            if (it_i <= tailL) return nm - (it_i++);
+            return 1u + (it_p++);
+        }
         if ((order_mode & 3) == 2) {
             // the first and the last chunk first (they feed the starting bound: sorted rows,
             // ascending or descending, then start from their exact k-th when k <= 512),

@@ -433,3 +433,40 @@ def test_fuzz_select_host(K, oracle_mod, seed):
         gv, gi = K.ksel_select_host(x, k, workspace=ws)
         ev, ei = oracle_mod.select(x.numpy(), k)
         assert_same(ev, ei, gv.numpy(), gi.numpy(), "host fuzz seed=%d case=%d Q=%d N=%d k=%d %s" % (seed, case, Q, N, k, dist))
+
+
+_ORDER_CHILD = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+import paper_conf_ipps_tang0emg15_b200 as K, synth
+out = {}
+for dist in ("U", "T", "SA", "SD", "X"):
+    x = synth.rows(dist, 61, 0, 300, 20011, device="cuda")
+    for k in (1, 100, 1024):
+        for wpr in (0, 1, 4):
+            v, i = K.ksel_select(x, k, algo=2, warps_per_row=wpr)
+            out["%s_%d_%d_v" % (dist, k, wpr)] = v.cpu().numpy()
+            out["%s_%d_%d_i" % (dist, k, wpr)] = i.cpu().numpy()
+np.savez(sys.argv[2], **out)
+"""
+
+
+@pytest.mark.parametrize("order", ["0", "1", "2", "3"])
+def test_chunk_visit_orders_bit_exact(oracle_mod, order, tmp_path):
+    # the chunk visit order (KSEL_ORDER, read once per process; default 3) changes only
+    # which candidates are admitted when, never the result
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    f = str(tmp_path / "res.npz")
+    env = dict(os.environ, KSEL_ORDER=order)
+    subprocess.run([sys.executable, "-c", _ORDER_CHILD, root, f], env=env, check=True, timeout=600)
+    res = np.load(f)
+    for dist in ("U", "T", "SA", "SD", "X"):
+        x = synth.rows(dist, 61, 0, 300, 20011).numpy()
+        for k in (1, 100, 1024):
+            ev, ei = oracle_mod.select(x, k)
+            for wpr in (0, 1, 4):
+                assert_same(ev, ei, res["%s_%d_%d_v" % (dist, k, wpr)], res["%s_%d_%d_i" % (dist, k, wpr)],
+                            "KSEL_ORDER=%s %s k=%d wpr=%d" % (order, dist, k, wpr))
