@@ -1009,6 +1009,13 @@ static cudaError_t knn_run(const float* ref, const float* query, int64_t N, int6
             ref, query + q0 * (int64_t)D, g, nt, ref_img, q_img, qstat, stats);
         note_launch();
         e = cudaGetLastError();
+#ifdef KSEL_EXPERIMENTS
+        // experiment: keep the previous call's final bounds (same inputs: the best bounds
+        // the filter could start from -- an upper limit on what better bounds can gain;
+        // profiles/r02_knn_bounds_exp.txt)
+        static const bool keep_thr = env_int("KSEL_KNN_KEEPTHR", 0) == 1;
+        if (!keep_thr)
+#endif
         if (e == cudaSuccess) e = cudaMemsetAsync(work + w.qthr, 0xff, (size_t)nq * 8, stream);  // "no bound yet"
         if (e == cudaSuccess) e = cudaMemsetAsync(work + w.qfail, 0, (size_t)nq * 4, stream);
         if (e != cudaSuccess) return e;

@@ -23,7 +23,7 @@ ap.add_argument("--save", default="")
 a = ap.parse_args()
 ref = synth.knn_points(a.kind, 41, 0, a.N, a.D, device="cuda")
 qry = synth.knn_points(a.kind, 42, 0, a.Q, a.D, device="cuda")
-ws = torch.empty(K.knn_search_workspace(a.N, a.Q, a.D, a.k), dtype=torch.uint8, device="cuda")
+ws = torch.full((K.knn_search_workspace(a.N, a.Q, a.D, a.k),), 255, dtype=torch.uint8, device="cuda")
 ov = torch.empty((a.Q, a.k), dtype=torch.float32, device="cuda")
 oi = torch.empty((a.Q, a.k), dtype=torch.int32, device="cuda")
 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
