@@ -470,3 +470,28 @@ def test_chunk_visit_orders_bit_exact(oracle_mod, order, tmp_path):
             for wpr in (0, 1, 4):
                 assert_same(ev, ei, res["%s_%d_%d_v" % (dist, k, wpr)], res["%s_%d_%d_i" % (dist, k, wpr)],
                             "KSEL_ORDER=%s %s k=%d wpr=%d" % (order, dist, k, wpr))
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_fuzz_clustered_ties_many_narrowings(K, oracle_mod, seed):
+    # rows long enough for many mid-stream narrowings (which stop early at a valid, not
+    # exact, bound) with values drawn from a few hundred levels -- tie runs of random length
+    # straddle every rank a narrowing may stop at -- plus -0.0/+0.0, +-Inf and NaN sprinkled in
+    rng = np.random.default_rng(7000 + seed)
+    for case in range(3):
+        Q = int(rng.integers(3, 40))
+        N = int(rng.integers(60000, 260000))
+        levels = np.sort(rng.standard_normal(int(rng.integers(20, 400))).astype(np.float32))
+        x = levels[rng.integers(0, levels.size, size=(Q, N))]
+        specials = np.array([0.0, -0.0, np.inf, -np.inf, np.nan], dtype=np.float32)
+        mask = rng.random((Q, N)) < 0.002
+        x[mask] = specials[rng.integers(0, specials.size, size=int(mask.sum()))]
+        x_cpu = torch.from_numpy(np.ascontiguousarray(x))
+        xg = x_cpu.cuda()
+        for k in (int(rng.integers(1, 64)), int(rng.integers(64, 600)), int(rng.integers(600, 1025))):
+            ev, ei = oracle_mod.select(x, k)
+            for algo, wpr in ((0, 0), (2, 1), (2, 2), (2, 8)):
+                gv, gi = K.ksel_select(xg, k, algo=algo, warps_per_row=wpr)
+                torch.cuda.synchronize()
+                assert_same(ev, ei, gv, gi, "clustered seed=%d case=%d Q=%d N=%d k=%d algo=%d wpr=%d"
+                            % (seed, case, Q, N, k, algo, wpr))
