@@ -933,8 +933,12 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
         if (cost < best_cost) { best_cost = cost; best = s; }
     }
     g.S = best;
-    static const int coldw_env = env_int("KSEL_KNN_COLDW", 1000);  // experiments: first-wave split weight (per mille)
-    g.cold_w = (coldw_env > 0 && coldw_env <= 1000) ? coldw_env : 1000;
+    // first-wave (cold) splits take twice the references of the others: their published
+    // k-th then covers more of each query's row before the later splits start from it
+    // (late r2, run_knn.py: C4 filter 6.03 -> 5.84 ms, k = 1024 13.66 -> 13.20 ms; 1.5x
+    // and 2.5-4x measured worse on one of the two)
+    static const int coldw_env = env_int("KSEL_KNN_COLDW", 2000);  // first-wave split weight (per mille)
+    g.cold_w = (coldw_env > 0 && coldw_env <= 8000) ? coldw_env : 2000;
     static const int splits_env = env_int("KSEL_KNN_SPLITS", 0);  // experiments: force the split count
     if (splits_env > 0) {
         g.S = std::min(splits_env, smax);
