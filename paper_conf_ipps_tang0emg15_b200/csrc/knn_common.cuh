@@ -59,7 +59,8 @@ struct KnnRescoreArgs {
     const int32_t* cnt;                // [S][Q]
     int S;                             // lists per query (reference splits x column halves)
     const unsigned long long* thr;     // [Q] tightest published k-th (d~, row) pair
-    const int32_t* qfail;              // [Q] band overflowed: exact fallback
+    int32_t* qfail;                    // [Q] band overflowed / speculation unverified: exact fallback
+    const unsigned long long* spec;    // [Q] speculative starting bound T_spec (nullptr: none)
     const float4* qstat;               // [Q] (-, -, -, |q|^2)
     const KnnStats* stats;
     uint8_t* fb;                       // fallback workspace

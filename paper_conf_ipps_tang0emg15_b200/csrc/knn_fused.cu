@@ -38,6 +38,7 @@
 //     (atomicMin) so all splits share bounds.
 //   * queries are processed in chunks so that the pools stay below 2 GiB.
 #include <algorithm>
+#include <cmath>
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
@@ -348,7 +349,8 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
     knn_fused_kernel(KnnGeom g, const uint8_t* __restrict__ ref_img, const uint8_t* __restrict__ q_img,
                      const float4* __restrict__ qstat, const KnnStats* __restrict__ st,
                      unsigned long long* __restrict__ pool64, int32_t* __restrict__ cnt_out,
-                     unsigned long long* __restrict__ qthr, int32_t* __restrict__ qfail, float* __restrict__ dump) {
+                     unsigned long long* __restrict__ qthr, int32_t* __restrict__ qfail, float* __restrict__ dump,
+                     const unsigned long long* __restrict__ qspec) {
     constexpr int HALVES = (QPC == 1) ? EW / 4 : 1;
     constexpr int WCOLS = BN / HALVES;  // columns of each tile this epilogue warp scans
     constexpr int SB = 2 * KNN_KS * BN * 2;   // bytes of one reference stage
@@ -389,7 +391,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
     // Cold CTAs (the first wave: no split of their queries has published a bound
     // yet) first stream their first Fs tiles through the pipeline for a distance
     // histogram per query (starting bound, see the epilogue), then all t1 - t0.
-    const int Fs = (!DUMP && !PIPE_ONLY && (int)blockIdx.x < g.sample_ctas && g.k <= BN && g.tstride == 1 &&
+    const int Fs = (!DUMP && !PIPE_ONLY && qspec == nullptr && (int)blockIdx.x < g.sample_ctas && g.k <= BN && g.tstride == 1 &&
                     t1 - t0 >= 4 * g.sample_tiles && (int64_t)(t0 + g.sample_tiles) * BN <= g.N)
                        ? g.sample_tiles
                        : 0;
@@ -551,6 +553,15 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                 if (PAIR > 1) atomicMin(Tp, t);
             }
         };
+        // Speculative start (knn_run's sampled pre-pass): T_spec, the j-th smallest d~ of a
+        // strided sample, is very likely above the row's k-th d~ -- admitting against it from
+        // the first tile replaces the slow convergence of S independent running bounds.
+        // Unverified here: knn_rescore_kernel checks that >= k pooled pairs are <= T_spec
+        // (else the query takes the exact fallback).
+        if (qspec != nullptr && qvalid && !DUMP && !PIPE_ONLY) {
+            const unsigned long long ts = __ldg(qspec + q);
+            if ((uint32_t)(ts >> 32) != kSentKey) set_T(ts);
+        }
         // after a pair barrier: the pair's shared bound and failure flag
         auto refresh = [&]() {
             if constexpr (PAIR > 1) {
@@ -835,7 +846,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
 static size_t al256(size_t x) { return (x + 255u) & ~(size_t)255u; }
 
 struct KnnWork {
-    size_t ref_img, stats, q_img, qstat, pool, cnt, qthr, qfail, fb, prof, total;
+    size_t ref_img, stats, q_img, qstat, pool, cnt, qthr, qspec, qfail, fb, prof, total;
 };
 
 // Queries are processed in chunks (multiples of 128 queries) so that the pools,
@@ -948,6 +959,39 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     return g;
 }
 
+// Speculative bounds (late r2).  With S splits per query, each split's running bound
+// converges on its own 1/S of the references, so a query admits ~S k ln(N / (S k))
+// candidates (C4: ~6200 per query, 60x its k) and almost every 32 x 32 epilogue chunk
+// takes the rare path.  A pre-pass of the same kernel over a strided sample of m = ms x BN
+// references (S = 1, target j) yields T_spec = the j-th smallest sampled d~.  The count
+// of ALL references with d~ <= T_spec is ~ (N / m) Gamma(j); j = lambda + 6 sqrt(lambda) + 6
+// with lambda = k m / N (the count's expected k-th position in the sample) makes
+// P(count < k) < 1e-10 on i.i.d. rows.  The main pass admits against T_spec from its first
+// tile; knn_rescore_kernel verifies it (>= k pooled pairs <= T_spec, or a published
+// bound <= T_spec), else the query takes the exact fallback -- exact either way.
+static int knn_spec_tiles(const KnnGeom& g) {
+    static const int env = env_int("KSEL_KNN_SPEC", 64);  // sampled tiles (0: off)
+    if (env <= 0 || g.NT < 16 * env || g.tstride != 1) return 0;
+    return env;
+}
+static KnnGeom knn_spec_geometry(const KnnGeom& g, int ms) {
+    KnnGeom p = g;
+    const double lam = (double)g.k * (double)ms * g.BN / (double)g.N;
+    int j = (int)std::ceil(lam + 6.0 * std::sqrt(lam) + 6.0);
+    p.k = std::min(j, KNN_BN);
+    const int kk = p.k < 32 ? 32 : p.k;
+    const int P = (kk <= 128) ? 1152 : kk + 8 * 256;
+    p.P = (P + 31) / 32 * 32;
+    p.pcap = std::max(kk + 32 + g.BN, std::min(p.P, kk <= 128 ? 512 : p.P));
+    p.ntiles = ms;
+    p.tstride = g.NT / ms;
+    p.S = 1;
+    p.sample_tiles = 0;
+    p.sample_ctas = 0;
+    p.cold_splits = 0;
+    return p;
+}
+
 static KnnWork knn_work_layout(const KnnGeom& g) {
     KnnWork w{};
     size_t off = 0;
@@ -958,6 +1002,7 @@ static KnnWork knn_work_layout(const KnnGeom& g) {
     w.pool = off;    off += al256((size_t)g.S * g.Q * g.P * 8);  // one pool per (split, query)
     w.cnt = off;     off += al256((size_t)g.S * g.Q * 4);
     w.qthr = off;    off += al256((size_t)g.Q * 8);
+    w.qspec = off;   off += al256((size_t)g.Q * 8);
     w.qfail = off;   off += al256((size_t)g.Q * 4);
     w.fb = off;      off += al256(knn_fallback_bytes(g.k));
     w.prof = off;    off += al256((size_t)g.QTp * g.S * KNN_MAX_EW * 16 * 8);  // MODE 3 counters
@@ -1023,7 +1068,6 @@ static cudaError_t knn_run(const float* ref, const float* query, int64_t N, int6
         if (e == cudaSuccess) e = cudaMemsetAsync(work + w.qthr, 0xff, (size_t)nq * 8, stream);  // "no bound yet"
         if (e == cudaSuccess) e = cudaMemsetAsync(work + w.qfail, 0, (size_t)nq * 4, stream);
         if (e != cudaSuccess) return e;
-        const int smem = KnnSmem::total(g);
         float* kdump = dump ? dump + q0 * N : nullptr;
 #ifdef KSEL_EXPERIMENTS
         // Timing experiments only (a -DKSEL_EXPERIMENTS build; the product library has none of
@@ -1044,35 +1088,54 @@ static cudaError_t knn_run(const float* ref, const float* query, int64_t N, int6
                     : mode_env == 3 ? (ew8 ? knn_fused_kernel<3, 8, 256, 1> : knn_fused_kernel<3, 4, 256, 1>)
                     : mode_env == 4 ? knn_fused_kernel<4, 4, 256, 1>
                                     : (ew8 ? knn_fused_kernel<0, 8, 256, 1> : knn_fused_kernel<0, 4, 256, 1>);
+        auto sel_kern = (g.QPC == 2) ? knn_fused_kernel<0, 8, 128, 2>
+                                     : (ew8 ? knn_fused_kernel<0, 8, 256, 1> : knn_fused_kernel<0, 4, 256, 1>);
         if (!dump && mode_env == 3) kdump = reinterpret_cast<float*>(work + w.prof);
 #else
         constexpr int mode_env = 0;
         auto kern = dump ? knn_fused_kernel<1, 8, 256, 1> : knn_fused_kernel<0, 8, 256, 1>;
+        auto sel_kern = knn_fused_kernel<0, 8, 256, 1>;
 #endif
-        e = ensure_smem_attr(reinterpret_cast<const void*>(kern), smem);
-        if (e != cudaSuccess) return e;
-        const int slot = dump ? -1 : timing_begin(stream);
-        cudaLaunchConfig_t cfg{};
-        cudaLaunchAttribute attr[1];
-        cfg.gridDim = dim3((unsigned)(g.QTp * g.S));
-        cfg.blockDim = dim3((unsigned)knn_threads(g.EW));
-        cfg.dynamicSmemBytes = (size_t)smem;
-        cfg.stream = stream;
-        attr[0].id = cudaLaunchAttributeClusterDimension;
-        attr[0].val.clusterDim.x = (unsigned)g.cs;
-        attr[0].val.clusterDim.y = 1;
-        attr[0].val.clusterDim.z = 1;
-        cfg.attrs = attr;
-        cfg.numAttrs = 1;
-        e = cudaLaunchKernelEx(&cfg, kern, g, reinterpret_cast<const uint8_t*>(ref_img),
-                               reinterpret_cast<const uint8_t*>(q_img), static_cast<const float4*>(qstat),
-                               static_cast<const KnnStats*>(stats), reinterpret_cast<unsigned long long*>(work + w.pool),
-                               reinterpret_cast<int32_t*>(work + w.cnt),
-                               reinterpret_cast<unsigned long long*>(work + w.qthr),
-                               reinterpret_cast<int32_t*>(work + w.qfail), kdump);
-        note_launch();
-        timing_end(slot, stream);
-        if (e == cudaSuccess) e = cudaGetLastError();
+        auto launch = [&](decltype(kern) kf, const KnnGeom& gg, unsigned long long* thr,
+                          const unsigned long long* spec, float* kd, bool timed) -> cudaError_t {
+            const int smem = KnnSmem::total(gg);
+            cudaError_t le = ensure_smem_attr(reinterpret_cast<const void*>(kf), smem);
+            if (le != cudaSuccess) return le;
+            const int slot = timed ? timing_begin(stream) : -1;
+            cudaLaunchConfig_t cfg{};
+            cudaLaunchAttribute attr[1];
+            cfg.gridDim = dim3((unsigned)(gg.QTp * gg.S));
+            cfg.blockDim = dim3((unsigned)knn_threads(gg.EW));
+            cfg.dynamicSmemBytes = (size_t)smem;
+            cfg.stream = stream;
+            attr[0].id = cudaLaunchAttributeClusterDimension;
+            attr[0].val.clusterDim.x = (unsigned)gg.cs;
+            attr[0].val.clusterDim.y = 1;
+            attr[0].val.clusterDim.z = 1;
+            cfg.attrs = attr;
+            cfg.numAttrs = 1;
+            le = cudaLaunchKernelEx(&cfg, kf, gg, reinterpret_cast<const uint8_t*>(ref_img),
+                                    reinterpret_cast<const uint8_t*>(q_img), static_cast<const float4*>(qstat),
+                                    static_cast<const KnnStats*>(stats),
+                                    reinterpret_cast<unsigned long long*>(work + w.pool),
+                                    reinterpret_cast<int32_t*>(work + w.cnt), thr,
+                                    reinterpret_cast<int32_t*>(work + w.qfail), kd, spec);
+            note_launch();
+            if (timed) timing_end(slot, stream);
+            return le == cudaSuccess ? cudaGetLastError() : le;
+        };
+        // speculative pre-pass (selection only): T_spec per query into qspec
+        const int ms = (dump || mode_env != 0) ? 0 : knn_spec_tiles(g);
+        unsigned long long* qspec = ms > 0 ? reinterpret_cast<unsigned long long*>(work + w.qspec) : nullptr;
+        if (ms > 0) {
+            e = cudaMemsetAsync(qspec, 0xff, (size_t)nq * 8, stream);
+            if (e == cudaSuccess) e = launch(sel_kern, knn_spec_geometry(g, ms), qspec, nullptr, nullptr, false);
+            if (e != cudaSuccess) return e;
+        }
+        // with a speculative start no split is cold: equal splits
+        KnnGeom gm = g;
+        if (ms > 0) gm.cold_splits = 0;
+        e = launch(kern, gm, reinterpret_cast<unsigned long long*>(work + w.qthr), qspec, kdump, !dump);
         if (e != cudaSuccess) return e;
         if (dump) {
             if (dump_eps) {
@@ -1097,7 +1160,8 @@ static cudaError_t knn_run(const float* ref, const float* query, int64_t N, int6
         a.cnt = reinterpret_cast<const int32_t*>(work + w.cnt);
         a.S = g.S;
         a.thr = reinterpret_cast<const unsigned long long*>(work + w.qthr);
-        a.qfail = reinterpret_cast<const int32_t*>(work + w.qfail);
+        a.qfail = reinterpret_cast<int32_t*>(work + w.qfail);
+        a.spec = qspec;
         a.qstat = qstat;
         a.stats = stats;
         a.fb = work + w.fb;

@@ -177,6 +177,27 @@ __global__ void __launch_bounds__(32 * kRsWarps) knn_rescore_kernel(const KnnRes
         int tot = 0;
         for (int s = (int)lane; s < a.S; s += 32) tot += a.cnt[(int64_t)s * a.Q + q];
         tot = __reduce_add_sync(kFull, tot);
+        // A speculative start T_spec (knn_fused.cu knn_spec_geometry) made every split admit
+        // against min(T_spec, its verified bounds).  The pools then hold every reference with
+        // d~ <= min(T_spec, thr) + band, so the band may start from T_spec only once T_spec is
+        // VERIFIED -- at least k pooled pairs <= T_spec -- or from thr if thr <= T_spec.
+        // Otherwise the pools may miss part of the top-k: exact fallback.
+        const unsigned long long ts = a.spec ? a.spec[q] : ~0ull;
+        if ((uint32_t)(ts >> 32) != kSentKey) {
+            int le = 0;
+            for (int s = 0; s < a.S; ++s) {
+                const int ns = a.cnt[(int64_t)s * a.Q + q];
+                const unsigned long long* pr = a.pools + ((int64_t)s * a.Q + q) * a.P;
+                for (int x = (int)lane; x < ns; x += 32) le += (__ldcg(pr + x) <= ts) ? 1 : 0;
+            }
+            le = __reduce_add_sync(kFull, le);
+            if (le >= a.k) {
+                T0 = ts < T0 ? ts : T0;
+            } else if (!(T0 <= ts)) {
+                if (lane == 0) a.qfail[q] = 1;
+                return;
+            }
+        }
         if (tot > kRsCap && tot >= a.k) {  // (a union that fits the buffer is band-narrowed there)
             const uint32_t kk = lists_kth_key(a.pools, a.cnt, a.S, a.Q, q, a.P, (uint32_t)a.k, hist_all[w]);
             const unsigned long long t = ((unsigned long long)kk << 32) | 0xffffffffull;
