@@ -10,28 +10,35 @@ constexpr int KNN_MAX_D = 256;
 
 // Maxima over the reference set (non-negative floats as bits; reset per call).
 struct KnnStats {
-    uint32_t R2;  // max |r|^2 (rounded up)
-    uint32_t pad[3];
+    uint32_t R2;    // max |r'|^2 of the centred references (rounded up)
+    uint32_t isig;  // max 1 / sigma_t over the reference tiles
+    uint32_t pad[2];
 };
 
 // eps_q: a rigorous bound on |d~(q, r) - d(q, r)| for every reference r, where d~ is the
-// filter's tensor-core distance (bf16 hi/lo split operands, three MMA passes, norms
-// folded into the fp32 accumulator; knn_fused.cu) and d the exact one (DESIGN.md
-// reading R21).  qs = (-, -, -, |q|^2).
-//   * x = hi + lo + res with |res| <= 2^-16 |x|, and the dropped lo.lo term is
-//     <= 2^-16 (1 + 2^-7) |q_i r_i|: each product of the MMA operands (-2 q_i, r_i) is
-//     off by <= 6.1 2^-16 |q_i r_i|, and sum |q_i r_i| <= |q| |r| <= sqrt(|q|^2 R2);
-//   * fp32 accumulation of 3D products and 6 norm terms, each rounding <= 2^-24 of the
-//     absolute sum <= 2.02 (|q|^2 + |r|^2), and the 24-bit norm splits:
-//     (3D + 16) 2^-23 (|q|^2 + R2), plus (3D + 16) 2^-124 for underflow;
+// filter's tensor-core distance and d the exact one (reading R21).  The filter
+// (knn_fused.cu) centres every point (x' = fl(x - c)), scales each tile by a power of two
+// sigma and rounds to fp16: A = fp16(-2 sigma_q q'), B = fp16(sigma_t r'), one kind::f16
+// MMA pass; the norms |q'|^2, |r'|^2 (double, rounded to fp32, split three ways in bf16)
+// ride in the same fp32 accumulation.  qs = (sigma_q, -, -, |q'|^2), na = |q'|^2, R2 = max
+// |r'|^2.  In unscaled units:
+//   * operand rounding: each fp16 operand is off by <= 2^-11 of itself (normal) or 2^-25
+//     absolute (subnormal); a product -2 q'_i r'_i is off by <= (2^-10 + 2^-22) |2 q'_i r'_i|
+//     plus 2^-25 (|A_i| + |B_i|) / (sigma_q sigma_t) <= 2^-9 / (sigma_q sigma_t) (|A|, |B|
+//     <= 2^15), and sum |q'_i r'_i| <= |q'| |r'| <= sqrt(na R2):
+//     2 (2^-10 + 2^-21) sqrt(na R2) + D 2^-9 / (sigma_q sigma_t,min);
+//   * fp32 accumulation of D products and 6 norm terms, each rounding <= 2^-24 of the
+//     absolute sum <= 2.02 (na + |r'|^2): (D + 16) 2^-23 1.01 (na + R2), plus
+//     (D + 16) 2^-124 / (sigma_q sigma_t,min) for underflow;
+//   * centring (|fl(x - c) - (x - c)| <= 2^-24 |x'|, so d' = |q' - r'|^2 is within
+//     2^-22 (na + |r'|^2) of d) and the 24-bit norm splits: 2^-21 (na + R2);
 // times 2 for safety.  Returned rounded up; +Inf if an input is not finite (the query
 // then takes the exact fallback).
 __device__ __forceinline__ float knn_eps(float4 qs, const KnnStats& st, int D) {
     const double R2 = (double)__uint_as_float(st.R2), nq = (double)qs.w;
-    // (+ (3D + 16) 2^-124: products and partial sums that underflow the fp32 range -- flushed
-    // or denormal in the tensor core -- each lose less than 2^-126)
-    const double e = 2.0 * (6.1 * 0x1p-16 * sqrt(nq * R2) + (double)(3 * D + 16) * 0x1p-23 * (nq + R2) +
-                            (double)(3 * D + 16) * 0x1p-124);
+    const double isq = (double)__uint_as_float(st.isig) / (double)qs.x;  // 1 / (sigma_q sigma_t,min)
+    const double e = 2.0 * ((0x1p-10 + 0x1p-21) * 2.0 * sqrt(nq * R2) + (double)(D + 16) * 0x1p-23 * 1.01 * (nq + R2) +
+                            0x1p-21 * (nq + R2) + ((double)D * 0x1p-9 + (double)(D + 16) * 0x1p-124) * isq);
     const float f = __double2float_ru(e);
     return (f == f) ? f : __int_as_float(0x7f800000);
 }

@@ -44,6 +44,7 @@
 #include <cstring>
 
 #include <cuda_bf16.h>
+#include <cuda_fp16.h>
 #include <cuda_runtime.h>
 
 #include "ksel.h"
@@ -60,7 +61,7 @@ constexpr int KNN_KS = 32;                               // dims per pipeline st
 constexpr int KNN_NORM_A_BYTES = 16 * KNN_BM * 2;         // norm block of a query tile
 // epilogue warps EW: 4 (one per TMEM lane quadrant, all 256 columns of a tile) or
 // 8 (two per quadrant, 128 columns each); + producer + MMA issuer
-constexpr int KNN_MAX_EW = 8;
+constexpr int KNN_MAX_EW = 16;
 __host__ __device__ constexpr int knn_threads(int ew) { return 64 + 32 * ew; }
 constexpr int KNN_SB = 32;                                // sampling histogram buckets
 constexpr int KNN_CW = 64;                                // accumulator columns per epilogue step
@@ -82,7 +83,6 @@ struct KnnGeom {
     int cs;              // cluster size: CTAs (consecutive query tiles, same reference range) that
                          // share every reference stage through one multicast load
     int QTp;             // query tiles padded to a multiple of cs (padding tiles select nothing)
-    int passes;          // 3 (hi.hi + hi.lo + lo.hi); 1 = hi.hi only (experiments: pipeline timing)
     int cold_splits;     // leading splits run by first-wave CTAs (no published bound yet)
     int cold_w;          // their share of the reference tiles relative to the others (per mille)
     // first logical tile of split s: split s weighs cold_w / 1000 if s < cold_splits, else 1
@@ -96,118 +96,237 @@ struct KnnGeom {
     int BN;              // references per tile (accumulator columns): 256, or 128 with QPC = 2
     int QPC;             // query tiles per CTA sharing every reference stage (1 or 2)
     int EW;              // epilogue warps of the launch (4, or 8)
-    __host__ __device__ int stage_bytes() const { return 2 * KNN_KS * BN * 2; }  // hi + lo bf16
+    __host__ __device__ int stage_bytes() const { return KNN_KS * BN * 2; }  // fp16
     __host__ __device__ int norm_b_bytes() const { return 16 * BN * 2; }
     __host__ __device__ size_t tile_bytes() const { return (size_t)KS * stage_bytes() + norm_b_bytes(); }
-    __host__ __device__ int a_bytes() const { return Dp * 512 + KNN_NORM_A_BYTES; }
+    __host__ __device__ int a_bytes() const { return Dp * 256 + KNN_NORM_A_BYTES; }
 };
 
 // ---------------------------------------------------------------------------
-// prologue: bf16 hi/lo split into the UMMA canonical (K-major, no-swizzle) image
+// prologue: centred, per-tile scaled fp16 operands in the UMMA canonical
+// (K-major, no-swizzle) image
 // ---------------------------------------------------------------------------
-// Core matrix = 8 rows x 16 bytes (8 bf16 along K), rows 16 B apart; 8-row
+// Core matrix = 8 rows x 16 bytes (8 halves along K), rows 16 B apart; 8-row
 // groups 128 B apart (SBO); 8-element K chunks ROWS*16 B apart (LBO).
-//   ref image : [tile][stage][hi,lo][4 chunks][256 rows][8]   (32 KB per stage)
-//   query img : [tile][hi,lo][Dp/8 chunks][128 rows][8]
+//   ref image : [tile][stage][4 chunks][256 rows][8] fp16 (16 KB per stage), then the
+//               tile's bf16 norm block [2 chunks][256 rows][8]
+//   query img : [tile][Dp/8 chunks][128 rows][8] fp16, then the bf16 norm block
+//
+// Distances are translation invariant: every point is first centred, x' = fl(x - c)
+// with c the mean of a reference sample (knn_center_kernel), which shrinks |x'| and
+// with it every term of the error bound (U[0,1]^128: |x|^2 ~ 43 -> |x'|^2 ~ 11).  Each
+// tile (256 references / 128 queries) is then scaled by a power of two sigma so that its
+// largest magnitude lands in [2^14, 2^15) (queries: of -2 sigma x'), and rounded to
+// fp16 once -- one kind::f16 MMA pass instead of bf16 hi/lo x 3.  The accumulator holds
+// sigma_q sigma_t d~; the epilogue compares it with the bound scaled the same way and
+// unscales (exactly, powers of two) only the candidates it keeps.
 
 // bf16 pair of two floats (round to nearest even)
 __device__ __forceinline__ uint32_t bf2(float a, float b) {
     return (uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(a)) |
            ((uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(b)) << 16);
 }
+__device__ __forceinline__ uint32_t h2(float a, float b) {
+    return (uint32_t)__half_as_ushort(__float2half_rn(a)) | ((uint32_t)__half_as_ushort(__float2half_rn(b)) << 16);
+}
 
-// One launch builds both operand images: blocks [0, NT) are reference tiles
-// (256 rows), blocks [NT, NT + QT) query tiles (128 rows, scaled by -2).  Each
-// block reads its rows once, 32 dims at a time, coalesced (a warp reads 32
-// consecutive floats of one row) into shared memory; thread i then owns row i:
-// accumulates |x|^2 in double and writes the hi/lo chunks of its row (16 B per
-// thread, consecutive threads -> consecutive 16 B).  Last, the norm block (the
-// extra 16-wide K block): |x|^2 split three ways in bf16 (x = n1 + n2 + n3 to
-// ~2^-24); queries [n1, n2, n3, 1, 1, 1, 0, 0], references [1, 1, 1, n1, n2, n3,
-// 0, 0], second 8-element chunk zero.  Rows past the end are all zeros.
+// c[d] = the mean of a strided sample of <= 16384 reference rows, rounded to a multiple of
+// 2^(ilogb(sd_d) - 4) (sd_d the sample's spread in dim d): any c is exact (it only has to
+// make |x'| small), and a coarse c keeps x' = x - c exact for integer-valued data (then
+// every fp16 operand is exact).  c = 0 for the padding dims.  knn_sum_kernel: block
+// (x, y) adds dims [32x, 32x + 32) of rows y*8 + warp + 256 i of the sample into csum
+// (double atomics; [2][Dp]: sums, sums of squares); knn_center_value turns them into c.
+__global__ void __launch_bounds__(256)
+    knn_sum_kernel(const float* __restrict__ ref, int64_t N, int D, int Dp, double* __restrict__ csum) {
+    __shared__ double part[2][8][33];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int d = blockIdx.x * 32 + lane;
+    const int64_t ns = N < 16384 ? N : 16384;
+    const int64_t stride = N / ns;
+    double s = 0.0, s2 = 0.0;
+    if (d < D)
+        for (int64_t i = (int64_t)blockIdx.y * 8 + warp; i < ns; i += 8 * (int64_t)gridDim.y) {
+            const double v = (double)__ldg(ref + (i * stride) * D + d);
+            s += v;
+            s2 += v * v;
+        }
+    part[0][warp][lane] = s;
+    part[1][warp][lane] = s2;
+    __syncthreads();
+    if (warp == 0 && d < D) {
+        double t = 0.0, t2 = 0.0;
+        for (int w = 0; w < 8; ++w) { t += part[0][w][lane]; t2 += part[1][w][lane]; }
+        atomicAdd(csum + d, t);
+        atomicAdd(csum + Dp + d, t2);
+    }
+}
+__device__ __forceinline__ float knn_center_value(const double* csum, int64_t N, int D, int Dp, int d) {
+    if (d >= D) return 0.f;
+    const double ns = (double)(N < 16384 ? N : 16384);
+    const double m = csum[d] / ns;
+    const double var = csum[Dp + d] / ns - m * m;
+    if (!(fabs(m) < 1e38) || !(var < 1e76)) return 0.f;  // non-finite sample: no centring
+    if (var <= 0.0) return (float)m;
+    const double gstep = ldexp(1.0, ilogb(sqrt(var)) - 4);
+    return (float)(rint(m / gstep) * gstep);
+}
+
 constexpr int KNN_PREP_THREADS = 256;
 
+// knn_stats_kernel: one block per tile (blocks [0, nt): reference tiles of BN rows, then
+// query tiles of 128 rows); a warp per row, coalesced.  Per row |x'|^2 in double (rownorm),
+// per tile max |x'| -> sigma = 2^e with (2 for queries) x max |x'| x sigma in [2^14, 2^15)
+// (tscale for reference tiles, qstat.x for queries), max |r'|^2 and max 1/sigma_t (st).
 __global__ void __launch_bounds__(KNN_PREP_THREADS)
-    knn_prep_kernel(const float* __restrict__ ref, const float* __restrict__ qry, KnnGeom g, int nt,
-                    uint4* __restrict__ ref_img, uint4* __restrict__ q_img, float4* __restrict__ qstat,
-                    KnnStats* __restrict__ st) {
-    // blocks [0, nt): reference tiles (nt = NT on a call's first query chunk, else 0)
-    __shared__ float tile[KNN_BN][KNN_KS + 1];
-    __shared__ uint32_t smax;  // max |r|^2 of this block's references (one global atomic per block)
-    if (threadIdx.x == 0) smax = 0u;
+    knn_stats_kernel(const float* __restrict__ ref, const float* __restrict__ qry, KnnGeom g, int nt,
+                     const double* __restrict__ csum, double* __restrict__ rownorm, float4* __restrict__ qstat,
+                     float* __restrict__ tscale, KnnStats* __restrict__ st) {
+    __shared__ float cs[KNN_MAX_D];
+    __shared__ uint32_t samx, smax;
+    __shared__ int sbad;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tid == 0) { samx = 0u; smax = 0u; sbad = 0; }
+    for (int d = tid; d < g.Dp; d += KNN_PREP_THREADS) cs[d] = knn_center_value(csum, g.N, g.D, g.Dp, d);
+    __syncthreads();
     const bool is_q = blockIdx.x >= (unsigned)nt;
     const int64_t t = is_q ? (int64_t)blockIdx.x - nt : (int64_t)blockIdx.x;
     const int rows = is_q ? KNN_BM : g.BN;
     const int64_t n = is_q ? g.Q : g.N;
     const float* x = is_q ? qry : ref;
-    const float scale = is_q ? -2.f : 1.f;  // exact
+    float mx = 0.f;
+    bool bad = false;
+    uint32_t rmax = 0u;
+    for (int r0 = warp * 4; r0 < rows; r0 += 4 * (KNN_PREP_THREADS / 32)) {
+        double s[4] = {0.0, 0.0, 0.0, 0.0};
+#pragma unroll 2
+        for (int d0 = 0; d0 < g.D; d0 += 32) {
+            const int d = d0 + lane;
+            float v[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                const int64_t gr = t * rows + r0 + u;
+                v[u] = (gr < n && d < g.D) ? __ldg(x + gr * (int64_t)g.D + d) - cs[d] : 0.f;
+            }
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                s[u] += (double)v[u] * (double)v[u];
+                const float a = fabsf(v[u]);
+                bad |= !(a <= 3.4028235e38f);
+                mx = fmaxf(mx, a);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) s[u] += __shfl_xor_sync(kFull, s[u], o);
+            const int64_t gr = t * rows + r0 + u;
+            if (lane == 0 && r0 + u < rows) {
+                rownorm[blockIdx.x * (int64_t)KNN_BN + r0 + u] = s[u];
+                if (gr < n) {
+                    float sr = __double2float_ru(s[u]);
+                    if (!(sr == sr)) sr = __int_as_float(0x7f800000);
+                    if (is_q) qstat[gr] = make_float4(0.f, 0.f, 0.f, sr);
+                    else rmax = max(rmax, __float_as_uint(sr));
+                }
+            }
+        }
+    }
+    mx = __uint_as_float(__reduce_max_sync(kFull, __float_as_uint(mx)));  // (non-negative: bits order)
+    if (lane == 0) {
+        if (mx > 0.f) atomicMax(&samx, __float_as_uint(mx));
+        if (rmax) atomicMax(&smax, rmax);
+    }
+    if (__any_sync(kFull, bad) && lane == 0) sbad = 1;
+    __syncthreads();
+    const float tmx = __uint_as_float(samx);
+    int e = 0;
+    if (!sbad && tmx > 0.f) e = min(max((is_q ? 13 : 14) - ilogbf(tmx), -120), 120);
+    const float sig = ldexpf(1.f, e);
+    if (is_q) {
+        for (int r = tid; r < rows; r += KNN_PREP_THREADS) {
+            const int64_t gr = t * rows + r;
+            if (gr < n) {
+                qstat[gr].x = sig;
+                if (sbad) qstat[gr].w = __int_as_float(0x7f800000);
+            }
+        }
+    } else if (tid == 0) {
+        tscale[t] = sig;
+        atomicMax(&st->R2, sbad ? 0x7f800000u : smax);
+        atomicMax(&st->isig, __float_as_uint(1.f / sig));
+    }
+}
+
+// knn_prep_kernel: the operand images.  Each block reads its tile 32 dims at a time
+// (coalesced: a warp reads 32 consecutive floats of one row) into shared memory; thread i
+// then owns row i and writes its scaled fp16 chunks (16 B per thread, consecutive threads ->
+// consecutive 16 B).  Last, the bf16 norm block (the extra 16-wide K block): |x'|^2 split
+// three ways (n1 + n2 + n3 to ~2^-24), queries [s n1, s n2, s n3, s, s, s, 0, 0],
+// references [s, s, s, s m1, s m2, s m3, 0, 0] (s the tile's sigma; products of powers of
+// two are exact), so the accumulator is sigma_q sigma_t (|q'|^2 + |r'|^2 - 2 q'.r').
+// Rows past the end are all zeros.
+__global__ void __launch_bounds__(KNN_PREP_THREADS)
+    knn_prep_kernel(const float* __restrict__ ref, const float* __restrict__ qry, KnnGeom g, int nt,
+                    const double* __restrict__ csum, const double* __restrict__ rownorm,
+                    const float4* __restrict__ qstat, const float* __restrict__ tscale,
+                    uint4* __restrict__ ref_img, uint4* __restrict__ q_img) {
+    __shared__ float tile[KNN_BN][KNN_KS + 1];
+    __shared__ float cs[KNN_MAX_D];
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    for (int d = tid; d < g.Dp; d += KNN_PREP_THREADS) cs[d] = knn_center_value(csum, g.N, g.D, g.Dp, d);
+    const bool is_q = blockIdx.x >= (unsigned)nt;
+    const int64_t t = is_q ? (int64_t)blockIdx.x - nt : (int64_t)blockIdx.x;
+    const int rows = is_q ? KNN_BM : g.BN;
+    const int64_t n = is_q ? g.Q : g.N;
+    const float* x = is_q ? qry : ref;
     const int64_t row = t * rows + tid;
-    double s = 0.0;
+    const float sig = is_q ? (t * rows < n ? qstat[t * rows].x : 1.f) : tscale[t];
+    const float mul = is_q ? -2.f * sig : sig;  // exact
     for (int ks = 0; ks < g.KS; ++ks) {
+        __syncthreads();
         const int d = ks * KNN_KS + lane;
 #pragma unroll 8
         for (int r = warp; r < rows; r += KNN_PREP_THREADS / 32) {
             const int64_t gr = t * rows + r;
-            tile[r][lane] = (gr < n && d < g.D) ? __ldcs(x + gr * (int64_t)g.D + d) : 0.f;
+            tile[r][lane] = (gr < n && d < g.D) ? __ldcs(x + gr * (int64_t)g.D + d) - cs[d] : 0.f;
         }
         __syncthreads();
         if (tid < rows) {
             uint4* dst;
             int cstride;
-            if (is_q) {  // [hi,lo][Dp/8 chunks][128 rows][8]
+            if (is_q) {  // [Dp/8 chunks][128 rows][8]
                 dst = q_img + t * (int64_t)(g.a_bytes() / 16) + (int64_t)(ks * 4) * KNN_BM + tid;
                 cstride = KNN_BM;
-            } else {     // [stage][hi,lo][4 chunks][BN rows][8]
+            } else {     // [stage][4 chunks][BN rows][8]
                 dst = ref_img + t * (int64_t)(g.tile_bytes() / 16) + (int64_t)ks * (g.stage_bytes() / 16) + tid;
                 cstride = g.BN;
             }
-            const int64_t lo_off = is_q ? (int64_t)(g.Dp / 8) * KNN_BM : 4 * (int64_t)g.BN;
 #pragma unroll
             for (int kc = 0; kc < 4; ++kc) {
-                uint32_t h[4], l[4];
+                uint32_t h[4];
 #pragma unroll
-                for (int p = 0; p < 4; ++p) {
-                    const float v0 = tile[tid][kc * 8 + 2 * p], v1 = tile[tid][kc * 8 + 2 * p + 1];
-                    s += (double)v0 * (double)v0;
-                    s += (double)v1 * (double)v1;
-                    const float x0 = scale * v0, x1 = scale * v1;
-                    const __nv_bfloat16 h0 = __float2bfloat16_rn(x0), h1 = __float2bfloat16_rn(x1);
-                    h[p] = (uint32_t)__bfloat16_as_ushort(h0) | ((uint32_t)__bfloat16_as_ushort(h1) << 16);
-                    l[p] = bf2(x0 - __bfloat162float(h0), x1 - __bfloat162float(h1));
-                }
+                for (int p = 0; p < 4; ++p) h[p] = h2(mul * tile[tid][kc * 8 + 2 * p], mul * tile[tid][kc * 8 + 2 * p + 1]);
                 dst[kc * cstride] = make_uint4(h[0], h[1], h[2], h[3]);
-                dst[lo_off + kc * cstride] = make_uint4(l[0], l[1], l[2], l[3]);
             }
         }
-        __syncthreads();
     }
     if (tid < rows) {
-        // the filter's error bound needs |q|^2 per query and max |r|^2 (rounded up)
-        const float sr = __double2float_ru(s);
-        if (row < n) {
-            if (is_q) qstat[row] = make_float4(0.f, 0.f, 0.f, sr);
-            else atomicMax(&smax, __float_as_uint(sr == sr ? sr : __int_as_float(0x7f800000)));  // block max
-        }
+        const double s = rownorm[blockIdx.x * (int64_t)KNN_BN + tid];
         const float n1 = __bfloat162float(__float2bfloat16_rn((float)s));
         const float n2 = __bfloat162float(__float2bfloat16_rn((float)(s - (double)n1)));
         const float n3 = __bfloat162float(__float2bfloat16_rn((float)(s - (double)n1 - (double)n2)));
-        const float one = (row < n) ? 1.f : 0.f;
         uint4* blk;
         uint4 c0;
         if (is_q) {
-            blk = q_img + (t * (int64_t)g.a_bytes() + (int64_t)g.Dp * 512) / 16;
-            c0 = make_uint4(bf2(n1, n2), bf2(n3, one), bf2(one, one), 0u);
+            blk = q_img + (t * (int64_t)g.a_bytes() + (int64_t)g.Dp * 256) / 16;
+            c0 = make_uint4(bf2(sig * n1, sig * n2), bf2(sig * n3, sig), bf2(sig, sig), 0u);
         } else {
             blk = ref_img + (t * (int64_t)g.tile_bytes() + (int64_t)g.KS * g.stage_bytes()) / 16;
-            c0 = make_uint4(bf2(one, one), bf2(one, n1), bf2(n2, n3), 0u);
+            c0 = make_uint4(bf2(sig, sig), bf2(sig, sig * n1), bf2(sig * n2, sig * n3), 0u);
         }
+        if (row >= n) c0 = make_uint4(0u, 0u, 0u, 0u);
         blk[tid] = c0;
         blk[rows + tid] = make_uint4(0u, 0u, 0u, 0u);
-    }
-    if (!is_q) {  // (uniform per block)
-        __syncthreads();
-        if (tid == 0 && smax) atomicMax(&st->R2, smax);
     }
 }
 
@@ -223,6 +342,11 @@ __device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint
 // kind::f16 instruction descriptor: bf16 x bf16 -> fp32, K-major A and B, M x N
 __host__ __device__ constexpr uint32_t umma_idesc_bf16(int M, int N) {
     return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+}
+
+// kind::f16 instruction descriptor: fp16 x fp16 -> fp32 (a/b format 0), K-major, M x N
+__host__ __device__ constexpr uint32_t umma_idesc_f16(int M, int N) {
+    return (1u << 4) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
 }
 
 __device__ __forceinline__ void umma_bf16(uint32_t d_tmem, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
@@ -285,6 +409,13 @@ __device__ __forceinline__ void tmem_wait32(uint32_t (&v)[32]) {
                    "+r"(v[29]), "+r"(v[30]), "+r"(v[31])
                  :
                  : "memory");
+}
+
+// min of three floats in one instruction (sm_100: FMNMX3; a NaN operand is ignored like fminf)
+__device__ __forceinline__ float fmin3(float a, float b, float c) {
+    float r;
+    asm("min.f32 %0, %1, %2, %3;" : "=f"(r) : "f"(a), "f"(b), "f"(c));
+    return r;
 }
 
 __device__ __forceinline__ void red_add_shared(uint32_t saddr, uint32_t v) {
@@ -350,10 +481,10 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                      const float4* __restrict__ qstat, const KnnStats* __restrict__ st,
                      unsigned long long* __restrict__ pool64, int32_t* __restrict__ cnt_out,
                      unsigned long long* __restrict__ qthr, int32_t* __restrict__ qfail, float* __restrict__ dump,
-                     const unsigned long long* __restrict__ qspec) {
+                     const unsigned long long* __restrict__ qspec, const float* __restrict__ tscale) {
     constexpr int HALVES = (QPC == 1) ? EW / 4 : 1;
     constexpr int WCOLS = BN / HALVES;  // columns of each tile this epilogue warp scans
-    constexpr int SB = 2 * KNN_KS * BN * 2;   // bytes of one reference stage
+    constexpr int SB = KNN_KS * BN * 2;       // bytes of one reference stage (fp16)
     constexpr int NBB = 16 * BN * 2;          // bytes of a reference tile's norm block
     constexpr bool DUMP = (MODE == 1);
     constexpr bool PIPE_ONLY = (MODE == 2 || MODE == 4);
@@ -453,7 +584,8 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
     } else if (warp == 1) {
         // ===== MMA issuer (one thread) =====
         if (lane == 0) {
-            constexpr uint32_t idesc = umma_idesc_bf16(KNN_BM, BN);
+            constexpr uint32_t idesc = umma_idesc_f16(KNN_BM, BN);      // fp16 x fp16 -> fp32
+            constexpr uint32_t idesc_n = umma_idesc_bf16(KNN_BM, BN);   // the bf16 norm block
             const uint32_t abytes = (uint32_t)g.a_bytes();
             mbar_wait(afull, 0);
             tc_fence_after();
@@ -471,25 +603,18 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                     for (int h = 0; h < QPC; ++h) {  // every query tile of the CTA on this stage
                         const uint32_t d_tmem = tmem_base + (uint32_t)((b * QPC + h) * BN);
                         const uint32_t a0 = smem_u32(sA) + (uint32_t)h * abytes;
-                        if (ks == g.KS) {  // norm block: |q|^2 + |r|^2 into the same accumulator
-                            const uint64_t an = umma_desc(a0 + (uint32_t)(g.Dp * 512), KNN_BM * 16, 128);
+                        if (ks == g.KS) {  // norm block: |q'|^2 + |r'|^2 into the same accumulator
+                            const uint64_t an = umma_desc(a0 + (uint32_t)(g.Dp * 256), KNN_BM * 16, 128);
                             const uint64_t bn = umma_desc(bs, BN * 16, 128);
-                            umma_bf16(d_tmem, an, bn, idesc, 1u);
+                            umma_bf16(d_tmem, an, bn, idesc_n, 1u);
                             continue;
                         }
-                        const uint32_t alo = a0 + (uint32_t)(g.Dp / 8) * (KNN_BM * 16);
 #pragma unroll
                         for (int j = 0; j < 2; ++j) {
                             const int kk = ks * 2 + j;
-                            const uint64_t ah = umma_desc(a0 + (uint32_t)(2 * kk) * (KNN_BM * 16), KNN_BM * 16, 128);
-                            const uint64_t al = umma_desc(alo + (uint32_t)(2 * kk) * (KNN_BM * 16), KNN_BM * 16, 128);
-                            const uint64_t bh = umma_desc(bs + (uint32_t)(2 * j) * (BN * 16), BN * 16, 128);
-                            const uint64_t bl = umma_desc(bs + SB / 2 + (uint32_t)(2 * j) * (BN * 16), BN * 16, 128);
-                            umma_bf16(d_tmem, ah, bh, idesc, (ks | j) ? 1u : 0u);
-                            if (g.passes == 3) {
-                                umma_bf16(d_tmem, ah, bl, idesc, 1u);
-                                umma_bf16(d_tmem, al, bh, idesc, 1u);
-                            }
+                            const uint64_t ad = umma_desc(a0 + (uint32_t)(2 * kk) * (KNN_BM * 16), KNN_BM * 16, 128);
+                            const uint64_t bd = umma_desc(bs + (uint32_t)(2 * j) * (BN * 16), BN * 16, 128);
+                            umma_bf16(d_tmem, ad, bd, idesc, (ks | j) ? 1u : 0u);
                         }
                     }
                     // frees the stage (in every CTA of the cluster) when these MMAs complete
@@ -530,6 +655,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
         unsigned long long T = kSentPair;  // running bound on the k-th (d~, index) pair
         // the band: 2 eps_q above the k-th d~ (every reference that can be in the exact top-k)
         const float band = (qvalid && !DUMP) ? __fmul_ru(2.f, knn_eps(qstat[q], *st, g.D)) : 0.f;
+        const float sq = qvalid ? qstat[q].x : 1.f;  // sigma of this query tile
         float tv = 0.f;                    // filter value: value(T) + band, rounded up
         bool fast = false;                 // finite filter value: the fp32 compare d~ <= tv pre-filters
         bool failed = !(band < __int_as_float(0x7f800000));  // no finite band: exact fallback
@@ -598,7 +724,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                 const unsigned long long t =
                     (jn <= 256)   ? pool_narrow64<8>(jp, jn, (uint32_t)target, &nn, jb, slk)
                     : (jn <= 512) ? pool_narrow64<16>(jp, jn, (uint32_t)target, &nn, jb, slk)
-                    : (jn <= 32 * kNarrowRegs) ? pool_narrow64<kNarrowRegs>(jp, jn, (uint32_t)target, &nn, jb, slk)
+                    : (EW <= 8 && jn <= 32 * kNarrowRegs) ? pool_narrow64<(EW <= 8 ? kNarrowRegs : 16)>(jp, jn, (uint32_t)target, &nn, jb, slk)
                                                : pool_select64(jp, jn, (uint32_t)target, hist, &nn, jb, slk);
                 if ((int)lane == j) {
                     *np = nn;
@@ -642,6 +768,11 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
             const unsigned long long cc0 = PROF ? clock64() : 0;
             tc_fence_after();
             const uint32_t taddr = tmem_base + ((uint32_t)(quad * 32) << 16) + (uint32_t)((b * QPC + hq) * BN);
+            // the accumulator is sigma_q sigma_t d~: compare it with the bound scaled the same
+            // way (rounded up: never rejects a candidate) and unscale what is kept (powers of
+            // two: exact unless subnormal, covered by knn_eps)
+            const float stl = sq * __ldg(tscale + t);
+            const float inv = __frcp_rn(stl);
             if (!DUMP && !PIPE_ONLY && lt == 0 && g.k <= BN && (int64_t)t * BN + BN <= g.N &&
                 (Fs > 0 || __any_sync(kFull, qvalid && (uint32_t)(T >> 32) == kSentKey))) {
                 // Starting bound without a fill phase: the exact k-th smallest distance of
@@ -660,7 +791,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                         tmem_ld32(taddr + (uint32_t)(c * 32), v);
 #pragma unroll
                         for (int j = 0; j < 32; ++j) {
-                            const float x = __uint_as_float(v[j]);
+                            const float x = __uint_as_float(v[j]) * inv;
                             cnt += (__float_as_uint(x < 0.f ? 0.f : x) < cand) ? 1u : 0u;
                         }
                     }
@@ -675,7 +806,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                         uint32_t v[KNN_CW];
                         tmem_ld64(taddr + (uint32_t)(c * KNN_CW), v);
 #pragma unroll
-                        for (int j = 0; j < KNN_CW; ++j) mn = fminf(mn, __uint_as_float(v[j]));
+                        for (int j = 0; j < KNN_CW; ++j) mn = fminf(mn, __uint_as_float(v[j]) * inv);
                     }
                     s_lo = fmaxf(mn, 0.f);
                     s_hi = __uint_as_float(vb);
@@ -698,7 +829,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                     tmem_ld64(taddr + (uint32_t)(c * KNN_CW), v);
 #pragma unroll
                     for (int j = 0; j < KNN_CW; ++j) {
-                        const float d = __uint_as_float(v[j]);
+                        const float d = __uint_as_float(v[j]) * inv;
                         if (d <= s_hi) {
                             const int bk = min(max((int)((d - s_lo) * s_inv), 0), KNN_SB - 1);
                             red_add_shared(shist_s + (uint32_t)(bk * 128), 1u);
@@ -736,15 +867,17 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                 const uint32_t colt = (uint32_t)t * BN;  // N < 2^31
                 const int nlim = (int)min((int64_t)BN, g.N - (int64_t)colt);  // valid columns of the tile
                 const bool live = qvalid && !failed;
+                const float tvs = __fmul_ru(tv, stl);  // (after this tile's starting-bound updates)
                 auto scan32 = [&](const uint32_t(&v)[32], int c0) {
-                    float gmn[8];
+                    float gmn[8];  // 3-input minima (FMNMX3): 20 instructions per 32 values
 #pragma unroll
                     for (int j = 0; j < 8; ++j)
-                        gmn[j] = fminf(fminf(__uint_as_float(v[4 * j]), __uint_as_float(v[4 * j + 1])),
-                                       fminf(__uint_as_float(v[4 * j + 2]), __uint_as_float(v[4 * j + 3])));
-                    const float mn = fminf(fminf(fminf(gmn[0], gmn[1]), fminf(gmn[2], gmn[3])),
-                                           fminf(fminf(gmn[4], gmn[5]), fminf(gmn[6], gmn[7])));
-                    if (!__any_sync(kFull, live && (!fast || mn <= tv))) return;
+                        gmn[j] = fminf(fmin3(__uint_as_float(v[4 * j]), __uint_as_float(v[4 * j + 1]),
+                                             __uint_as_float(v[4 * j + 2])),
+                                       __uint_as_float(v[4 * j + 3]));
+                    const float mn = fmin3(fmin3(gmn[0], gmn[1], gmn[2]), fmin3(gmn[3], gmn[4], gmn[5]),
+                                           fminf(gmn[6], gmn[7]));
+                    if (!__any_sync(kFull, live && (!fast || mn <= tvs))) return;
                     const unsigned long long cr0 = PROF ? clock64() : 0;
                     // rare path: each lane visits only its own candidate groups (a divergent
                     // loop of max-over-lanes length); the group's 4 values are picked from the
@@ -753,7 +886,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                     // harmless extra pool entry (narrowing applies the exact pair order).
                     uint32_t gm = 0;
 #pragma unroll
-                    for (int u = 0; u < 8; ++u) gm |= (uint32_t)(!fast || gmn[u] <= tv) << u;
+                    for (int u = 0; u < 8; ++u) gm |= (uint32_t)(!fast || gmn[u] <= tvs) << u;
                     if (!live) gm = 0;
                     while (gm) {
                         const int u = __ffs(gm) - 1;
@@ -766,8 +899,9 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                             const uint32_t a2 = b0 ? v[20 + i] : v[16 + i], a3 = b0 ? v[28 + i] : v[24 + i];
                             const uint32_t c01 = b1 ? a1 : a0, c23 = b1 ? a3 : a2;
                             const float x = __uint_as_float(b2 ? c23 : c01);
-                            if (cu + i < nlim && (!fast || x <= tv)) {
-                                const float dc = (x < 0.f) ? 0.f : x;  // clamp, NaN propagates
+                            if (cu + i < nlim && (!fast || x <= tvs)) {
+                                const float xu = x * inv;
+                                const float dc = (xu < 0.f) ? 0.f : xu;  // clamp, NaN propagates
                                 const int slot = (PAIR > 1) ? atomicAdd(np, 1) : (*np)++;
                                 pool[slot] = ((unsigned long long)key_of(dc) << 32) | (colt + (uint32_t)(cu + i));
                                 if (PROF) prof_app++;
@@ -802,7 +936,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                 // (knn_distances) the accumulator is d = |q|^2 + |r|^2 - 2 q.r; clamped at 0
                 float d[KNN_CW];
 #pragma unroll
-                for (int j = 0; j < KNN_CW; ++j) d[j] = __uint_as_float(v[j]);
+                for (int j = 0; j < KNN_CW; ++j) d[j] = __uint_as_float(v[j]) * inv;
                 if (qvalid)
                     for (int j = 0; j < KNN_CW; ++j)
                         if (col0 + j < g.N) dump[q * g.N + col0 + j] = (d[j] < 0.f) ? 0.f : d[j];
@@ -846,7 +980,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
 static size_t al256(size_t x) { return (x + 255u) & ~(size_t)255u; }
 
 struct KnnWork {
-    size_t ref_img, stats, q_img, qstat, pool, cnt, qthr, qspec, qfail, fb, prof, total;
+    size_t ref_img, tscale, csum, rownorm, stats, q_img, qstat, pool, cnt, qthr, qspec, qfail, fb, prof, total;
 };
 
 // Queries are processed in chunks (multiples of 128 queries) so that the pools,
@@ -893,12 +1027,6 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     // 5.14 ms), so L2 is not the floor and the default is cs = 1.
     g.cs = (g.QPC == 1 && g.QT >= cs_env) ? cs_env : 1;
     g.QTp = (g.QPC == 2) ? (g.QT + 1) / 2 : (g.QT + g.cs - 1) / g.cs * g.cs;  // CTA rows of the grid
-#ifdef KSEL_EXPERIMENTS
-    static const int passes_env = env_int("KSEL_KNN_PASSES", 3) == 1 ? 1 : 3;  // experiments only: 1 breaks the accuracy bound
-#else
-    constexpr int passes_env = 3;
-#endif
-    g.passes = passes_env;
     g.k = k;
     const int kk = k < 32 ? 32 : k;
     // room for >= 1 tile of candidates after narrowing to k; register narrowing holds 1152
@@ -906,18 +1034,22 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     // room for 8 tiles of candidates between narrowings (radix select, pool_select64)
     int P = (kk <= 128) ? 1152 : kk + 8 * 256;
     g.P = (P + 31) / 32 * 32;
+    // epilogue warps: 16 (four per TMEM lane quadrant, 64 columns of every tile each) or 8;
+    // result-preserving (the warps of a quadrant share each query's pool and bound)
+    static const int ew_env = [] {
+        const int v = env_int("KSEL_KNN_EW", 16);
 #ifdef KSEL_EXPERIMENTS
-    static const int ew_env = env_int("KSEL_KNN_EW", 4) == 8 ? 8 : 4;  // experiments: 4 or 8 epilogue warps
-#else
-    constexpr int ew_env = 8;
+        if (v == 4) return 4;
 #endif
+        return v == 8 ? 8 : 16;
+    }();
     g.halves = (g.QPC == 2) ? 1 : ew_env / 4;
     g.EW = (g.QPC == 2) ? 8 : 4 * g.halves;
     // ring depth: as many stages as fit next to the resident query tile(s)
     const int fixed =
         1024 + g.QPC * (g.Dp * 512 + KNN_NORM_A_BYTES) + KnnSmem::scratch(g.EW, g.QPC) + 512;
     g.NS = (kMaxSmemPerBlock - fixed) / g.stage_bytes();
-    if (g.NS > 6) g.NS = 6;
+    if (g.NS > 12) g.NS = 12;
     g.idx_offset = idx_offset;
     static const int cap_env = env_int("KSEL_KNN_SOFTCAP", 0);  // experiments: narrow early (pool fill cap)
     // narrow before a pool reaches P when queues are small: the bound then tracks the
@@ -996,6 +1128,9 @@ static KnnWork knn_work_layout(const KnnGeom& g) {
     KnnWork w{};
     size_t off = 0;
     w.ref_img = off; off += al256((size_t)g.NT * g.tile_bytes());
+    w.tscale = off;  off += al256((size_t)g.NT * 4);
+    w.csum = off;    off += al256((size_t)g.Dp * 16);
+    w.rownorm = off; off += al256((size_t)(g.NT + g.QTp * g.QPC) * KNN_BN * 8);
     w.stats = off;   off += al256(sizeof(KnnStats));
     w.q_img = off;   off += al256((size_t)g.QTp * g.QPC * g.a_bytes());
     w.qstat = off;   off += al256((size_t)g.Q * 16);
@@ -1048,14 +1183,26 @@ static cudaError_t knn_run(const float* ref, const float* query, int64_t N, int6
     uint4* q_img = reinterpret_cast<uint4*>(work + w.q_img);
     float4* qstat = reinterpret_cast<float4*>(work + w.qstat);
     KnnStats* stats = reinterpret_cast<KnnStats*>(work + w.stats);
+    float* tscale = reinterpret_cast<float*>(work + w.tscale);
+    double* csum = reinterpret_cast<double*>(work + w.csum);
+    double* rownorm = reinterpret_cast<double*>(work + w.rownorm);
     cudaError_t e = cudaMemsetAsync(stats, 0, sizeof(KnnStats), stream);
     if (e != cudaSuccess) return e;
     for (int64_t q0 = 0; q0 < Q; q0 += Qc) {
         const int64_t nq = std::min(Qc, Q - q0);
         const KnnGeom g = knn_geometry(N, nq, D, k, sms, idx_offset, (int64_t)gq.S * Qc);
         const int nt = (q0 == 0) ? g.NT : 0;  // reference tiles: first chunk only
+        if (nt > 0) {
+            e = cudaMemsetAsync(csum, 0, (size_t)g.Dp * 16, stream);
+            if (e != cudaSuccess) return e;
+            knn_sum_kernel<<<dim3((unsigned)(g.Dp / 32), 32), 256, 0, stream>>>(ref, N, D, g.Dp, csum);
+            note_launch();
+        }
+        knn_stats_kernel<<<(unsigned)(nt + g.QT), KNN_PREP_THREADS, 0, stream>>>(
+            ref, query + q0 * (int64_t)D, g, nt, csum, rownorm, qstat, tscale, stats);
+        note_launch();
         knn_prep_kernel<<<(unsigned)(nt + g.QT), KNN_PREP_THREADS, 0, stream>>>(
-            ref, query + q0 * (int64_t)D, g, nt, ref_img, q_img, qstat, stats);
+            ref, query + q0 * (int64_t)D, g, nt, csum, rownorm, qstat, tscale, ref_img, q_img);
         note_launch();
         e = cudaGetLastError();
 #ifdef KSEL_EXPERIMENTS
@@ -1076,25 +1223,27 @@ static cudaError_t knn_run(const float* ref, const float* query, int64_t N, int6
             const int m = env_int("KSEL_KNN_MODE", 0);
             return (m >= 2 && m <= 4) ? m : 0;
         }();
-        const bool ew8 = g.halves == 2;
+        const int ewh = g.halves;
         auto kern = (g.QPC == 2)
                         ? (dump ? knn_fused_kernel<1, 8, 128, 2>
                            : mode_env == 2 ? knn_fused_kernel<2, 8, 128, 2>
                            : mode_env == 3 ? knn_fused_kernel<3, 8, 128, 2>
                            : mode_env == 4 ? knn_fused_kernel<4, 8, 128, 2>
                                            : knn_fused_kernel<0, 8, 128, 2>)
-                    : dump ? (ew8 ? knn_fused_kernel<1, 8, 256, 1> : knn_fused_kernel<1, 4, 256, 1>)
-                    : mode_env == 2 ? (ew8 ? knn_fused_kernel<2, 8, 256, 1> : knn_fused_kernel<2, 4, 256, 1>)
-                    : mode_env == 3 ? (ew8 ? knn_fused_kernel<3, 8, 256, 1> : knn_fused_kernel<3, 4, 256, 1>)
+                    : dump ? (ewh == 4 ? knn_fused_kernel<1, 16, 256, 1> : ewh == 2 ? knn_fused_kernel<1, 8, 256, 1> : knn_fused_kernel<1, 4, 256, 1>)
+                    : mode_env == 2 ? (ewh == 2 ? knn_fused_kernel<2, 8, 256, 1> : knn_fused_kernel<2, 4, 256, 1>)
+                    : mode_env == 3 ? (ewh == 4 ? knn_fused_kernel<3, 16, 256, 1> : ewh == 2 ? knn_fused_kernel<3, 8, 256, 1> : knn_fused_kernel<3, 4, 256, 1>)
                     : mode_env == 4 ? knn_fused_kernel<4, 4, 256, 1>
-                                    : (ew8 ? knn_fused_kernel<0, 8, 256, 1> : knn_fused_kernel<0, 4, 256, 1>);
+                                    : (ewh == 4 ? knn_fused_kernel<0, 16, 256, 1> : ewh == 2 ? knn_fused_kernel<0, 8, 256, 1> : knn_fused_kernel<0, 4, 256, 1>);
         auto sel_kern = (g.QPC == 2) ? knn_fused_kernel<0, 8, 128, 2>
-                                     : (ew8 ? knn_fused_kernel<0, 8, 256, 1> : knn_fused_kernel<0, 4, 256, 1>);
+                                     : (ewh == 4 ? knn_fused_kernel<0, 16, 256, 1> : ewh == 2 ? knn_fused_kernel<0, 8, 256, 1> : knn_fused_kernel<0, 4, 256, 1>);
         if (!dump && mode_env == 3) kdump = reinterpret_cast<float*>(work + w.prof);
 #else
         constexpr int mode_env = 0;
-        auto kern = dump ? knn_fused_kernel<1, 8, 256, 1> : knn_fused_kernel<0, 8, 256, 1>;
-        auto sel_kern = knn_fused_kernel<0, 8, 256, 1>;
+        const bool ew16 = g.halves == 4;
+        auto kern = dump ? (ew16 ? knn_fused_kernel<1, 16, 256, 1> : knn_fused_kernel<1, 8, 256, 1>)
+                         : (ew16 ? knn_fused_kernel<0, 16, 256, 1> : knn_fused_kernel<0, 8, 256, 1>);
+        auto sel_kern = ew16 ? knn_fused_kernel<0, 16, 256, 1> : knn_fused_kernel<0, 8, 256, 1>;
 #endif
         auto launch = [&](decltype(kern) kf, const KnnGeom& gg, unsigned long long* thr,
                           const unsigned long long* spec, float* kd, bool timed) -> cudaError_t {
@@ -1119,7 +1268,7 @@ static cudaError_t knn_run(const float* ref, const float* query, int64_t N, int6
                                     static_cast<const KnnStats*>(stats),
                                     reinterpret_cast<unsigned long long*>(work + w.pool),
                                     reinterpret_cast<int32_t*>(work + w.cnt), thr,
-                                    reinterpret_cast<int32_t*>(work + w.qfail), kd, spec);
+                                    reinterpret_cast<int32_t*>(work + w.qfail), kd, spec, tscale);
             note_launch();
             if (timed) timing_end(slot, stream);
             return le == cudaSuccess ? cudaGetLastError() : le;
