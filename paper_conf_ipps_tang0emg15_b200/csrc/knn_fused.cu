@@ -80,6 +80,8 @@ struct KnnGeom {
     int sample_ctas;
     int halves;          // column halves per tile (EW / 4): pools per split
     int pcap;            // pool fill that triggers a narrowing before a tile (<= P)
+    int nstride;         // tiles between two bound refreshes / narrowing checks (room: nstride x BN)
+    int spec_ms;         // speculative pre-pass: sampled tiles (0: none)
     int cs;              // cluster size: CTAs (consecutive query tiles, same reference range) that
                          // share every reference stage through one multicast load
     int QTp;             // query tiles padded to a multiple of cs (padding tiles select nothing)
@@ -180,7 +182,7 @@ constexpr int KNN_PREP_THREADS = 256;
 __global__ void __launch_bounds__(KNN_PREP_THREADS)
     knn_stats_kernel(const float* __restrict__ ref, const float* __restrict__ qry, KnnGeom g, int nt,
                      const double* __restrict__ csum, double* __restrict__ rownorm, float4* __restrict__ qstat,
-                     float* __restrict__ tscale, KnnStats* __restrict__ st) {
+                     float2* __restrict__ tscale, KnnStats* __restrict__ st) {
     __shared__ float cs[KNN_MAX_D];
     __shared__ uint32_t samx, smax;
     __shared__ int sbad;
@@ -251,7 +253,7 @@ __global__ void __launch_bounds__(KNN_PREP_THREADS)
             }
         }
     } else if (tid == 0) {
-        tscale[t] = sig;
+        tscale[t] = make_float2(sig, 1.f / sig);  // (exact: a power of two)
         atomicMax(&st->R2, sbad ? 0x7f800000u : smax);
         atomicMax(&st->isig, __float_as_uint(1.f / sig));
     }
@@ -268,7 +270,7 @@ __global__ void __launch_bounds__(KNN_PREP_THREADS)
 __global__ void __launch_bounds__(KNN_PREP_THREADS)
     knn_prep_kernel(const float* __restrict__ ref, const float* __restrict__ qry, KnnGeom g, int nt,
                     const double* __restrict__ csum, const double* __restrict__ rownorm,
-                    const float4* __restrict__ qstat, const float* __restrict__ tscale,
+                    const float4* __restrict__ qstat, const float2* __restrict__ tscale,
                     uint4* __restrict__ ref_img, uint4* __restrict__ q_img) {
     __shared__ float tile[KNN_BN][KNN_KS + 1];
     __shared__ float cs[KNN_MAX_D];
@@ -280,7 +282,7 @@ __global__ void __launch_bounds__(KNN_PREP_THREADS)
     const int64_t n = is_q ? g.Q : g.N;
     const float* x = is_q ? qry : ref;
     const int64_t row = t * rows + tid;
-    const float sig = is_q ? (t * rows < n ? qstat[t * rows].x : 1.f) : tscale[t];
+    const float sig = is_q ? (t * rows < n ? qstat[t * rows].x : 1.f) : tscale[t].x;
     const float mul = is_q ? -2.f * sig : sig;  // exact
     for (int ks = 0; ks < g.KS; ++ks) {
         __syncthreads();
@@ -460,7 +462,7 @@ struct KnnSmem {
     // quadrant of a query tile: the EW / 4 warps scanning its column parts share it), and
     // the per-query state those warps share: pool fill, failure flag, bound pair
     __host__ __device__ static int scratch(int ew, int qpc) {
-        return ew * kHistWarp + 4 * qpc * kWarpScratch + qpc * 128 * 16;
+        return ew * kHistWarp + 4 * qpc * kWarpScratch + qpc * 128 * 24;
     }
     __host__ __device__ static int total(const KnnGeom& g) {
         return 1024 /*align slack*/ + g.QPC * g.a_bytes() + g.NS * g.stage_bytes() + scratch(g.EW, g.QPC) +
@@ -481,7 +483,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                      const float4* __restrict__ qstat, const KnnStats* __restrict__ st,
                      unsigned long long* __restrict__ pool64, int32_t* __restrict__ cnt_out,
                      unsigned long long* __restrict__ qthr, int32_t* __restrict__ qfail, float* __restrict__ dump,
-                     const unsigned long long* __restrict__ qspec, const float* __restrict__ tscale) {
+                     const unsigned long long* __restrict__ qspec, const float2* __restrict__ tscale) {
     constexpr int HALVES = (QPC == 1) ? EW / 4 : 1;
     constexpr int WCOLS = BN / HALVES;  // columns of each tile this epilogue warp scans
     constexpr int SB = KNN_KS * BN * 2;       // bytes of one reference stage (fp16)
@@ -503,7 +505,8 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                                                                      4 * QPC * KnnSmem::kWarpScratch);  // [QPC*128]
     int* qs_n = reinterpret_cast<int*>(qs_T + QPC * 128);                                              // [QPC*128]
     int* qs_f = qs_n + QPC * 128;                                                                      // [QPC*128]
-    uint64_t* bars = reinterpret_cast<uint64_t*>(qs_f + QPC * 128);
+    uint32_t* qs_v = reinterpret_cast<uint32_t*>(qs_f + QPC * 128);                                   // [QPC*128]
+    uint64_t* bars = reinterpret_cast<uint64_t*>(qs_v + QPC * 256);
     uint64_t* full = bars;
     uint64_t* empty = bars + NS;
     uint64_t* accf = bars + 2 * NS;
@@ -656,6 +659,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
         // the band: 2 eps_q above the k-th d~ (every reference that can be in the exact top-k)
         const float band = (qvalid && !DUMP) ? __fmul_ru(2.f, knn_eps(qstat[q], *st, g.D)) : 0.f;
         const float sq = qvalid ? qstat[q].x : 1.f;  // sigma of this query tile
+        const float sqi = __frcp_rn(sq);               // (exact: a power of two)
         float tv = 0.f;                    // filter value: value(T) + band, rounded up
         bool fast = false;                 // finite filter value: the fp32 compare d~ <= tv pre-filters
         bool failed = !(band < __int_as_float(0x7f800000));  // no finite band: exact fallback
@@ -753,13 +757,13 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
             const bool sampling = lt < Fs;
             const int t = (sampling ? t0 + lt : t0 + lt - Fs) * g.tstride;
             const int b = lt & 1;
-            if (!DUMP && !PIPE_ONLY) {
+            if (!DUMP && !PIPE_ONLY && lt % g.nstride == 0) {
                 // adopt the tightest bound any split of this query had published when the
-                // previous tile started (the load's latency hides behind that tile)
+                // previous check started (the load's latency hides behind those tiles)
                 adopt(thr_next);
                 if (qvalid) thr_next = __ldcg(&qthr[q]);
                 const unsigned long long c0 = PROF ? clock64() : 0;
-                narrow_lanes(BN, g.k, g.pcap, false);  // room: both column parts of a tile
+                narrow_lanes(g.nstride * BN, g.k, g.pcap, false);  // room: every column of nstride tiles
                 if (PROF) prof_narrow += clock64() - c0;
             }
             const unsigned long long cw0 = PROF ? clock64() : 0;
@@ -771,18 +775,19 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
             // the accumulator is sigma_q sigma_t d~: compare it with the bound scaled the same
             // way (rounded up: never rejects a candidate) and unscale what is kept (powers of
             // two: exact unless subnormal, covered by knn_eps)
-            const float stl = sq * __ldg(tscale + t);
-            const float inv = __frcp_rn(stl);
-            if (!DUMP && !PIPE_ONLY && lt == 0 && g.k <= BN && (int64_t)t * BN + BN <= g.N &&
-                (Fs > 0 || __any_sync(kFull, qvalid && (uint32_t)(T >> 32) == kSentKey))) {
+            const float2 tsc = __ldg(tscale + t);  // (sigma_t, 1 / sigma_t)
+            const float stl = sq * tsc.x;
+            const float inv = sqi * tsc.y;
+            if (!DUMP && !PIPE_ONLY && lt == 0 && g.k <= BN && (int64_t)t * BN + BN <= g.N && qspec == nullptr) {
                 // Starting bound without a fill phase: the exact k-th smallest distance of
                 // this first (full) tile, by bisection on the bits of the clamped value
                 // (non-negative floats order like their bit patterns), re-reading the
                 // accumulator from TMEM each step.  At least k pairs of the row are <= it,
                 // so (that key, any index) is a valid bound.
+                // (one warp of the query group bisects; the others read its result)
                 uint32_t vb = 0;
 #pragma unroll 1
-                for (int bit = 30; bit >= 0; --bit) {
+                for (int bit = 30; bit >= 0 && half == 0; --bit) {
                     const uint32_t cand = vb | (1u << bit);
                     uint32_t cnt = 0;
 #pragma unroll 1
@@ -797,7 +802,13 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                     }
                     if (cnt < (uint32_t)g.k) vb = cand;
                 }
-                if (qvalid) adopt(((unsigned long long)key_of(__uint_as_float(vb)) << 32) | 0x7ffffffeu);
+                if (half == 0) {
+                    qs_v[qidx] = vb;
+                    if (qvalid) adopt(((unsigned long long)key_of(__uint_as_float(vb)) << 32) | 0x7ffffffeu);
+                }
+                pair_bar();
+                vb = qs_v[qidx];
+                refresh();
                 if (Fs > 0) {
                     // histogram range: [max(0, tile minimum), k-th of the tile]
                     float mn = __int_as_float(0x7f800000);
@@ -988,6 +999,12 @@ struct KnnWork {
 // points would otherwise need tens of GB of workspace).
 constexpr size_t kPoolBudget = 2ull << 30;
 
+static int knn_spec_tiles(const KnnGeom& g) {
+    static const int env = env_int("KSEL_KNN_SPEC", 64);  // sampled tiles (0: off)
+    if (env <= 0 || g.NT < 16 * env || g.tstride != 1) return 0;
+    return env;
+}
+
 // max_lists > 0: cap the split count so that S * halves * Q <= max_lists (a later query
 // chunk must fit the workspace laid out for the first)
 static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int64_t idx_offset,
@@ -1088,6 +1105,17 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
         if (max_lists > 0) g.S = (int)std::max<int64_t>(1, std::min<int64_t>(g.S, max_lists / Q));
     }
     g.cold_splits = std::min(g.S, (num_sms + g.QTp - 1) / g.QTp);
+    g.nstride = 1;
+    g.spec_ms = knn_spec_tiles(g);
+    if (g.spec_ms > 0) {
+        // a speculative start: no split is cold (equal splits); bounds are refreshed and
+        // pools checked every 4 tiles, so pools get room for 4 tiles of candidates beyond
+        // k + a band's worth, and narrow only when that room runs out
+        g.cold_splits = 0;
+        g.nstride = 4;
+        g.P = std::max(g.P, (kk + 4 * g.BN + 256 + 31) / 32 * 32);
+        g.pcap = g.P;
+    }
     return g;
 }
 
@@ -1101,11 +1129,6 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
 // P(count < k) < 1e-10 on i.i.d. rows.  The main pass admits against T_spec from its first
 // tile; knn_rescore_kernel verifies it (>= k pooled pairs <= T_spec, or a published
 // bound <= T_spec), else the query takes the exact fallback -- exact either way.
-static int knn_spec_tiles(const KnnGeom& g) {
-    static const int env = env_int("KSEL_KNN_SPEC", 64);  // sampled tiles (0: off)
-    if (env <= 0 || g.NT < 16 * env || g.tstride != 1) return 0;
-    return env;
-}
 static KnnGeom knn_spec_geometry(const KnnGeom& g, int ms) {
     KnnGeom p = g;
     const double lam = (double)g.k * (double)ms * g.BN / (double)g.N;
@@ -1121,6 +1144,8 @@ static KnnGeom knn_spec_geometry(const KnnGeom& g, int ms) {
     p.sample_tiles = 0;
     p.sample_ctas = 0;
     p.cold_splits = 0;
+    p.nstride = 1;
+    p.spec_ms = 0;
     return p;
 }
 
@@ -1128,7 +1153,7 @@ static KnnWork knn_work_layout(const KnnGeom& g) {
     KnnWork w{};
     size_t off = 0;
     w.ref_img = off; off += al256((size_t)g.NT * g.tile_bytes());
-    w.tscale = off;  off += al256((size_t)g.NT * 4);
+    w.tscale = off;  off += al256((size_t)g.NT * 8);
     w.csum = off;    off += al256((size_t)g.Dp * 16);
     w.rownorm = off; off += al256((size_t)(g.NT + g.QTp * g.QPC) * KNN_BN * 8);
     w.stats = off;   off += al256(sizeof(KnnStats));
@@ -1183,7 +1208,7 @@ static cudaError_t knn_run(const float* ref, const float* query, int64_t N, int6
     uint4* q_img = reinterpret_cast<uint4*>(work + w.q_img);
     float4* qstat = reinterpret_cast<float4*>(work + w.qstat);
     KnnStats* stats = reinterpret_cast<KnnStats*>(work + w.stats);
-    float* tscale = reinterpret_cast<float*>(work + w.tscale);
+    float2* tscale = reinterpret_cast<float2*>(work + w.tscale);
     double* csum = reinterpret_cast<double*>(work + w.csum);
     double* rownorm = reinterpret_cast<double*>(work + w.rownorm);
     cudaError_t e = cudaMemsetAsync(stats, 0, sizeof(KnnStats), stream);
@@ -1274,16 +1299,18 @@ static cudaError_t knn_run(const float* ref, const float* query, int64_t N, int6
             return le == cudaSuccess ? cudaGetLastError() : le;
         };
         // speculative pre-pass (selection only): T_spec per query into qspec
-        const int ms = (dump || mode_env != 0) ? 0 : knn_spec_tiles(g);
+        const int ms = (dump || mode_env != 0) ? 0 : g.spec_ms;
         unsigned long long* qspec = ms > 0 ? reinterpret_cast<unsigned long long*>(work + w.qspec) : nullptr;
         if (ms > 0) {
             e = cudaMemsetAsync(qspec, 0xff, (size_t)nq * 8, stream);
             if (e == cudaSuccess) e = launch(sel_kern, knn_spec_geometry(g, ms), qspec, nullptr, nullptr, false);
             if (e != cudaSuccess) return e;
         }
-        // with a speculative start no split is cold: equal splits
         KnnGeom gm = g;
-        if (ms > 0) gm.cold_splits = 0;
+        if (ms == 0) {  // (knn_distances / experiment modes: no speculative start)
+            gm.nstride = 1;
+            gm.pcap = std::min(gm.pcap, gm.P);
+        }
         e = launch(kern, gm, reinterpret_cast<unsigned long long*>(work + w.qthr), qspec, kdump, !dump);
         if (e != cudaSuccess) return e;
         if (dump) {
