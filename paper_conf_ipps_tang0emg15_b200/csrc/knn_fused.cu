@@ -82,6 +82,8 @@ struct KnnGeom {
     int pcap;            // pool fill that triggers a narrowing before a tile (<= P)
     int nstride;         // tiles between two bound refreshes / narrowing checks (room: nstride x BN)
     int spec_ms;         // speculative pre-pass: sampled tiles (0: none)
+    int prepass;         // this launch IS the pre-pass: a query whose band overflows is not
+                         // failed (it merely gets a looser T_spec); qthr = the T_spec output
     int cs;              // cluster size: CTAs (consecutive query tiles, same reference range) that
                          // share every reference stage through one multicast load
     int QTp;             // query tiles padded to a multiple of cs (padding tiles select nothing)
@@ -478,7 +480,7 @@ struct KnnSmem {
 // queries: with QPC = 2, BN = 128 and four 128-column accumulators, half the bytes
 // land in shared memory per output)
 template <int MODE, int EW, int BN, int QPC>
-__global__ void __launch_bounds__(knn_threads(EW), 1)
+__global__ void __launch_bounds__(knn_threads(EW), 1)  // (EW = 16: 18 warps, 5 on one SM sub-partition -> <= 96 registers)
     knn_fused_kernel(KnnGeom g, const uint8_t* __restrict__ ref_img, const uint8_t* __restrict__ q_img,
                      const float4* __restrict__ qstat, const KnnStats* __restrict__ st,
                      unsigned long long* __restrict__ pool64, int32_t* __restrict__ cnt_out,
@@ -663,7 +665,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
         float tv = 0.f;                    // filter value: value(T) + band, rounded up
         bool fast = false;                 // finite filter value: the fp32 compare d~ <= tv pre-filters
         bool failed = !(band < __int_as_float(0x7f800000));  // no finite band: exact fallback
-        if (qvalid && !DUMP && !PIPE_ONLY && failed && half == 0) qfail[q] = 1;
+        if (qvalid && !DUMP && !PIPE_ONLY && failed && half == 0 && !g.prepass) qfail[q] = 1;
         if (half == 0) {
             *np = 0;
             *fp = failed ? 1 : 0;
@@ -739,7 +741,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                         failed = true;
                         *np = 0;
                         *fp = 1;
-                        qfail[q] = 1;
+                        if (!g.prepass) qfail[q] = 1;  // (pre-pass: just no speculation)
                     }
                 }
             }
@@ -921,18 +923,29 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)
                     }
                     if (PROF) { prof_rare += clock64() - cr0; prof_nrare++; }
                 };
-                uint32_t va[32], vb[32];
-                tmem_ld32_issue(taddr + (uint32_t)(half * WCOLS), va);
-                tmem_wait32(va);
                 const int cb = half * (WCOLS / 32), ce = cb + WCOLS / 32;
+                if constexpr (EW >= 16) {
+                    // (16 warps: TMEM load latency is short next to the warp count; one
+                    // 32-register buffer keeps the epilogue within its register budget)
 #pragma unroll 1
-                for (int c = cb; c < ce; c += 2) {
-                    tmem_ld32_issue(taddr + (uint32_t)((c + 1) * 32), vb);
-                    scan32(va, c * 32);
-                    tmem_wait32(vb);
-                    if (c + 2 < ce) tmem_ld32_issue(taddr + (uint32_t)((c + 2) * 32), va);
-                    scan32(vb, (c + 1) * 32);
-                    if (c + 2 < ce) tmem_wait32(va);
+                    for (int c = cb; c < ce; ++c) {
+                        uint32_t va[32];
+                        tmem_ld32(taddr + (uint32_t)(c * 32), va);
+                        scan32(va, c * 32);
+                    }
+                } else {
+                    uint32_t va[32], vb[32];
+                    tmem_ld32_issue(taddr + (uint32_t)(half * WCOLS), va);
+                    tmem_wait32(va);
+#pragma unroll 1
+                    for (int c = cb; c < ce; c += 2) {
+                        tmem_ld32_issue(taddr + (uint32_t)((c + 1) * 32), vb);
+                        scan32(va, c * 32);
+                        tmem_wait32(vb);
+                        if (c + 2 < ce) tmem_ld32_issue(taddr + (uint32_t)((c + 2) * 32), va);
+                        scan32(vb, (c + 1) * 32);
+                        if (c + 2 < ce) tmem_wait32(va);
+                    }
                 }
             }
 #pragma unroll 1
@@ -1106,6 +1119,7 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
     }
     g.cold_splits = std::min(g.S, (num_sms + g.QTp - 1) / g.QTp);
     g.nstride = 1;
+    g.prepass = 0;
     g.spec_ms = knn_spec_tiles(g);
     if (g.spec_ms > 0) {
         // a speculative start: no split is cold (equal splits); bounds are refreshed and
@@ -1137,7 +1151,9 @@ static KnnGeom knn_spec_geometry(const KnnGeom& g, int ms) {
     const int kk = p.k < 32 ? 32 : p.k;
     const int P = (kk <= 128) ? 1152 : kk + 8 * 256;
     p.P = (P + 31) / 32 * 32;
-    p.pcap = std::max(kk + 32 + g.BN, std::min(p.P, kk <= 128 ? 512 : p.P));
+    // narrow as soon as a tile's room is left: the running bound (cold: the first tile's
+    // j-th) then tightens every few tiles instead of after ~30 (j << the sample)
+    p.pcap = kk + g.BN + 128;
     p.ntiles = ms;
     p.tstride = g.NT / ms;
     p.S = 1;
@@ -1146,6 +1162,7 @@ static KnnGeom knn_spec_geometry(const KnnGeom& g, int ms) {
     p.cold_splits = 0;
     p.nstride = 1;
     p.spec_ms = 0;
+    p.prepass = 1;
     return p;
 }
 

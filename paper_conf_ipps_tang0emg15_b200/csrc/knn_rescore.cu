@@ -38,8 +38,9 @@
 namespace ksel {
 
 constexpr int kRsWarps = 4;
-constexpr int kRsRegs = 36;              // exact-pair buffer of 1152 per warp (>= k' + 32 for k' <= 1024)
-constexpr int kRsCap = 32 * kRsRegs;
+// exact-pair buffer per warp: 32 x rs_regs(R) pairs (>= k' + 32 for the queue k' = 32 R),
+// sized per queue so that small k keeps registers (the narrowing's) and occupancy up
+__host__ __device__ constexpr int rs_regs(int R) { return R <= 4 ? 12 : R <= 8 ? 16 : R <= 16 ? 24 : 36; }
 
 // The oracle's distance of one reference row (r: D floats, global) to the query held in
 // double (qd, shared memory): differences and squares in double, summed in index order.
@@ -156,7 +157,9 @@ static __device__ __noinline__ uint32_t lists_kth_key(const unsigned long long* 
 }
 
 template <int R>
-__global__ void __launch_bounds__(32 * kRsWarps) knn_rescore_kernel(const KnnRescoreArgs a) {
+__global__ void __launch_bounds__(32 * kRsWarps, 4) knn_rescore_kernel(const KnnRescoreArgs a) {
+    constexpr int kRsRegs = rs_regs(R);
+    constexpr int kRsCap = 32 * kRsRegs;
     __shared__ unsigned long long buf_all[kRsWarps][kRsCap];
     __shared__ double qd_all[kRsWarps][KNN_MAX_D];
     __shared__ uint32_t hist_all[kRsWarps][256];
