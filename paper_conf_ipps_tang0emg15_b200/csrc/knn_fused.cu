@@ -415,6 +415,12 @@ __device__ __forceinline__ void tmem_wait32(uint32_t (&v)[32]) {
                  : "memory");
 }
 
+__device__ __forceinline__ uint32_t atom_add_shared(uint32_t saddr, uint32_t v) {
+    uint32_t r;
+    asm volatile("atom.shared.add.u32 %0, [%1], %2;" : "=r"(r) : "r"(saddr), "r"(v) : "memory");
+    return r;
+}
+
 // min of three floats in one instruction (sm_100: FMNMX3; a NaN operand is ignored like fminf)
 __device__ __forceinline__ float fmin3(float a, float b, float c) {
     float r;
@@ -755,11 +761,13 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)  // (EW = 16: 18 warps, 5 
         const uint32_t shist_s = smem_u32(shist);
         float s_lo = 0.f, s_hi = -1.f, s_inv = 0.f;
         unsigned long long thr_next = (qvalid && !DUMP && !PIPE_ONLY) ? __ldcg(&qthr[q]) : kSentPair;
+        int ncheck = 1;  // tiles until the next bound refresh / narrowing check
         for (int lt = 0; lt < nsteps; ++lt) {
             const bool sampling = lt < Fs;
             const int t = (sampling ? t0 + lt : t0 + lt - Fs) * g.tstride;
             const int b = lt & 1;
-            if (!DUMP && !PIPE_ONLY && lt % g.nstride == 0) {
+            if (!DUMP && !PIPE_ONLY && --ncheck <= 0) {
+                ncheck = g.nstride;
                 // adopt the tightest bound any split of this query had published when the
                 // previous check started (the load's latency hides behind those tiles)
                 adopt(thr_next);
@@ -880,7 +888,12 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)  // (EW = 16: 18 warps, 5 
                 const uint32_t colt = (uint32_t)t * BN;  // N < 2^31
                 const int nlim = (int)min((int64_t)BN, g.N - (int64_t)colt);  // valid columns of the tile
                 const bool live = qvalid && !failed;
-                const float tvs = __fmul_ru(tv, stl);  // (after this tile's starting-bound updates)
+                // the filter value of this tile in accumulator units: value(T) + band scaled up
+                // (rounded up: never rejects a candidate), +Inf without a finite bound (all
+                // values pass), NaN for a lane that takes nothing (every compare fails)
+                const float tvl = !live ? __int_as_float(0x7fc00000)
+                                        : (fast ? __fmul_ru(tv, stl) : __int_as_float(0x7f800000));
+                const uint32_t np_s = smem_u32(np);
                 auto scan32 = [&](const uint32_t(&v)[32], int c0) {
                     float gmn[8];  // 3-input minima (FMNMX3): 20 instructions per 32 values
 #pragma unroll
@@ -890,17 +903,17 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)  // (EW = 16: 18 warps, 5 
                                        __uint_as_float(v[4 * j + 3]));
                     const float mn = fmin3(fmin3(gmn[0], gmn[1], gmn[2]), fmin3(gmn[3], gmn[4], gmn[5]),
                                            fminf(gmn[6], gmn[7]));
-                    if (!__any_sync(kFull, live && (!fast || mn <= tvs))) return;
+                    if (!__any_sync(kFull, mn <= tvl)) return;
                     const unsigned long long cr0 = PROF ? clock64() : 0;
                     // rare path: each lane visits only its own candidate groups (a divergent
                     // loop of max-over-lanes length); the group's 4 values are picked from the
                     // registers by a 3-level select tree (registers cannot be indexed
-                    // dynamically).  An element with d == tv and a larger index than T's is a
+                    // dynamically; measured faster than a warp vote per group with static
+                    // indices).  An element with d == tv and a larger index than T's is a
                     // harmless extra pool entry (narrowing applies the exact pair order).
                     uint32_t gm = 0;
 #pragma unroll
-                    for (int u = 0; u < 8; ++u) gm |= (uint32_t)(!fast || gmn[u] <= tvs) << u;
-                    if (!live) gm = 0;
+                    for (int u = 0; u < 8; ++u) gm |= (uint32_t)(gmn[u] <= tvl) << u;
                     while (gm) {
                         const int u = __ffs(gm) - 1;
                         gm &= gm - 1u;
@@ -912,10 +925,12 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)  // (EW = 16: 18 warps, 5 
                             const uint32_t a2 = b0 ? v[20 + i] : v[16 + i], a3 = b0 ? v[28 + i] : v[24 + i];
                             const uint32_t c01 = b1 ? a1 : a0, c23 = b1 ? a3 : a2;
                             const float x = __uint_as_float(b2 ? c23 : c01);
-                            if (cu + i < nlim && (!fast || x <= tvs)) {
+                            if (x <= tvl && cu + i < nlim) {
                                 const float xu = x * inv;
-                                const float dc = (xu < 0.f) ? 0.f : xu;  // clamp, NaN propagates
-                                const int slot = (PAIR > 1) ? atomicAdd(np, 1) : (*np)++;
+                                const float dc = (xu < 0.f) ? 0.f : xu;  // clamp
+                                int slot;
+                                if constexpr (PAIR > 1) slot = (int)atom_add_shared(np_s, 1u);
+                                else slot = (*np)++;
                                 pool[slot] = ((unsigned long long)key_of(dc) << 32) | (colt + (uint32_t)(cu + i));
                                 if (PROF) prof_app++;
                             }
