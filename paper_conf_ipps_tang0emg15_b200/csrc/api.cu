@@ -78,6 +78,9 @@ int chunk_order_mode() {
         int m = (e && e[0] >= '0' && e[0] <= '3') ? e[0] - '0' : 3;
         const char* l = std::getenv("KSEL_LOOSE");
         if (l && l[0] == '1') m |= 4;
+        // bit 6: no speculative starting bound (KSEL_SPEC=0; result-preserving)
+        const char* sp = std::getenv("KSEL_SPEC");
+        if (sp && sp[0] == '0') m |= 64;
 #ifdef KSEL_EXPERIMENTS
         // phase-cost experiments of the pool kernel (results are wrong): bit 3 = no exact
         // admission path, bit 4 = no final select/sort/merge, bit 5 = no starting bound

@@ -233,6 +233,8 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
     float tv = 0.f;
     bool fast = false;
     int n = 0;
+    uint32_t bkey_r = kSentKey;  // the rigorous starting bound (kept for a failed speculation)
+    bool spec_active = false;    // the bound in force is a speculative one, not yet verified
 
     auto tighten = [&](uint32_t kk, uint32_t ki) {
         if (pair_lt(kk, ki, Tk, Ti)) { Tk = kk; Ti = ki; }
@@ -260,6 +262,7 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
         if (ties > 16u) exact_ties = true;
         const uint32_t kk = (uint32_t)(t >> 32), ki = (uint32_t)t;
         tighten(kk, ki);
+        spec_active = false;  // (the pool's k-th: >= k seen pairs at or below the bound now)
         if (WPR > 1 && lane == 0) atomicMin(grp_thr, t);
     };
     // Exact path of one sub-step: the elements of this lane are the 4*G floats at
@@ -316,7 +319,8 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
     };
 
     // ---- unaligned head and tail (< 4 elements each; pool is empty, cannot overflow) ---------
-    if (wig == 0) {
+    auto head_tail = [&]() {
+        if (wig != 0) return;
         const uint32_t nh = (uint32_t)(a0 - g0), nt = (uint32_t)(g1 - a1);
         bool valid = false;
         uint64_t g = 0;
@@ -330,7 +334,8 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
         }
         n += __popc(bal);
         __syncwarp();
-    }
+    };
+    head_tail();
 
     // ---- starting bound: the k-th smallest key of the first S staged chunks -----------
     // (up to S*CH = 2048 values already in flight; bisection over their keys with
@@ -338,7 +343,7 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
     // (key, largest index) bounds the k-th pair -- the stream then admits a few
     // times k candidates instead of everything until the pool first fills.
     constexpr int NB = Cfg::NB;
-    if (nmine >= NB && k <= NB * CH / 2 && !(order_mode & 32)) {
+    if (nmine >= NB && !(order_mode & 32)) {
         uint32_t keys[NB * CH / 128 * 4];
         uint32_t nreal = 0;
 #pragma unroll
@@ -360,7 +365,7 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
             }
         }
         nreal = __reduce_add_sync(kFull, nreal);
-        if (nreal >= (uint32_t)k) {
+        if (nreal >= (uint32_t)k && k <= NB * CH / 2) {
             // Bisection on the key bits below the common prefix of the smallest and
             // largest real key, stopped at bit kLow: the k-th key then lies in
             // [vkey, vkey + 2^kLow), so vkey | (2^kLow - 1) bounds it (>= k keys are
@@ -396,15 +401,79 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
             }
             const uint32_t bkey = early ? early - 1u : (top >= kLow) ? (vkey | ((1u << kLow) - 1u)) : kmax;
             tighten(bkey, 0x7ffffffeu);
+            bkey_r = bkey;
             if (WPR > 1 && lane == 0) atomicMin(grp_thr, ((unsigned long long)bkey << 32) | 0x7ffffffeu);
+        }
+        // Speculative bound (late r2; the kNN filter's idea, knn_fused.cu knn_spec_geometry):
+        // the j-th smallest of the m sampled keys, j = lambda + 6 sqrt(lambda) + 6 with lambda
+        // = k m / (this warp's element count).  On i.i.d. data the warp's count of keys <= it
+        // is ~ (len / m) Gamma(j) >= k except with probability < 1e-10, so the stream admits
+        // ~j len / m candidates instead of the ~k len / m of the rigorous bound (k-th of the
+        // sample) and rarely narrows.  Verified at the end of the warp's share (>= k pool
+        // pairs, or a narrowing / a group bound below it); otherwise the share is streamed
+        // again from the rigorous bound.  Sampled chunks with disjoint key ranges (sorted
+        // data: not a random sample) get no speculation.
+        // (k > 128 only: measured on C2, speculation gains 7-46 % at k = 256 / 1024 and
+        // costs 0-7 % at k <= 32 -- a few narrowings at most to save there)
+        if (!(order_mode & 64) && k > 128 && nreal >= 64u) {
+            uint32_t cmin[NB], cmax[NB];
+#pragma unroll
+            for (int li = 0; li < NB; ++li) {
+                uint32_t lo = 0xffffffffu, hi = 0u;
+#pragma unroll
+                for (int j = 0; j < CH / 128 * 4; ++j) {
+                    const uint32_t kk2 = keys[li * (CH / 128) * 4 + j];
+                    if (kk2 != 0xffffffffu) { lo = min(lo, kk2); hi = max(hi, kk2); }
+                }
+                cmin[li] = __reduce_min_sync(kFull, lo);
+                cmax[li] = __reduce_max_sync(kFull, hi);
+            }
+            uint32_t lo_max = 0u, hi_min = 0xffffffffu;
+#pragma unroll
+            for (int li = 0; li < NB; ++li) { lo_max = max(lo_max, cmin[li]); hi_min = min(hi_min, cmax[li]); }
+            const uint64_t wlen = min((uint64_t)c_end * CH, (uint64_t)body_len) - (uint64_t)c_begin * CH;
+            const double lam = (double)k * (double)nreal / (double)wlen;
+            const uint32_t jj = (uint32_t)ceil(lam + 6.0 * sqrt(lam) + 6.0);
+            if (lo_max <= hi_min && jj < (uint32_t)k && jj < nreal) {
+                uint32_t kmin2 = 0xffffffffu, kmax2 = 0u;
+#pragma unroll
+                for (int j = 0; j < NB * CH / 128 * 4; ++j) {
+                    kmin2 = min(kmin2, keys[j]);
+                    kmax2 = max(kmax2, keys[j]);
+                }
+                kmin2 = __reduce_min_sync(kFull, kmin2);
+                kmax2 = __reduce_max_sync(kFull, kmax2);
+                constexpr int kLow = 16;
+                const int top = (kmin2 == kmax2) ? -1 : 31 - __clz(kmin2 ^ kmax2);
+                uint32_t vj = (top < 0) ? kmin2 : (kmin2 & ~((2u << top) - 1u));
+#pragma unroll 1
+                for (int bit = top; bit >= kLow; --bit) {
+                    const uint32_t cand = vj | (1u << bit);
+                    uint32_t c = 0;
+#pragma unroll
+                    for (int j = 0; j < NB * CH / 128 * 4; ++j) c += (keys[j] < cand) ? 1u : 0u;
+                    c = __reduce_add_sync(kFull, c);
+                    if (c < jj) vj = cand;
+                }
+                const uint32_t skey = (top >= kLow) ? (vj | ((1u << kLow) - 1u)) : kmax2;
+                if (skey < Tk) {  // (the speculative pair (skey, 0x7ffffffe) below the bound in force)
+                    tighten(skey, 0x7ffffffeu);
+                    spec_active = true;
+                }
+            }
         }
     }
 
     // ---- streaming body ------------------------------------------------------------------
-    for (int li = 0; li < nmine; ++li) {
+    // (pass 2, after a failed speculation, continues the ring's stage / barrier-phase
+    // sequence: li runs on from nmine, so every mbarrier keeps its phase parity)
+    int li0 = 0;
+    for (;;) {
+    for (int li = li0; li < li0 + nmine; ++li) {
         const int st = li % S;
         if (WPR > 1) {
             const unsigned long long sh = *reinterpret_cast<volatile unsigned long long*>(grp_thr);
+            if (pair_lt((uint32_t)(sh >> 32), (uint32_t)sh, Tk, Ti)) spec_active = false;  // a verified bound takes over
             tighten((uint32_t)(sh >> 32), (uint32_t)sh);
         }
         // (a suspended wait: a warp whose data has not landed leaves its issue slots to
@@ -463,9 +532,29 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
             if (go && !(order_mode & 8)) exact(srcf, (uint32_t)g, len, col0, x);
             if (last) {
                 __syncwarp();
-                if (lane == 0 && li + S < nmine) issue(li + S);
+                if (lane == 0 && li + S < li0 + nmine) issue(li + S);
             }
         }
+    }
+
+    if (!(spec_active && n < k)) break;
+    // The speculative bound failed (fewer than k of this warp's pairs at or below it): stream
+    // the share again from the rigorous bound (the ring is drained: every issued chunk was
+    // consumed; the visit order restarts, the stage sequence continues).
+    spec_active = false;
+    n = 0;
+    Tk = kSentKey;
+    Ti = kSentIdx;
+    fast = false;
+    if (bkey_r != kSentKey) tighten(bkey_r, 0x7ffffffeu);
+    __syncwarp();
+    li0 = nmine;
+    if (lane == 0) {
+        it_i = 0; it_blk = 0; it_off = 1; it_tail = np * step; it_p = 0;
+        for (int li = li0; li < li0 + S && li < li0 + nmine; ++li) issue(li);
+    }
+    __syncwarp();
+    head_tail();
     }
 
     // ---- finish: exact top-k of this warp's share, sorted -----------------------------------

@@ -495,3 +495,23 @@ def test_fuzz_clustered_ties_many_narrowings(K, oracle_mod, seed):
                 torch.cuda.synchronize()
                 assert_same(ev, ei, gv, gi, "clustered seed=%d case=%d Q=%d N=%d k=%d algo=%d wpr=%d"
                             % (seed, case, Q, N, k, algo, wpr))
+
+
+@pytest.mark.parametrize("k", [32, 256, 1000])
+@pytest.mark.parametrize("wpr", [1, 2])
+def test_speculative_bound_failure_restreams(K, oracle_mod, k, wpr):
+    """The pool kernel's speculative starting bound (the j-th of the sampled chunks) assumes the
+    sample is representative.  Here every warp's sampled chunks (its first and last chunks:
+    visit order 3) hold the row's smallest values, so the j-th sampled key has fewer than k of
+    the warp's keys below it: the verification at the end of the share fails, the share is
+    streamed again from the rigorous bound -- and the result must still be the oracle's."""
+    Q, N = 24, 65536
+    x = synth.rows("U", synth.seed_for(21, "U"), 0, Q, N) * 0.5 + 0.5  # U[0.5, 1)
+    small = synth.rows("U", synth.seed_for(22, "U"), 0, Q, N) * 1e-3    # U[0, 1e-3)
+    nch = N // 512
+    L = (k + 511) // 512 + 1
+    for w in range(wpr):
+        c0, c1 = nch * w // wpr, nch * (w + 1) // wpr
+        for c in [c0] + list(range(c1 - L, c1)):
+            x[:, c * 512:(c + 1) * 512] = small[:, c * 512:(c + 1) * 512]
+    _check_select(K, oracle_mod, x.contiguous(), k, "spec-fail k=%d wpr=%d" % (k, wpr), algo=2, wpr=wpr)
