@@ -153,12 +153,15 @@ KSEL_API int ksel_merge(const float* cand_val, const int32_t* cand_idx, int64_t 
  *   d_work   device workspace of >= knn_search_workspace(N, Q, D, k) bytes
  *            (fp16 operand images, per-query candidate pools; queries are
  *            processed in chunks so that the pools stay below 2 GiB).
- * Method: a one-pass fp16 tcgen05 GEMM (|q|^2 + |r|^2 - 2 q.r, TMEM accumulator)
- * FILTERS the references with a rigorous error bound eps_q (R21),
- * keeping every reference whose filter distance is within 2 eps_q of a k-th
- * value; the survivors are rescored exactly and selected.  Queries whose band of
- * near-equal filter distances overflows a pool (or with non-finite inputs) are
- * solved by an exact brute-force fallback on the device.
+ * Method: a one-pass fp16 tcgen05 GEMM on centred operands scaled per tile by
+ * powers of two (|q'|^2 + |r'|^2 - 2 q'.r', TMEM accumulator) FILTERS the
+ * references with a rigorous error bound eps_q (R21), keeping every
+ * reference whose filter distance is within 2 eps_q of a k-th value, starting
+ * from a speculative per-query bound (a sampled pre-pass of the same kernel,
+ * verified afterwards); the survivors are rescored exactly and selected.  Queries
+ * whose band of near-equal filter distances overflows a pool, whose speculative
+ * bound fails its verification, or with non-finite inputs are solved by an exact
+ * brute-force fallback on the device.
  * The Q x N distance matrix is never written to memory. */
 KSEL_API size_t knn_search_workspace(int64_t N, int64_t Q, int D, int k);
 KSEL_API int knn_search(const float* ref, const float* query, int64_t N, int64_t Q, int D, int k,
