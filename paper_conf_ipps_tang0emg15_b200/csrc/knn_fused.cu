@@ -139,29 +139,48 @@ __device__ __forceinline__ uint32_t h2(float a, float b) {
 // make |x'| small), and a coarse c keeps x' = x - c exact for integer-valued data (then
 // every fp16 operand is exact).  c = 0 for the padding dims.  knn_sum_kernel: block
 // (x, y) adds dims [32x, 32x + 32) of rows y*8 + warp + 256 i of the sample into csum
-// (double atomics; [2][Dp]: sums, sums of squares); knn_center_value turns them into c.
+// (double atomics; [2][Dp]: sums, sums of squares; then [2][Dp] u32: the sample's min and
+// max per dim as order keys, min stored inverted so that both are atomicMax from 0);
+// knn_center_value turns them into c, knn_sample_range into the largest |x - c| sampled.
 __global__ void __launch_bounds__(256)
     knn_sum_kernel(const float* __restrict__ ref, int64_t N, int D, int Dp, double* __restrict__ csum) {
     __shared__ double part[2][8][33];
+    __shared__ uint32_t pk[2][8][33];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int d = blockIdx.x * 32 + lane;
     const int64_t ns = N < 16384 ? N : 16384;
     const int64_t stride = N / ns;
     double s = 0.0, s2 = 0.0;
+    uint32_t kmn = 0u, kmx = 0u;  // (inverted min key, max key)
     if (d < D)
         for (int64_t i = (int64_t)blockIdx.y * 8 + warp; i < ns; i += 8 * (int64_t)gridDim.y) {
-            const double v = (double)__ldg(ref + (i * stride) * D + d);
+            const float f = __ldg(ref + (i * stride) * D + d);
+            const double v = (double)f;
             s += v;
             s2 += v * v;
+            const uint32_t kk = key_of(f);
+            kmn = max(kmn, ~kk);
+            kmx = max(kmx, kk);
         }
     part[0][warp][lane] = s;
     part[1][warp][lane] = s2;
+    pk[0][warp][lane] = kmn;
+    pk[1][warp][lane] = kmx;
     __syncthreads();
     if (warp == 0 && d < D) {
         double t = 0.0, t2 = 0.0;
-        for (int w = 0; w < 8; ++w) { t += part[0][w][lane]; t2 += part[1][w][lane]; }
+        uint32_t a = 0u, b = 0u;
+        for (int w = 0; w < 8; ++w) {
+            t += part[0][w][lane];
+            t2 += part[1][w][lane];
+            a = max(a, pk[0][w][lane]);
+            b = max(b, pk[1][w][lane]);
+        }
         atomicAdd(csum + d, t);
         atomicAdd(csum + Dp + d, t2);
+        uint32_t* ck = reinterpret_cast<uint32_t*>(csum + 2 * Dp);
+        atomicMax(ck + d, a);
+        atomicMax(ck + Dp + d, b);
     }
 }
 __device__ __forceinline__ float knn_center_value(const double* csum, int64_t N, int D, int Dp, int d) {
@@ -175,7 +194,149 @@ __device__ __forceinline__ float knn_center_value(const double* csum, int64_t N,
     return (float)(rint(m / gstep) * gstep);
 }
 
+// largest |x - c_d| over the sample in dim d (0 for padding dims; +Inf if not finite)
+__device__ __forceinline__ float knn_sample_range(const double* csum, int D, int Dp, int d, float c) {
+    if (d >= D) return 0.f;
+    const uint32_t* ck = reinterpret_cast<const uint32_t*>(csum + 2 * Dp);
+    const float vmin = __uint_as_float(bits_of_key(~ck[d])), vmax = __uint_as_float(bits_of_key(ck[Dp + d]));
+    const double r = fmax((double)vmax - (double)c, (double)c - (double)vmin);
+    return (r == r && r < 3.0e38) ? (float)r : __int_as_float(0x7f800000);
+}
+
 constexpr int KNN_PREP_THREADS = 256;
+
+// knn_prep1_kernel: the operand images in ONE read of the points.  Every tile takes the
+// call's common power-of-two scale sigma from the sample's range M (the largest |x - c|
+// sampled): refs 2^(13 - ilogb M), queries 2^(12 - ilogb M), so a value up to 2 M still
+// lands below 2^15 in fp16.  A tile holding a larger value (an outlier the sample missed)
+// is listed for knn_stats_kernel + knn_prep_kernel, which rebuild it from its own max.
+// Each block reads its tile 32 dims at a time (coalesced: a warp reads 32 consecutive
+// floats of one row) into shared memory; thread i owns row i: |x'|^2 in double, the
+// scaled fp16 chunks (16 B per thread, consecutive threads -> consecutive 16 B), then the
+// bf16 norm block.  Rows past the end are all zeros.
+__global__ void __launch_bounds__(256)
+    knn_prep1_kernel(const float* __restrict__ ref, const float* __restrict__ qry, KnnGeom g, int nt,
+                     const double* __restrict__ csum, float4* __restrict__ qstat, float2* __restrict__ tscale,
+                     KnnStats* __restrict__ st, uint4* __restrict__ ref_img, uint4* __restrict__ q_img,
+                     int* __restrict__ fixlist, int* __restrict__ fixcnt) {
+    __shared__ float tile[KNN_BN][KNN_KS + 1];
+    __shared__ float cs[KNN_MAX_D];
+    __shared__ uint32_t srange, smax;
+    __shared__ int sover, sbad;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tid == 0) { srange = 0u; smax = 0u; sover = 0; sbad = 0; }
+    __syncthreads();
+    for (int d = tid; d < g.Dp; d += 256) {
+        const float c = knn_center_value(csum, g.N, g.D, g.Dp, d);
+        cs[d] = c;
+        const float r = knn_sample_range(csum, g.D, g.Dp, d, c);
+        if (r > 0.f) atomicMax(&srange, __float_as_uint(r));
+    }
+    __syncthreads();
+    const bool is_q = blockIdx.x >= (unsigned)nt;
+    const int64_t t = is_q ? (int64_t)blockIdx.x - nt : (int64_t)blockIdx.x;
+    const int rows = is_q ? KNN_BM : g.BN;
+    const int64_t n = is_q ? g.Q : g.N;
+    const float* x = is_q ? qry : ref;
+    const int64_t row = t * rows + tid;
+    const float M = __uint_as_float(srange);
+    int e = 0;
+    if (M > 0.f && M < 3.0e38f) e = min(max((is_q ? 12 : 13) - ilogbf(M), -120), 120);
+    const float sig = ldexpf(1.f, e);
+    const float mul = is_q ? -2.f * sig : sig;  // exact
+    // (D % 4 == 0 and a 16-byte aligned base: every row is 16-byte aligned)
+    const bool vec4 = (g.D & 3) == 0 && (reinterpret_cast<uintptr_t>(x) & 15u) == 0;
+    double s = 0.0;
+    bool over = false, bad = false;
+    for (int ks = 0; ks < g.KS; ++ks) {
+        __syncthreads();
+        if (vec4) {
+            // 16-byte loads: lane l reads dims 4 (l % 8) .. + 3 of row r + l / 8 (512 B per
+            // warp instruction, 8 loads in flight per lane)
+            const int dq = ks * KNN_KS + 4 * (lane & 7);
+#pragma unroll 8
+            for (int r = warp * 4 + (lane >> 3); r < rows; r += 32) {
+                const int64_t gr = t * rows + r;
+                float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+                if (gr < n && dq < g.D) v = __ldcs(reinterpret_cast<const float4*>(x + gr * (int64_t)g.D + dq));
+                const bool ok = gr < n && dq < g.D;
+                float* tr = &tile[r][4 * (lane & 7)];
+                tr[0] = ok ? v.x - cs[dq] : 0.f;
+                tr[1] = ok ? v.y - cs[dq + 1] : 0.f;
+                tr[2] = ok ? v.z - cs[dq + 2] : 0.f;
+                tr[3] = ok ? v.w - cs[dq + 3] : 0.f;
+            }
+        } else {
+            const int d = ks * KNN_KS + lane;
+#pragma unroll 8
+            for (int r = warp; r < rows; r += 8) {
+                const int64_t gr = t * rows + r;
+                tile[r][lane] = (gr < n && d < g.D) ? __ldcs(x + gr * (int64_t)g.D + d) - cs[d] : 0.f;
+            }
+        }
+        __syncthreads();
+        if (tid < rows) {
+            uint4* dst;
+            int cstride;
+            if (is_q) {  // [Dp/8 chunks][128 rows][8]
+                dst = q_img + t * (int64_t)(g.a_bytes() / 16) + (int64_t)(ks * 4) * KNN_BM + tid;
+                cstride = KNN_BM;
+            } else {     // [stage][4 chunks][BN rows][8]
+                dst = ref_img + t * (int64_t)(g.tile_bytes() / 16) + (int64_t)ks * (g.stage_bytes() / 16) + tid;
+                cstride = g.BN;
+            }
+#pragma unroll
+            for (int kc = 0; kc < 4; ++kc) {
+                uint32_t h[4];
+#pragma unroll
+                for (int p = 0; p < 4; ++p) {
+                    const float v0 = tile[tid][kc * 8 + 2 * p], v1 = tile[tid][kc * 8 + 2 * p + 1];
+                    s += (double)v0 * (double)v0;
+                    s += (double)v1 * (double)v1;
+                    const float a0 = fabsf(v0), a1 = fabsf(v1);
+                    bad |= !(a0 <= 3.4028235e38f) || !(a1 <= 3.4028235e38f);
+                    over |= fabsf(mul * v0) >= 32768.f || fabsf(mul * v1) >= 32768.f;
+                    h[p] = h2(mul * v0, mul * v1);
+                }
+                dst[kc * cstride] = make_uint4(h[0], h[1], h[2], h[3]);
+            }
+        }
+    }
+    if (tid < rows) {
+        float sr = __double2float_ru(s);
+        if (bad || !(sr == sr)) sr = __int_as_float(0x7f800000);
+        if (row < n) {
+            if (is_q) qstat[row] = make_float4(sig, 0.f, 0.f, sr);
+            else atomicMax(&smax, __float_as_uint(sr));
+        }
+        const float n1 = __bfloat162float(__float2bfloat16_rn((float)s));
+        const float n2 = __bfloat162float(__float2bfloat16_rn((float)(s - (double)n1)));
+        const float n3 = __bfloat162float(__float2bfloat16_rn((float)(s - (double)n1 - (double)n2)));
+        uint4* blk;
+        uint4 c0;
+        if (is_q) {
+            blk = q_img + (t * (int64_t)g.a_bytes() + (int64_t)g.Dp * 256) / 16;
+            c0 = make_uint4(bf2(sig * n1, sig * n2), bf2(sig * n3, sig), bf2(sig, sig), 0u);
+        } else {
+            blk = ref_img + (t * (int64_t)g.tile_bytes() + (int64_t)g.KS * g.stage_bytes()) / 16;
+            c0 = make_uint4(bf2(sig, sig), bf2(sig, sig * n1), bf2(sig * n2, sig * n3), 0u);
+        }
+        if (row >= n) c0 = make_uint4(0u, 0u, 0u, 0u);
+        blk[tid] = c0;
+        blk[rows + tid] = make_uint4(0u, 0u, 0u, 0u);
+        if (over && !bad) sover = 1;
+        if (bad) sbad = 1;
+    }
+    __syncthreads();
+    if (tid == 0) {
+        if (sover && !sbad) fixlist[atomicAdd(fixcnt, 1)] = (int)blockIdx.x;  // rebuilt from its own max
+        if (!is_q) {
+            tscale[t] = make_float2(sig, 1.f / sig);  // (exact: a power of two)
+            if (smax) atomicMax(&st->R2, smax);
+            atomicMax(&st->isig, __float_as_uint(1.f / sig));
+        }
+    }
+}
 
 // knn_stats_kernel: one block per tile (blocks [0, nt): reference tiles of BN rows, then
 // query tiles of 128 rows); a warp per row, coalesced.  Per row |x'|^2 in double (rownorm),
@@ -184,16 +345,22 @@ constexpr int KNN_PREP_THREADS = 256;
 __global__ void __launch_bounds__(KNN_PREP_THREADS)
     knn_stats_kernel(const float* __restrict__ ref, const float* __restrict__ qry, KnnGeom g, int nt,
                      const double* __restrict__ csum, double* __restrict__ rownorm, float4* __restrict__ qstat,
-                     float2* __restrict__ tscale, KnnStats* __restrict__ st) {
+                     float2* __restrict__ tscale, KnnStats* __restrict__ st, const int* __restrict__ list,
+                     const int* __restrict__ lcnt) {
     __shared__ float cs[KNN_MAX_D];
     __shared__ uint32_t samx, smax;
     __shared__ int sbad;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    if (tid == 0) { samx = 0u; smax = 0u; sbad = 0; }
     for (int d = tid; d < g.Dp; d += KNN_PREP_THREADS) cs[d] = knn_center_value(csum, g.N, g.D, g.Dp, d);
+    // (list != nullptr: the tiles knn_prep1_kernel listed, a grid-stride loop over them)
+    const int nb = list ? *lcnt : (int)gridDim.x;
+    for (int li = (int)blockIdx.x; li < nb; li += (int)gridDim.x) {
+    const unsigned bid = list ? (unsigned)list[li] : blockIdx.x;
     __syncthreads();
-    const bool is_q = blockIdx.x >= (unsigned)nt;
-    const int64_t t = is_q ? (int64_t)blockIdx.x - nt : (int64_t)blockIdx.x;
+    if (tid == 0) { samx = 0u; smax = 0u; sbad = 0; }
+    __syncthreads();
+    const bool is_q = bid >= (unsigned)nt;
+    const int64_t t = is_q ? (int64_t)bid - nt : (int64_t)bid;
     const int rows = is_q ? KNN_BM : g.BN;
     const int64_t n = is_q ? g.Q : g.N;
     const float* x = is_q ? qry : ref;
@@ -225,7 +392,7 @@ __global__ void __launch_bounds__(KNN_PREP_THREADS)
             for (int o = 16; o > 0; o >>= 1) s[u] += __shfl_xor_sync(kFull, s[u], o);
             const int64_t gr = t * rows + r0 + u;
             if (lane == 0 && r0 + u < rows) {
-                rownorm[blockIdx.x * (int64_t)KNN_BN + r0 + u] = s[u];
+                rownorm[bid * (int64_t)KNN_BN + r0 + u] = s[u];
                 if (gr < n) {
                     float sr = __double2float_ru(s[u]);
                     if (!(sr == sr)) sr = __int_as_float(0x7f800000);
@@ -259,6 +426,7 @@ __global__ void __launch_bounds__(KNN_PREP_THREADS)
         atomicMax(&st->R2, sbad ? 0x7f800000u : smax);
         atomicMax(&st->isig, __float_as_uint(1.f / sig));
     }
+    }
 }
 
 // knn_prep_kernel: the operand images.  Each block reads its tile 32 dims at a time
@@ -273,13 +441,17 @@ __global__ void __launch_bounds__(KNN_PREP_THREADS)
     knn_prep_kernel(const float* __restrict__ ref, const float* __restrict__ qry, KnnGeom g, int nt,
                     const double* __restrict__ csum, const double* __restrict__ rownorm,
                     const float4* __restrict__ qstat, const float2* __restrict__ tscale,
-                    uint4* __restrict__ ref_img, uint4* __restrict__ q_img) {
+                    uint4* __restrict__ ref_img, uint4* __restrict__ q_img, const int* __restrict__ list,
+                    const int* __restrict__ lcnt) {
     __shared__ float tile[KNN_BN][KNN_KS + 1];
     __shared__ float cs[KNN_MAX_D];
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     for (int d = tid; d < g.Dp; d += KNN_PREP_THREADS) cs[d] = knn_center_value(csum, g.N, g.D, g.Dp, d);
-    const bool is_q = blockIdx.x >= (unsigned)nt;
-    const int64_t t = is_q ? (int64_t)blockIdx.x - nt : (int64_t)blockIdx.x;
+    const int nb = list ? *lcnt : (int)gridDim.x;
+    for (int li = (int)blockIdx.x; li < nb; li += (int)gridDim.x) {
+    const unsigned bid = list ? (unsigned)list[li] : blockIdx.x;
+    const bool is_q = bid >= (unsigned)nt;
+    const int64_t t = is_q ? (int64_t)bid - nt : (int64_t)bid;
     const int rows = is_q ? KNN_BM : g.BN;
     const int64_t n = is_q ? g.Q : g.N;
     const float* x = is_q ? qry : ref;
@@ -315,7 +487,7 @@ __global__ void __launch_bounds__(KNN_PREP_THREADS)
         }
     }
     if (tid < rows) {
-        const double s = rownorm[blockIdx.x * (int64_t)KNN_BN + tid];
+        const double s = rownorm[bid * (int64_t)KNN_BN + tid];
         const float n1 = __bfloat162float(__float2bfloat16_rn((float)s));
         const float n2 = __bfloat162float(__float2bfloat16_rn((float)(s - (double)n1)));
         const float n3 = __bfloat162float(__float2bfloat16_rn((float)(s - (double)n1 - (double)n2)));
@@ -331,6 +503,8 @@ __global__ void __launch_bounds__(KNN_PREP_THREADS)
         if (row >= n) c0 = make_uint4(0u, 0u, 0u, 0u);
         blk[tid] = c0;
         blk[rows + tid] = make_uint4(0u, 0u, 0u, 0u);
+    }
+    __syncthreads();
     }
 }
 
@@ -1019,7 +1193,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)  // (EW = 16: 18 warps, 5 
 static size_t al256(size_t x) { return (x + 255u) & ~(size_t)255u; }
 
 struct KnnWork {
-    size_t ref_img, tscale, csum, rownorm, stats, q_img, qstat, pool, cnt, qthr, qspec, qfail, fb, prof, total;
+    size_t ref_img, tscale, csum, rownorm, fix, stats, q_img, qstat, pool, cnt, qthr, qspec, qfail, fb, prof, total;
 };
 
 // Queries are processed in chunks (multiples of 128 queries) so that the pools,
@@ -1186,7 +1360,8 @@ static KnnWork knn_work_layout(const KnnGeom& g) {
     size_t off = 0;
     w.ref_img = off; off += al256((size_t)g.NT * g.tile_bytes());
     w.tscale = off;  off += al256((size_t)g.NT * 8);
-    w.csum = off;    off += al256((size_t)g.Dp * 16);
+    w.csum = off;    off += al256((size_t)g.Dp * 24);
+    w.fix = off;     off += al256((size_t)(g.NT + g.QTp * g.QPC + 1) * 4);  // [count][tiles to rebuild]
     w.rownorm = off; off += al256((size_t)(g.NT + g.QTp * g.QPC) * KNN_BN * 8);
     w.stats = off;   off += al256(sizeof(KnnStats));
     w.q_img = off;   off += al256((size_t)g.QTp * g.QPC * g.a_bytes());
@@ -1243,6 +1418,8 @@ static cudaError_t knn_run(const float* ref, const float* query, int64_t N, int6
     float2* tscale = reinterpret_cast<float2*>(work + w.tscale);
     double* csum = reinterpret_cast<double*>(work + w.csum);
     double* rownorm = reinterpret_cast<double*>(work + w.rownorm);
+    int* fixcnt = reinterpret_cast<int*>(work + w.fix);
+    int* fixlist = fixcnt + 1;
     cudaError_t e = cudaMemsetAsync(stats, 0, sizeof(KnnStats), stream);
     if (e != cudaSuccess) return e;
     for (int64_t q0 = 0; q0 < Q; q0 += Qc) {
@@ -1250,16 +1427,23 @@ static cudaError_t knn_run(const float* ref, const float* query, int64_t N, int6
         const KnnGeom g = knn_geometry(N, nq, D, k, sms, idx_offset, (int64_t)gq.S * Qc);
         const int nt = (q0 == 0) ? g.NT : 0;  // reference tiles: first chunk only
         if (nt > 0) {
-            e = cudaMemsetAsync(csum, 0, (size_t)g.Dp * 16, stream);
+            e = cudaMemsetAsync(csum, 0, (size_t)g.Dp * 24, stream);
             if (e != cudaSuccess) return e;
             knn_sum_kernel<<<dim3((unsigned)(g.Dp / 32), 32), 256, 0, stream>>>(ref, N, D, g.Dp, csum);
             note_launch();
         }
-        knn_stats_kernel<<<(unsigned)(nt + g.QT), KNN_PREP_THREADS, 0, stream>>>(
-            ref, query + q0 * (int64_t)D, g, nt, csum, rownorm, qstat, tscale, stats);
+        e = cudaMemsetAsync(fixcnt, 0, 4, stream);
+        if (e != cudaSuccess) return e;
+        // one read of the points at the call's common scale; then the (rare) tiles whose
+        // values exceed it rebuilt from their own max (grid-stride over the list: usually empty)
+        knn_prep1_kernel<<<(unsigned)(nt + g.QT), 256, 0, stream>>>(ref, query + q0 * (int64_t)D, g, nt, csum, qstat,
+                                                                    tscale, stats, ref_img, q_img, fixlist, fixcnt);
         note_launch();
-        knn_prep_kernel<<<(unsigned)(nt + g.QT), KNN_PREP_THREADS, 0, stream>>>(
-            ref, query + q0 * (int64_t)D, g, nt, csum, rownorm, qstat, tscale, ref_img, q_img);
+        knn_stats_kernel<<<(unsigned)sms, KNN_PREP_THREADS, 0, stream>>>(
+            ref, query + q0 * (int64_t)D, g, nt, csum, rownorm, qstat, tscale, stats, fixlist, fixcnt);
+        note_launch();
+        knn_prep_kernel<<<(unsigned)sms, KNN_PREP_THREADS, 0, stream>>>(
+            ref, query + q0 * (int64_t)D, g, nt, csum, rownorm, qstat, tscale, ref_img, q_img, fixlist, fixcnt);
         note_launch();
         e = cudaGetLastError();
 #ifdef KSEL_EXPERIMENTS

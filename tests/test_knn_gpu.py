@@ -335,3 +335,24 @@ def test_knn_search_query_chunks(K, oracle_mod):
     torch.cuda.synchronize()
     sample = list(range(0, Q, Q // 40)) + [Q - 1]
     check_knn(oracle_mod, ref.cpu(), qry[sample].cpu(), k, gv[sample], gi[sample])
+
+
+@pytest.mark.parametrize("k", [5, 100])
+def test_knn_outlier_tiles_rebuilt(K, oracle_mod, k):
+    """The operand images take one power-of-two scale per call from a strided sample of the
+    references (knn_prep1_kernel); a tile holding a value the sample missed (here 1e4 on
+    rows the stride-2 sample skips, and a query tile with an outlier) would overflow fp16
+    and is rebuilt from its own max (knn_stats_kernel + knn_prep_kernel over the listed
+    tiles).  Distances, the filter bound and the neighbours must still be the oracle's."""
+    N, Q, D = 40000, 300, 64
+    ref = synth.knn_points("knn-U", 31, 0, N, D).clone()
+    qry = synth.knn_points("knn-U", 32, 0, Q, D).clone()
+    ref[1::4000, 3] = 1.0e4          # odd rows: never in the sample
+    ref[7777, :] = -3.0e3
+    qry[130, 5] = 2.0e4              # one query tile rebuilt as well
+    qry[131, :] = ref[7777, :]       # its nearest neighbour is the outlier row
+    gv, gi = K.knn_search(ref.cuda(), qry.cuda(), k)
+    check_knn(oracle_mod, ref, qry, k, gv, gi)
+    dg, eps = K.knn_distances(ref.cuda(), qry[:140].contiguous().cuda(), with_eps=True)
+    do = oracle_mod.knn_dist(ref.numpy(), qry[:140].numpy()).astype(np.float64)
+    assert np.all(np.abs(dg.cpu().numpy().astype(np.float64) - do) <= eps.cpu().numpy().astype(np.float64)[:, None])
