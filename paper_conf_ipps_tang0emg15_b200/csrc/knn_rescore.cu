@@ -103,57 +103,69 @@ __device__ __forceinline__ void emit_sorted(const unsigned long long* buf, int c
     }
 }
 
-// The want-th smallest KEY (d~) over the union of a query's S pools (global memory):
-// MSD radix select on the 32-bit key below the union's common prefix, one warp, the
-// per-warp histogram in shared memory (hist_find: ksel_pool.cuh).  Returns the key v
-// with #{key < v} < want <= #{key <= v}.
+// A bound on the want-th smallest KEY (d~) over the union of a query's S pools (global
+// memory): min / max (and, fused in, the count of pairs <= ts -- the speculative bound's
+// verification), then 8-bit histograms of the keys below their common prefix (MSD radix
+// select [12], the per-warp histogram in shared memory, hist_find: ksel_pool.cuh) until the
+// bucket holding the want-th key has <= 64 keys; its upper edge is returned (>= want keys
+// are <= it, at most that bucket's keys lie between).  Usually one histogram pass for
+// k <= 128, two for k = 1024.  *le_out = #{pairs <= ts}.
 static __device__ __noinline__ uint32_t lists_kth_key(const unsigned long long* __restrict__ pools, const int32_t* __restrict__ cnt,
                                               int S, int64_t Q, int64_t q, int64_t P, uint32_t want,
-                                              uint32_t* __restrict__ hist) {
+                                              uint32_t* __restrict__ hist, unsigned long long ts, int* le_out) {
     const uint32_t lane = lane_id();
     auto scan = [&](auto f) {
         for (int s = 0; s < S; ++s) {
             const int ns = cnt[(int64_t)s * Q + q];
             const unsigned long long* pr = pools + ((int64_t)s * Q + q) * P;
-            for (int base = 0; base < ns; base += 128) {
-                unsigned long long v[4];
+            for (int base = 0; base < ns; base += 256) {
+                unsigned long long v[8];
 #pragma unroll
-                for (int j = 0; j < 4; ++j) {
+                for (int j = 0; j < 8; ++j) {
                     const int x = base + j * 32 + (int)lane;
                     v[j] = (x < ns) ? __ldcg(pr + x) : ~0ull;
                 }
 #pragma unroll
-                for (int j = 0; j < 4; ++j)
-                    if (base + j * 32 + (int)lane < ns) f((uint32_t)(v[j] >> 32));
+                for (int j = 0; j < 8; ++j)
+                    if (base + j * 32 + (int)lane < ns) f(v[j]);
             }
         }
     };
     uint32_t kmin = 0xffffffffu, kmax = 0u;
-    scan([&](uint32_t kk) {
+    int le = 0;
+    scan([&](unsigned long long pr) {
+        const uint32_t kk = (uint32_t)(pr >> 32);
         kmin = min(kmin, kk);
         kmax = max(kmax, kk);
+        le += (pr <= ts) ? 1 : 0;
     });
     kmin = __reduce_min_sync(kFull, kmin);
     kmax = __reduce_max_sync(kFull, kmax);
+    *le_out = __reduce_add_sync(kFull, le);
+    if (want == 0u) return 0u;
     int hi = (kmin == kmax) ? -1 : 31 - __clz(kmin ^ kmax);
-    uint32_t prefix = (hi < 0) ? kmin : (kmin & ~((2u << hi) - 1u));
-    uint32_t cnt_b;
-    while (hi >= 0) {
+    if (hi < 0) return kmin;
+    uint32_t prefix = kmin & ~((2u << hi) - 1u);
+    for (;;) {
         const int lo = hi >= 7 ? hi - 7 : 0;
         const uint32_t dmask = (2u << (hi - lo)) - 1u;
 #pragma unroll
         for (int j = 0; j < 8; ++j) hist[j * 32 + lane] = 0u;
         __syncwarp();
-        scan([&](uint32_t kk) {
+        scan([&](unsigned long long pr) {
+            const uint32_t kk = (uint32_t)(pr >> 32);
             if (hi == 31 || ((kk ^ prefix) >> (hi + 1)) == 0u) atomicAdd(&hist[hist_slot((kk >> lo) & dmask)], 1u);
         });
         __syncwarp();
+        uint32_t cnt_b;
         const uint32_t d = hist_find(hist, lane, want, cnt_b);
-        prefix |= d << lo;
         __syncwarp();
+        prefix |= d << lo;
+        // stop once the want-th key's bucket is small: its upper edge is then a bound with
+        // few keys between it and the want-th (<= 64 extra candidates for the band)
+        if (cnt_b <= 64u || lo == 0) return prefix | ((1u << lo) - 1u);
         hi = lo - 1;
     }
-    return prefix;
 }
 
 template <int R>
@@ -184,27 +196,27 @@ __global__ void __launch_bounds__(32 * kRsWarps, 4) knn_rescore_kernel(const Knn
         // against min(T_spec, its verified bounds).  The pools then hold every reference with
         // d~ <= min(T_spec, thr) + band, so the band may start from T_spec only once T_spec is
         // VERIFIED -- at least k pooled pairs <= T_spec -- or from thr if thr <= T_spec.
-        // Otherwise the pools may miss part of the top-k: exact fallback.
+        // Otherwise the pools may miss part of the top-k: exact fallback.  (The count rides in
+        // the union scan that also bounds the k-th d~ when the union exceeds the buffer.)
         const unsigned long long ts = a.spec ? a.spec[q] : ~0ull;
-        if ((uint32_t)(ts >> 32) != kSentKey) {
+        const bool spec = (uint32_t)(ts >> 32) != kSentKey;
+        const bool big = tot > kRsCap && tot >= a.k;  // (a union that fits the buffer is band-narrowed there)
+        if (spec || big) {
             int le = 0;
-            for (int s = 0; s < a.S; ++s) {
-                const int ns = a.cnt[(int64_t)s * a.Q + q];
-                const unsigned long long* pr = a.pools + ((int64_t)s * a.Q + q) * a.P;
-                for (int x = (int)lane; x < ns; x += 32) le += (__ldcg(pr + x) <= ts) ? 1 : 0;
+            const uint32_t kk = lists_kth_key(a.pools, a.cnt, a.S, a.Q, q, a.P, big ? (uint32_t)a.k : 0u, hist_all[w], ts,
+                                              &le);
+            if (spec) {
+                if (le >= a.k) {
+                    T0 = ts < T0 ? ts : T0;
+                } else if (!(T0 <= ts)) {
+                    if (lane == 0) a.qfail[q] = 1;
+                    return;
+                }
             }
-            le = __reduce_add_sync(kFull, le);
-            if (le >= a.k) {
-                T0 = ts < T0 ? ts : T0;
-            } else if (!(T0 <= ts)) {
-                if (lane == 0) a.qfail[q] = 1;
-                return;
+            if (big) {
+                const unsigned long long t = ((unsigned long long)kk << 32) | 0xffffffffull;
+                T0 = t < T0 ? t : T0;
             }
-        }
-        if (tot > kRsCap && tot >= a.k) {  // (a union that fits the buffer is band-narrowed there)
-            const uint32_t kk = lists_kth_key(a.pools, a.cnt, a.S, a.Q, q, a.P, (uint32_t)a.k, hist_all[w]);
-            const unsigned long long t = ((unsigned long long)kk << 32) | 0xffffffffull;
-            T0 = t < T0 ? t : T0;
         }
     }
     unsigned long long Kb = band_bound(T0, band);  // candidates: pair <= Kb
@@ -225,14 +237,8 @@ __global__ void __launch_bounds__(32 * kRsWarps, 4) knn_rescore_kernel(const Knn
         }
         __syncwarp();
     };
-#pragma unroll 1
-    for (int s = 0; s < a.S; ++s) {
-        const int ns = a.cnt[(int64_t)s * a.Q + q];
-        const unsigned long long* pr = a.pools + ((int64_t)s * a.Q + q) * a.P;
-#pragma unroll 1
-        for (int base = 0; base < ns; base += 32) {
-            const int x = base + (int)lane;
-            const unsigned long long v = (x < ns) ? __ldcg(pr + x) : ~0ull;
+    // one pair of the gather (phase A / B); x: its slot, ns: the list's length
+    auto gather_one = [&](unsigned long long v, int x, int ns) {
             if (!exact_mode) {
                 bool keep = x < ns && v <= Kb;
                 uint32_t bal = __ballot_sync(kFull, keep);
@@ -256,7 +262,7 @@ __global__ void __launch_bounds__(32 * kRsWarps, 4) knn_rescore_kernel(const Knn
                     if (keep) buf[c + __popc(bal & lt)] = v;
                     c += __popc(bal);
                     __syncwarp();
-                    continue;
+                    return;
                 }
             }
             // phase B: a candidate whose d~ - eps_q exceeds the exact k-th so far cannot win
@@ -279,6 +285,24 @@ __global__ void __launch_bounds__(32 * kRsWarps, 4) knn_rescore_kernel(const Knn
             if (keep) buf[c + __popc(bal & lt)] = ex;
             c += __popc(bal);
             __syncwarp();
+    };
+#pragma unroll 1
+    for (int s = 0; s < a.S; ++s) {
+        const int ns = a.cnt[(int64_t)s * a.Q + q];
+        const unsigned long long* pr = a.pools + ((int64_t)s * a.Q + q) * a.P;
+#pragma unroll 1
+        for (int base = 0; base < ns; base += 128) {
+            unsigned long long v[4];  // (4 loads in flight per lane)
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const int x = base + j * 32 + (int)lane;
+                v[j] = (x < ns) ? __ldcg(pr + x) : ~0ull;
+            }
+#pragma unroll 1
+            for (int j = 0; j < 4 && base + j * 32 < ns; ++j) {
+                const unsigned long long vj = j == 0 ? v[0] : j == 1 ? v[1] : j == 2 ? v[2] : v[3];  // (no local array)
+                gather_one(vj, base + j * 32 + (int)lane, ns);
+            }
         }
     }
     if (!exact_mode) {  // phase A ended: the band set, rescored exactly
