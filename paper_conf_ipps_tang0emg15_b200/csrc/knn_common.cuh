@@ -73,7 +73,10 @@ struct KnnRescoreArgs {
     uint8_t* fb;                       // fallback workspace
     float* out_val;
     int32_t* out_idx;
+    unsigned long long* cand;          // [Q][kCandCap] the band of each query (rescore -> exact -> finish)
+    int32_t* ccount;                   // [Q] its length; -1: finished (phase B) or flagged
 };
+constexpr int kCandCap = 1600;         // the largest rescore buffer (k' = 1024: k + the band)
 
 // knn_rescore.cu
 cudaError_t launch_knn_rescore(const KnnRescoreArgs& a, cudaStream_t stream);

@@ -1193,7 +1193,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)  // (EW = 16: 18 warps, 5 
 static size_t al256(size_t x) { return (x + 255u) & ~(size_t)255u; }
 
 struct KnnWork {
-    size_t ref_img, tscale, csum, rownorm, fix, stats, q_img, qstat, pool, cnt, qthr, qspec, qfail, fb, prof, total;
+    size_t ref_img, tscale, csum, rownorm, fix, cand, ccount, stats, q_img, qstat, pool, cnt, qthr, qspec, qfail, fb, prof, total;
 };
 
 // Queries are processed in chunks (multiples of 128 queries) so that the pools,
@@ -1371,6 +1371,8 @@ static KnnWork knn_work_layout(const KnnGeom& g) {
     w.qthr = off;    off += al256((size_t)g.Q * 8);
     w.qspec = off;   off += al256((size_t)g.Q * 8);
     w.qfail = off;   off += al256((size_t)g.Q * 4);
+    w.cand = off;    off += al256((size_t)g.Q * kCandCap * 8);
+    w.ccount = off;  off += al256((size_t)g.Q * 4);
     w.fb = off;      off += al256(knn_fallback_bytes(g.k));
     w.prof = off;    off += al256((size_t)g.QTp * g.S * KNN_MAX_EW * 16 * 8);  // MODE 3 counters
     w.total = off;
@@ -1557,6 +1559,8 @@ static cudaError_t knn_run(const float* ref, const float* query, int64_t N, int6
         a.qstat = qstat;
         a.stats = stats;
         a.fb = work + w.fb;
+        a.cand = reinterpret_cast<unsigned long long*>(work + w.cand);
+        a.ccount = reinterpret_cast<int32_t*>(work + w.ccount);
         a.out_val = out_dist + q0 * k;
         a.out_idx = out_idx + q0 * k;
         e = launch_knn_rescore(a, stream);

@@ -37,10 +37,22 @@
 
 namespace ksel {
 
-constexpr int kRsWarps = 4;
+// warps (queries) per block: 3 for k' = 1024 (its 12.8 KB buffers), else 4
+__host__ __device__ constexpr int rs_warps(int R) { return R >= 32 ? 3 : 4; }
 // exact-pair buffer per warp: 32 x rs_regs(R) pairs (>= k' + 32 for the queue k' = 32 R),
 // sized per queue so that small k keeps registers (the narrowing's) and occupancy up
 __host__ __device__ constexpr int rs_regs(int R) { return R <= 4 ? 12 : R <= 8 ? 16 : R <= 16 ? 24 : 36; }
+// buffer capacity: k' = 1024 needs room for k + the band (C5: ~1250 pairs) -- beyond the
+// register narrowing's 32 x 36, narrowings there use the shared-histogram radix select
+__host__ __device__ constexpr int rs_cap(int R) { return R >= 32 ? kCandCap : 32 * rs_regs(R); }
+
+// the want-th pair of buf[0, n) (band >= 0: keep the band above it), in place
+template <int NR, bool GLOBAL>
+__device__ __forceinline__ unsigned long long narrow_any(unsigned long long* buf, int n, uint32_t want, int* nn,
+                                                         uint32_t* hist, float band = -1.f) {
+    if (n <= 32 * NR) return pool_narrow64<NR, GLOBAL>(buf, n, want, nn, band);
+    return pool_select64<GLOBAL>(buf, n, want, hist, nn, band);
+}
 
 // The oracle's distance of one reference row (r: D floats, global) to the query held in
 // double (qd, shared memory): differences and squares in double, summed in index order.
@@ -169,16 +181,21 @@ static __device__ __noinline__ uint32_t lists_kth_key(const unsigned long long* 
 }
 
 template <int R>
-__global__ void __launch_bounds__(32 * kRsWarps, 4) knn_rescore_kernel(const KnnRescoreArgs a) {
+__global__ void __launch_bounds__(32 * rs_warps(R), 4) knn_rescore_kernel(const KnnRescoreArgs a) {
+    constexpr int kRsWarps = rs_warps(R);
     constexpr int kRsRegs = rs_regs(R);
-    constexpr int kRsCap = 32 * kRsRegs;
+    constexpr int kRsCap = rs_cap(R);
     __shared__ unsigned long long buf_all[kRsWarps][kRsCap];
     __shared__ double qd_all[kRsWarps][KNN_MAX_D];
     __shared__ uint32_t hist_all[kRsWarps][256];
     const uint32_t lane = lane_id();
     const int w = threadIdx.x >> 5;
     const int64_t q = (int64_t)blockIdx.x * kRsWarps + w;
-    if (q >= a.Q || a.qfail[q]) return;
+    if (q >= a.Q) return;
+    if (a.qfail[q]) {
+        if (lane == 0) a.ccount[q] = -1;
+        return;
+    }
     unsigned long long* buf = buf_all[w];
     double* qd = qd_all[w];
     for (int t = (int)lane; t < a.D; t += 32) qd[t] = (double)a.query[q * a.D + t];
@@ -209,7 +226,7 @@ __global__ void __launch_bounds__(32 * kRsWarps, 4) knn_rescore_kernel(const Knn
                 if (le >= a.k) {
                     T0 = ts < T0 ? ts : T0;
                 } else if (!(T0 <= ts)) {
-                    if (lane == 0) a.qfail[q] = 1;
+                    if (lane == 0) { a.qfail[q] = 1; a.ccount[q] = -1; }
                     return;
                 }
             }
@@ -244,7 +261,7 @@ __global__ void __launch_bounds__(32 * kRsWarps, 4) knn_rescore_kernel(const Knn
                 uint32_t bal = __ballot_sync(kFull, keep);
                 if (c + __popc(bal) > kRsCap) {
                     int nn;
-                    const unsigned long long Ta = pool_narrow64<kRsRegs, false>(buf, c, (uint32_t)a.k, &nn, band);
+                    const unsigned long long Ta = narrow_any<kRsRegs, false>(buf, c, (uint32_t)a.k, &nn, hist_all[w], band);
                     c = nn;
                     const unsigned long long Kn = band_bound(Ta, band);
                     Kb = Kn < Kb ? Kn : Kb;
@@ -252,7 +269,7 @@ __global__ void __launch_bounds__(32 * kRsWarps, 4) knn_rescore_kernel(const Knn
                     bal = __ballot_sync(kFull, keep);
                     if (c + __popc(bal) > kRsCap) {  // the band alone overflows: phase B
                         rescore_buffer();
-                        Tx = pool_narrow64<kRsRegs, false>(buf, c, (uint32_t)a.k, &nn);
+                        Tx = narrow_any<kRsRegs, false>(buf, c, (uint32_t)a.k, &nn, hist_all[w]);
                         c = nn;
                         txv = key_value((uint32_t)(Tx >> 32));
                         exact_mode = true;
@@ -276,7 +293,7 @@ __global__ void __launch_bounds__(32 * kRsWarps, 4) knn_rescore_kernel(const Knn
             uint32_t bal = __ballot_sync(kFull, keep);
             if (c + __popc(bal) > kRsCap) {  // full: narrow to the exact k-th pair
                 int nn;
-                Tx = pool_narrow64<kRsRegs, false>(buf, c, (uint32_t)a.k, &nn);
+                Tx = narrow_any<kRsRegs, false>(buf, c, (uint32_t)a.k, &nn, hist_all[w]);
                 c = nn;
                 txv = key_value((uint32_t)(Tx >> 32));
                 keep = keep && ex <= Tx;
@@ -305,20 +322,69 @@ __global__ void __launch_bounds__(32 * kRsWarps, 4) knn_rescore_kernel(const Knn
             }
         }
     }
-    if (!exact_mode) {  // phase A ended: the band set, rescored exactly
+    if (!exact_mode) {  // phase A ended: the band set, rescored exactly by knn_exact_kernel
         if (c > a.k) {
             int nn;
-            pool_narrow64<kRsRegs, false>(buf, c, (uint32_t)a.k, &nn, band);
+            narrow_any<kRsRegs, false>(buf, c, (uint32_t)a.k, &nn, hist_all[w], band);
             c = nn;
         }
-        rescore_buffer();
+        unsigned long long* cq = a.cand + q * (int64_t)kCandCap;
+        for (int e = (int)lane; e < c; e += 32) cq[e] = buf[e];
+        if (lane == 0) a.ccount[q] = c;
+        return;
     }
+    if (lane == 0) a.ccount[q] = -1;  // (phase B finished this query here)
     if (c > a.k) {
         int nn;
-        pool_narrow64<kRsRegs, false>(buf, c, (uint32_t)a.k, &nn);
+        narrow_any<kRsRegs, false>(buf, c, (uint32_t)a.k, &nn, hist_all[w]);
         c = nn;
     }
     emit_sorted<R>(buf, c, a.k, a.idx_offset, a.out_val + q * a.k, a.out_idx + q * a.k, lane);
+}
+
+// knn_exact_kernel: the exact distances of every query's band (cand[q][0, ccount[q])), one
+// warp per query, one lane per candidate row -- the register-light half of the rescoring
+// (no narrowing / sorting state), so 32+ warps per SM keep the random 512-byte row
+// gathers in flight (inside knn_rescore_kernel, at 16 warps per SM, they were latency-bound:
+// C5 k = 1024, 2.9 ms).
+template <int R>  // (R unused: one instantiation per compilation unit of this file)
+__global__ void __launch_bounds__(256, 3) knn_exact_kernel(const KnnRescoreArgs a) {
+    __shared__ double qd_all[8][KNN_MAX_D];
+    const uint32_t lane = lane_id();
+    const int w = threadIdx.x >> 5;
+    const int64_t q = (int64_t)blockIdx.x * 8 + w;
+    if (q >= a.Q) return;
+    const int c = a.ccount[q];
+    if (c <= 0) return;
+    double* qd = qd_all[w];
+    for (int t = (int)lane; t < a.D; t += 32) qd[t] = (double)a.query[q * a.D + t];
+    __syncwarp();
+    unsigned long long* cq = a.cand + q * (int64_t)kCandCap;
+    for (int e = (int)lane; e < c; e += 32) {
+        const uint32_t row = (uint32_t)cq[e];
+        cq[e] = ((unsigned long long)key_of(exact_dist(a.ref + (int64_t)row * a.D, qd, a.D)) << 32) | row;
+    }
+}
+
+// knn_finish_kernel: the exact top-k of each band (narrowing in global memory), sorted, emitted.
+template <int R>
+__global__ void __launch_bounds__(32 * rs_warps(R)) knn_finish_kernel(const KnnRescoreArgs a) {
+    constexpr int kRsWarps = rs_warps(R);
+    constexpr int kRsRegs = rs_regs(R);
+    __shared__ uint32_t hist_all[kRsWarps][256];
+    const uint32_t lane = lane_id();
+    const int64_t q = (int64_t)blockIdx.x * kRsWarps + (threadIdx.x >> 5);
+    if (q >= a.Q) return;
+    int c = a.ccount[q];
+    if (c < 0) return;
+    unsigned long long* cq = a.cand + q * (int64_t)kCandCap;
+    if (c > a.k) {
+        int nn;
+        narrow_any<kRsRegs, true>(cq, c, (uint32_t)a.k, &nn, hist_all[threadIdx.x >> 5]);
+        c = nn;
+        __syncwarp();
+    }
+    emit_sorted<R>(cq, c, a.k, a.idx_offset, a.out_val + q * a.k, a.out_idx + q * a.k, lane);
 }
 
 template <int R>
@@ -421,8 +487,13 @@ __global__ void __launch_bounds__(32 * kFbWarps) knn_fallback_kernel(const KnnRe
 
 template <int R>
 cudaError_t launch_knn_rescore_r(const KnnRescoreArgs& a, cudaStream_t stream) {
+    constexpr int kRsWarps = rs_warps(R);
     const int64_t grid = (a.Q + kRsWarps - 1) / kRsWarps;
     knn_rescore_kernel<R><<<(unsigned)grid, 32 * kRsWarps, 0, stream>>>(a);
+    note_launch();
+    knn_exact_kernel<R><<<(unsigned)((a.Q + 7) / 8), 256, 0, stream>>>(a);
+    note_launch();
+    knn_finish_kernel<R><<<(unsigned)grid, 32 * kRsWarps, 0, stream>>>(a);
     note_launch();
     return cudaGetLastError();
 }

@@ -421,7 +421,7 @@ __device__ __noinline__ unsigned long long pool_narrow64(unsigned long long* __r
 // before any use: the passes below are latency-bound otherwise, since the
 // compiler cannot hoist a global load above a shared-memory atomic of the
 // previous element); f(v) on every valid entry.
-template <typename F>
+template <bool GLOBAL = true, typename F>
 __device__ __forceinline__ void pool_scan64(const unsigned long long* __restrict__ pool, int n, uint32_t lane, F f) {
 #pragma unroll 1
     for (int base = 0; base < n; base += 256) {
@@ -429,7 +429,7 @@ __device__ __forceinline__ void pool_scan64(const unsigned long long* __restrict
 #pragma unroll
         for (int j = 0; j < 8; ++j) {
             const int e = base + j * 32 + (int)lane;
-            v[j] = (e < n) ? __ldcg(pool + e) : 0ull;
+            v[j] = (e < n) ? (GLOBAL ? __ldcg(pool + e) : pool[e]) : 0ull;
         }
 #pragma unroll
         for (int j = 0; j < 8; ++j)
@@ -444,14 +444,16 @@ __device__ __forceinline__ void pool_scan64(const unsigned long long* __restrict
 // transposed layout).  The pool is then compacted in place to the pairs <= it.
 // slack > 0: stop after the first key digit whose bucket, with everything below it,
 // holds at most want + slack pairs; the bound is then (bucket's last key, 0x7ffffffe).
-__device__ __noinline__ static unsigned long long pool_select64(unsigned long long* __restrict__ pool, int n,
+// (GLOBAL = false: a shared-memory pool -- generic loads instead of ld.global.cg)
+template <bool GLOBAL = true>
+__device__ __noinline__ unsigned long long pool_select64(unsigned long long* __restrict__ pool, int n,
                                                                uint32_t want, uint32_t* __restrict__ hist,
                                                                int* n_out, float band = -1.f, uint32_t slack = 0) {
     const uint32_t want0 = want;
     bool early = false;
     const uint32_t lane = lane_id();
     uint32_t kmin = 0xffffffffu, kmax = 0u;
-    pool_scan64(pool, n, lane, [&](unsigned long long v) {
+    pool_scan64<GLOBAL>(pool, n, lane, [&](unsigned long long v) {
         const uint32_t kk = (uint32_t)(v >> 32);
         kmin = min(kmin, kk);
         kmax = max(kmax, kk);
@@ -468,7 +470,7 @@ __device__ __noinline__ static unsigned long long pool_select64(unsigned long lo
 #pragma unroll
         for (int j = 0; j < 8; ++j) hist[j * 32 + lane] = 0u;
         __syncwarp();
-        pool_scan64(pool, n, lane, [&](unsigned long long v) {
+        pool_scan64<GLOBAL>(pool, n, lane, [&](unsigned long long v) {
             const uint32_t kk = (uint32_t)(v >> 32);
             const bool sel = (hi == 31) || ((kk ^ prefix) >> (hi + 1)) == 0u;
             if (sel) atomicAdd(&hist[hist_slot((kk >> lo) & dmask)], 1u);
@@ -490,7 +492,7 @@ __device__ __noinline__ static unsigned long long pool_select64(unsigned long lo
         vidx = 0x7ffffffeu;
     } else if (cnt == want) {
         uint32_t m = 0;
-        pool_scan64(pool, n, lane, [&](unsigned long long v) {
+        pool_scan64<GLOBAL>(pool, n, lane, [&](unsigned long long v) {
             if ((uint32_t)(v >> 32) == vkey) m = max(m, (uint32_t)v);
         });
         vidx = __reduce_max_sync(kFull, m);
@@ -502,7 +504,7 @@ __device__ __noinline__ static unsigned long long pool_select64(unsigned long lo
 #pragma unroll
             for (int j = 0; j < 8; ++j) hist[j * 32 + lane] = 0u;
             __syncwarp();
-            pool_scan64(pool, n, lane, [&](unsigned long long v) {
+            pool_scan64<GLOBAL>(pool, n, lane, [&](unsigned long long v) {
                 if ((uint32_t)(v >> 32) != vkey) return;
                 const uint32_t id = (uint32_t)v;
                 const bool sel = (pass == 0) || ((id ^ ip) >> (shift + 8)) == 0u;
@@ -527,7 +529,7 @@ __device__ __noinline__ static unsigned long long pool_select64(unsigned long lo
 #pragma unroll
         for (int j = 0; j < 8; ++j) {
             const int e = base + j * 32 + (int)lane;
-            v[j] = (e < n) ? __ldcg(pool + e) : ~0ull;
+            v[j] = (e < n) ? (GLOBAL ? __ldcg(pool + e) : pool[e]) : ~0ull;
         }
         __syncwarp();
 #pragma unroll
