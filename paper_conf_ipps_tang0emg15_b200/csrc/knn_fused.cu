@@ -1327,15 +1327,16 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
 // candidates (C4: ~6200 per query, 60x its k) and almost every 32 x 32 epilogue chunk
 // takes the rare path.  A pre-pass of the same kernel over a strided sample of m = ms x BN
 // references (S = 1, target j) yields T_spec = the j-th smallest sampled d~.  The count
-// of ALL references with d~ <= T_spec is ~ (N / m) Gamma(j); j = lambda + 6 sqrt(lambda) + 6
-// with lambda = k m / N (the count's expected k-th position in the sample) makes
-// P(count < k) < 1e-10 on i.i.d. rows.  The main pass admits against T_spec from its first
+// of ALL references with d~ <= T_spec is ~ (N / m) Gamma(j); the verification fails when
+// >= j of the k nearest fall in the sample: P = P(Poisson(lambda) >= j), lambda = k m / N.
+// j = lambda + 5 sqrt(lambda) + 5 keeps it below ~3e-9 per query at C4 (lambda = 1.64,
+// j = 14) and ~1e-6 at k = 1024 (lambda = 16.8, j = 43); 6 sigma was measured ~3 % slower.  The main pass admits against T_spec from its first
 // tile; knn_rescore_kernel verifies it (>= k pooled pairs <= T_spec, or a published
 // bound <= T_spec), else the query takes the exact fallback -- exact either way.
 static KnnGeom knn_spec_geometry(const KnnGeom& g, int ms) {
     KnnGeom p = g;
     const double lam = (double)g.k * (double)ms * g.BN / (double)g.N;
-    int j = (int)std::ceil(lam + 6.0 * std::sqrt(lam) + 6.0);
+    int j = (int)std::ceil(lam + 5.0 * std::sqrt(lam) + 5.0);
     p.k = std::min(j, KNN_BN);
     const int kk = p.k < 32 ? 32 : p.k;
     const int P = (kk <= 128) ? 1152 : kk + 8 * 256;
