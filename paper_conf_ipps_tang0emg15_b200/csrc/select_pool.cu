@@ -365,7 +365,35 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
             }
         }
         nreal = __reduce_add_sync(kFull, nreal);
-        if (nreal >= (uint32_t)k && k <= NB * CH / 2) {
+        // Whether the speculative bound below will be used (k > 128, sampled ranges that
+        // overlap): then the rigorous bisection is skipped -- a failed speculative share
+        // (~1e-10) restarts cold.
+        // (k' < 1024 only: the k' = 1024 kernel, which never has a rigorous bound here
+        // (k > NB * CH / 2), measured 3 % slower with this code shape -- it keeps the old one)
+        bool spec_ok = false;
+        uint32_t jj = 0;
+        if (R < 32 && !(order_mode & 64) && k > 128 && nreal >= 64u) {
+            uint32_t lo_max = 0u, hi_min = 0xffffffffu;
+#pragma unroll
+            for (int li = 0; li < NB; ++li) {
+                uint32_t lo = 0xffffffffu, hi = 0u;
+#pragma unroll
+                for (int j = 0; j < CH / 128 * 4; ++j) {
+                    const uint32_t kk2 = keys[li * (CH / 128) * 4 + j];
+                    if (kk2 != 0xffffffffu) { lo = min(lo, kk2); hi = max(hi, kk2); }
+                }
+                lo_max = max(lo_max, __reduce_min_sync(kFull, lo));
+                hi_min = min(hi_min, __reduce_max_sync(kFull, hi));
+            }
+            const uint64_t wlen = min((uint64_t)c_end * CH, (uint64_t)body_len) - (uint64_t)c_begin * CH;
+            const double lam = (double)k * (double)nreal / (double)wlen;
+            // (6 sigma as in the kNN filter: a failed share re-streams, and with ~2000 warps
+            // per launch the slowest one sets the time -- measured with 3 sigma, P(fail) ~1e-3
+            // per share: C2 U k = 256 0.103 -> 0.143 ms)
+            jj = (uint32_t)ceil(lam + 6.0 * sqrt(lam) + 6.0);
+            spec_ok = lo_max <= hi_min && jj < (uint32_t)k && jj < nreal;
+        }
+        if (!spec_ok && nreal >= (uint32_t)k && k <= NB * CH / 2) {
             // Bisection on the key bits below the common prefix of the smallest and
             // largest real key, stopped at bit kLow: the k-th key then lies in
             // [vkey, vkey + 2^kLow), so vkey | (2^kLow - 1) bounds it (>= k keys are
@@ -415,7 +443,7 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
         // data: not a random sample) get no speculation.
         // (k > 128 only: measured on C2, speculation gains 7-46 % at k = 256 / 1024 and
         // costs 0-7 % at k <= 32 -- a few narrowings at most to save there)
-        if (!(order_mode & 64) && k > 128 && nreal >= 64u) {
+        if (R == 32 && !(order_mode & 64) && k > 128 && nreal >= 64u) {
             uint32_t cmin[NB], cmax[NB];
 #pragma unroll
             for (int li = 0; li < NB; ++li) {
@@ -433,11 +461,11 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
             for (int li = 0; li < NB; ++li) { lo_max = max(lo_max, cmin[li]); hi_min = min(hi_min, cmax[li]); }
             const uint64_t wlen = min((uint64_t)c_end * CH, (uint64_t)body_len) - (uint64_t)c_begin * CH;
             const double lam = (double)k * (double)nreal / (double)wlen;
-            // (6 sigma as in the kNN filter: a failed share re-streams, and with ~2000 warps
-            // per launch the slowest one sets the time -- measured with 3 sigma, P(fail) ~1e-3
-            // per share: C2 U k = 256 0.103 -> 0.143 ms)
-            const uint32_t jj = (uint32_t)ceil(lam + 6.0 * sqrt(lam) + 6.0);
-            if (lo_max <= hi_min && jj < (uint32_t)k && jj < nreal) {
+            jj = (uint32_t)ceil(lam + 6.0 * sqrt(lam) + 6.0);
+            spec_ok = lo_max <= hi_min && jj < (uint32_t)k && jj < nreal;
+        }
+        {
+            if (spec_ok) {
                 uint32_t kmin2 = 0xffffffffu, kmax2 = 0u;
 #pragma unroll
                 for (int j = 0; j < NB * CH / 128 * 4; ++j) {
