@@ -365,14 +365,15 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
             }
         }
         nreal = __reduce_add_sync(kFull, nreal);
-        // Whether the speculative bound below will be used (k > 128, sampled ranges that
-        // overlap): then the rigorous bisection is skipped -- a failed speculative share
-        // (~1e-10) restarts cold.
+        // Whether the speculative bound below will be used (k > 64 -- k' = 1024: k > 128 --
+        // and sampled ranges that overlap): then the rigorous bisection is skipped (a failed
+        // speculative share, ~1e-10, restarts cold).  C2 A/B (profiles/r02_c2_spec_k128_ab.txt):
+        // k = 128 -2..-9 %, k = 64 mixed (+2 / -4 %), k = 32 +1..2 %: not below 65.
         // (k' < 1024 only: the k' = 1024 kernel, which never has a rigorous bound here
         // (k > NB * CH / 2), measured 3 % slower with this code shape -- it keeps the old one)
         bool spec_ok = false;
         uint32_t jj = 0;
-        if (R < 32 && !(order_mode & 64) && k > 128 && nreal >= 64u) {
+        if (R < 32 && !(order_mode & 64) && k > 64 && nreal >= 64u) {
             uint32_t lo_max = 0u, hi_min = 0xffffffffu;
 #pragma unroll
             for (int li = 0; li < NB; ++li) {
