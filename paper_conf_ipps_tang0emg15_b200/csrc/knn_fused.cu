@@ -589,6 +589,25 @@ __device__ __forceinline__ void tmem_wait32(uint32_t (&v)[32]) {
                  : "memory");
 }
 
+__device__ __forceinline__ uint32_t ld_vol_shared_u32(uint32_t a) {
+    uint32_t v;
+    asm volatile("ld.volatile.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+    return v;
+}
+__device__ __forceinline__ unsigned long long ld_vol_shared_u64(uint32_t a) {
+    unsigned long long v;
+    asm volatile("ld.volatile.shared.u64 %0, [%1];" : "=l"(v) : "r"(a) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_shared_u32(uint32_t a, uint32_t v) {
+    asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_shared_u64(uint32_t a, unsigned long long v) {
+    asm volatile("st.shared.u64 [%0], %1;" ::"r"(a), "l"(v) : "memory");
+}
+__device__ __forceinline__ void atom_min_shared_u64(uint32_t a, unsigned long long v) {
+    asm volatile("red.shared.min.u64 [%0], %1;" ::"r"(a), "l"(v) : "memory");
+}
 __device__ __forceinline__ uint32_t atom_add_shared(uint32_t saddr, uint32_t v) {
     uint32_t r;
     asm volatile("atom.shared.add.u32 %0, [%1], %2;" : "=r"(r) : "r"(saddr), "r"(v) : "memory");
@@ -827,9 +846,11 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)  // (EW = 16: 18 warps, 5 
         const int qgrp = hq * 4 + quad;
         const int qidx = hq * 128 + row;
         uint8_t* wscratch = reinterpret_cast<uint8_t*>(dstage_all) + qgrp * KnnSmem::kWarpScratch;
-        int* np = qs_n + qidx;
-        int* fp = qs_f + qidx;
-        unsigned long long* Tp = qs_T + qidx;
+        // the query group's shared state, by 32-bit shared-space address (explicit
+        // ld/st/atom.shared: no generic volatile accesses, fewer live registers)
+        const uint32_t np_s = smem_u32(qs_n + qidx);   // pool fill
+        const uint32_t fp_s = smem_u32(qs_f + qidx);   // failure flag
+        const uint32_t Tp_s = smem_u32(qs_T + qidx);   // shared bound pair
         auto pair_bar = [&]() {
             if constexpr (PAIR > 1) asm volatile("bar.sync %0, %1;" ::"r"(1 + qgrp), "r"(32 * PAIR) : "memory");
             else __syncwarp();
@@ -847,9 +868,9 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)  // (EW = 16: 18 warps, 5 
         bool failed = !(band < __int_as_float(0x7f800000));  // no finite band: exact fallback
         if (qvalid && !DUMP && !PIPE_ONLY && failed && half == 0 && !g.prepass) qfail[q] = 1;
         if (half == 0) {
-            *np = 0;
-            *fp = failed ? 1 : 0;
-            *Tp = kSentPair;
+            st_shared_u32(np_s, 0u);
+            st_shared_u32(fp_s, failed ? 1u : 0u);
+            st_shared_u64(Tp_s, kSentPair);
         }
         pair_bar();
 
@@ -862,7 +883,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)  // (EW = 16: 18 warps, 5 
         auto adopt = [&](unsigned long long t) {
             if (t < T) {
                 set_T(t);
-                if (PAIR > 1) atomicMin(Tp, t);
+                if (PAIR > 1) atom_min_shared_u64(Tp_s, t);
             }
         };
         // Speculative start (knn_run's sampled pre-pass): T_spec, the j-th smallest d~ of a
@@ -877,9 +898,9 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)  // (EW = 16: 18 warps, 5 
         // after a pair barrier: the pair's shared bound and failure flag
         auto refresh = [&]() {
             if constexpr (PAIR > 1) {
-                const unsigned long long t = *reinterpret_cast<volatile unsigned long long*>(Tp);
+                const unsigned long long t = ld_vol_shared_u64(Tp_s);
                 if (t < T) set_T(t);
-                failed = *reinterpret_cast<volatile int*>(fp) != 0;
+                failed = ld_vol_shared_u32(fp_s) != 0u;
             }
         };
         // warp-cooperative narrowing of every lane whose pool cannot take `room` more pairs:
@@ -889,7 +910,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)  // (EW = 16: 18 warps, 5 
         auto narrow_lanes = [&](int room, int target, int cap, bool final_pass) {
             pair_bar();
             refresh();
-            const int n = *reinterpret_cast<volatile int*>(np);
+            const int n = (int)ld_vol_shared_u32(np_s);
             // both warps of the pair have read the shared fills and bounds before either
             // narrows (and writes them): they derive the same `need` and split it consistently
             pair_bar();
@@ -913,14 +934,14 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)  // (EW = 16: 18 warps, 5 
                     : (EW <= 8 && jn <= 32 * kNarrowRegs) ? pool_narrow64<(EW <= 8 ? kNarrowRegs : 16)>(jp, jn, (uint32_t)target, &nn, jb, slk)
                                                : pool_select64(jp, jn, (uint32_t)target, hist, &nn, jb, slk);
                 if ((int)lane == j) {
-                    *np = nn;
+                    st_shared_u32(np_s, (uint32_t)nn);
                     adopt(t);
                     // publish: the k-th pair of this split's part bounds the whole row
                     if (target == g.k && (uint32_t)(t >> 32) != kSentKey) atomicMin(&qthr[q], t);
                     if (!final_pass && nn + room > cap) {  // the band alone fills the pool
                         failed = true;
-                        *np = 0;
-                        *fp = 1;
+                        st_shared_u32(np_s, 0u);
+                        st_shared_u32(fp_s, 1u);
                         if (!g.prepass) qfail[q] = 1;  // (pre-pass: just no speculation)
                     }
                 }
@@ -1067,7 +1088,6 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)  // (EW = 16: 18 warps, 5 
                 // values pass), NaN for a lane that takes nothing (every compare fails)
                 const float tvl = !live ? __int_as_float(0x7fc00000)
                                         : (fast ? __fmul_ru(tv, stl) : __int_as_float(0x7f800000));
-                const uint32_t np_s = smem_u32(np);
                 auto scan32 = [&](const uint32_t(&v)[32], int c0) {
                     float gmn[8];  // 3-input minima (FMNMX3): 20 instructions per 32 values
 #pragma unroll
@@ -1104,7 +1124,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)  // (EW = 16: 18 warps, 5 
                                 const float dc = (xu < 0.f) ? 0.f : xu;  // clamp
                                 int slot;
                                 if constexpr (PAIR > 1) slot = (int)atom_add_shared(np_s, 1u);
-                                else slot = (*np)++;
+                                else { slot = (int)ld_vol_shared_u32(np_s); st_shared_u32(np_s, (uint32_t)slot + 1u); }
                                 pool[slot] = ((unsigned long long)key_of(dc) << 32) | (colt + (uint32_t)(cu + i));
                                 if (PROF) prof_app++;
                             }
@@ -1142,7 +1162,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)  // (EW = 16: 18 warps, 5 
                 uint32_t v[KNN_CW];
                 tmem_ld64(taddr + (uint32_t)(c * KNN_CW), v);
                 if (PIPE_ONLY) {
-                    if (v[0] == 0x7fc00001u && v[KNN_CW - 1] == 0x7fc00001u) (*np)++;  // keep the load alive
+                    if (v[0] == 0x7fc00001u && v[KNN_CW - 1] == 0x7fc00001u) st_shared_u32(np_s, 1u);  // keep the load alive
                     continue;
                 }
                 const int64_t col0 = (int64_t)t * BN + c * KNN_CW;
@@ -1167,7 +1187,7 @@ __global__ void __launch_bounds__(knn_threads(EW), 1)  // (EW = 16: 18 warps, 5 
             // the pool's k smallest); launch_merge_pools gathers the pools' pairs <= the
             // final published bound and selects the exact top-k of the row.
             narrow_lanes(g.P - g.k, g.k, g.P, true);  // n > k  <=>  n + (P - k) > P
-            if (qvalid && half == 0) cnt_out[list * g.Q + q] = failed ? 0 : *np;
+            if (qvalid && half == 0) cnt_out[list * g.Q + q] = failed ? 0 : (int)ld_vol_shared_u32(np_s);
         }
         if (PROF) {
             __syncwarp();
