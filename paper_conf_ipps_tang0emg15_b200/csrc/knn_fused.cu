@@ -219,7 +219,10 @@ __global__ void __launch_bounds__(256)
                      const double* __restrict__ csum, float4* __restrict__ qstat, float2* __restrict__ tscale,
                      KnnStats* __restrict__ st, uint4* __restrict__ ref_img, uint4* __restrict__ q_img,
                      int* __restrict__ fixlist, int* __restrict__ fixcnt) {
-    __shared__ float tile[KNN_BN][KNN_KS + 1];
+    // (the shared transpose tile only on the scalar path: dynamic, 0 bytes when every row is
+    // 16-byte aligned -- more blocks per SM for the direct 16-byte loads)
+    extern __shared__ float prep_tile_raw[];
+    auto tile = reinterpret_cast<float(*)[KNN_KS + 1]>(prep_tile_raw);
     __shared__ float cs[KNN_MAX_D];
     __shared__ uint32_t srange, smax;
     __shared__ int sover, sbad;
@@ -245,36 +248,46 @@ __global__ void __launch_bounds__(256)
     const float sig = ldexpf(1.f, e);
     const float mul = is_q ? -2.f * sig : sig;  // exact
     // (D % 4 == 0 and a 16-byte aligned base: every row is 16-byte aligned)
-    const bool vec4 = (g.D & 3) == 0 && (reinterpret_cast<uintptr_t>(x) & 15u) == 0;
+    const bool vec4 = (g.D & 3) == 0 && (reinterpret_cast<uintptr_t>(ref) & 15u) == 0 &&
+                      (reinterpret_cast<uintptr_t>(qry) & 15u) == 0;  // (= the host's choice of smem)
     double s = 0.0;
     bool over = false, bad = false;
     for (int ks = 0; ks < g.KS; ++ks) {
-        __syncthreads();
+        float vv[KNN_KS];  // this thread's row, dims ks * 32 .. + 31, centred
         if (vec4) {
-            // 16-byte loads: lane l reads dims 4 (l % 8) .. + 3 of row r + l / 8 (512 B per
-            // warp instruction, 8 loads in flight per lane)
-            const int dq = ks * KNN_KS + 4 * (lane & 7);
-#pragma unroll 8
-            for (int r = warp * 4 + (lane >> 3); r < rows; r += 32) {
-                const int64_t gr = t * rows + r;
-                float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
-                if (gr < n && dq < g.D) v = __ldcs(reinterpret_cast<const float4*>(x + gr * (int64_t)g.D + dq));
-                const bool ok = gr < n && dq < g.D;
-                float* tr = &tile[r][4 * (lane & 7)];
-                tr[0] = ok ? v.x - cs[dq] : 0.f;
-                tr[1] = ok ? v.y - cs[dq + 1] : 0.f;
-                tr[2] = ok ? v.z - cs[dq + 2] : 0.f;
-                tr[3] = ok ? v.w - cs[dq + 3] : 0.f;
+            // (thread = row: its own 8 x 16-byte loads, L1-cached so that the other half of
+            // each 32-byte sector serves the next load; no shared-memory transpose, no barriers)
+            if (tid < rows) {
+                const bool okr = row < n;
+                const float4* xr = reinterpret_cast<const float4*>(x + (okr ? row : 0) * (int64_t)g.D + ks * KNN_KS);
+                float4 v4[KNN_KS / 4];
+#pragma unroll
+                for (int u = 0; u < KNN_KS / 4; ++u)
+                    v4[u] = (okr && ks * KNN_KS + 4 * u < g.D) ? __ldg(xr + u) : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+                for (int u = 0; u < KNN_KS / 4; ++u) {
+                    const int d = ks * KNN_KS + 4 * u;
+                    const bool ok = okr && d < g.D;
+                    vv[4 * u + 0] = ok ? v4[u].x - cs[d] : 0.f;
+                    vv[4 * u + 1] = ok ? v4[u].y - cs[d + 1] : 0.f;
+                    vv[4 * u + 2] = ok ? v4[u].z - cs[d + 2] : 0.f;
+                    vv[4 * u + 3] = ok ? v4[u].w - cs[d + 3] : 0.f;
+                }
             }
         } else {
+            __syncthreads();
             const int d = ks * KNN_KS + lane;
 #pragma unroll 8
             for (int r = warp; r < rows; r += 8) {
                 const int64_t gr = t * rows + r;
                 tile[r][lane] = (gr < n && d < g.D) ? __ldcs(x + gr * (int64_t)g.D + d) - cs[d] : 0.f;
             }
+            __syncthreads();
+            if (tid < rows) {
+#pragma unroll
+                for (int j = 0; j < KNN_KS; ++j) vv[j] = tile[tid][j];
+            }
         }
-        __syncthreads();
         if (tid < rows) {
             uint4* dst;
             int cstride;
@@ -290,7 +303,7 @@ __global__ void __launch_bounds__(256)
                 uint32_t h[4];
 #pragma unroll
                 for (int p = 0; p < 4; ++p) {
-                    const float v0 = tile[tid][kc * 8 + 2 * p], v1 = tile[tid][kc * 8 + 2 * p + 1];
+                    const float v0 = vv[kc * 8 + 2 * p], v1 = vv[kc * 8 + 2 * p + 1];
                     s += (double)v0 * (double)v0;
                     s += (double)v1 * (double)v1;
                     const float a0 = fabsf(v0), a1 = fabsf(v1);
@@ -1459,7 +1472,10 @@ static cudaError_t knn_run(const float* ref, const float* query, int64_t N, int6
         if (e != cudaSuccess) return e;
         // one read of the points at the call's common scale; then the (rare) tiles whose
         // values exceed it rebuilt from their own max (grid-stride over the list: usually empty)
-        knn_prep1_kernel<<<(unsigned)(nt + g.QT), 256, 0, stream>>>(ref, query + q0 * (int64_t)D, g, nt, csum, qstat,
+        const bool vec4 = (D & 3) == 0 && (reinterpret_cast<uintptr_t>(ref) & 15u) == 0 &&
+                          (reinterpret_cast<uintptr_t>(query + q0 * (int64_t)D) & 15u) == 0;
+        const size_t prep_smem = vec4 ? 0 : sizeof(float) * KNN_BN * (KNN_KS + 1);
+        knn_prep1_kernel<<<(unsigned)(nt + g.QT), 256, prep_smem, stream>>>(ref, query + q0 * (int64_t)D, g, nt, csum, qstat,
                                                                     tscale, stats, ref_img, q_img, fixlist, fixcnt);
         note_launch();
         knn_stats_kernel<<<(unsigned)sms, KNN_PREP_THREADS, 0, stream>>>(
