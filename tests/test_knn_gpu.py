@@ -375,3 +375,16 @@ def test_knn_speculative_bound_fails_verification(K, oracle_mod):
         ref[r0:r0 + 2] = qry[0] + 1e-3 * (ref[r0:r0 + 2] - 0.5)
     gv, gi = K.knn_search(ref.cuda(), qry.cuda(), k)
     check_knn(oracle_mod, ref, qry, k, gv, gi)
+
+
+def test_knn_nonfinite_reference_rows(K, oracle_mod):
+    """A NaN and an Inf reference row make max |r'|^2 infinite, so no query has a finite filter
+    bound: every query takes the exact fallback (reading R21).  Their distances are NaN / Inf and
+    sort last (R4); the k nearest are the oracle's."""
+    N, Q, D, k = 3000, 40, 16, 10
+    ref = synth.knn_points("knn-U", 61, 0, N, D).clone()
+    qry = synth.knn_points("knn-U", 62, 0, Q, D).clone()
+    ref[17, 3] = float("nan")
+    ref[2500, 0] = float("inf")
+    gv, gi = K.knn_search(ref.cuda(), qry.cuda(), k)
+    check_knn(oracle_mod, ref, qry, k, gv, gi)
