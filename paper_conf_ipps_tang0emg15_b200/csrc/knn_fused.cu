@@ -1234,10 +1234,13 @@ struct KnnWork {
 // points would otherwise need tens of GB of workspace).
 constexpr size_t kPoolBudget = 2ull << 30;
 
+// sampled tiles: up to 64 (KSEL_KNN_SPEC, 0: off), at most 1/16 of the references, at
+// least 8 (N >= 32768; smaller sets start cold)
 static int knn_spec_tiles(const KnnGeom& g) {
-    static const int env = env_int("KSEL_KNN_SPEC", 64);  // sampled tiles (0: off)
-    if (env <= 0 || g.NT < 16 * env || g.tstride != 1) return 0;
-    return env;
+    static const int env = env_int("KSEL_KNN_SPEC", 64);
+    if (env <= 0 || g.tstride != 1) return 0;
+    const int ms = std::min(env, g.NT / 16);
+    return ms >= 8 ? ms : 0;
 }
 
 // max_lists > 0: cap the split count so that S * halves * Q <= max_lists (a later query
