@@ -205,6 +205,10 @@ __global__ void __launch_bounds__(32 * rs_warps(R), 4) knn_rescore_kernel(const 
     // the k-th d~ over ALL of the query's pools (at least k references have a d~ <= it):
     // only the band above it can hold the exact top-k
     unsigned long long T0 = a.thr[q];
+    // (with a speculative start: gather against min(T_spec, thr) + band in ONE pass, count the
+    // verification inline, and let the buffer's narrowing find the k-th -- no union scans)
+    const unsigned long long ts = a.spec ? a.spec[q] : ~0ull;
+    const bool spec = (uint32_t)(ts >> 32) != kSentKey;
     {
         int tot = 0;
         for (int s = (int)lane; s < a.S; s += 32) tot += a.cnt[(int64_t)s * a.Q + q];
@@ -213,24 +217,15 @@ __global__ void __launch_bounds__(32 * rs_warps(R), 4) knn_rescore_kernel(const 
         // against min(T_spec, its verified bounds).  The pools then hold every reference with
         // d~ <= min(T_spec, thr) + band, so the band may start from T_spec only once T_spec is
         // VERIFIED -- at least k pooled pairs <= T_spec -- or from thr if thr <= T_spec.
-        // Otherwise the pools may miss part of the top-k: exact fallback.  (The count rides in
-        // the union scan that also bounds the k-th d~ when the union exceeds the buffer.)
-        const unsigned long long ts = a.spec ? a.spec[q] : ~0ull;
-        const bool spec = (uint32_t)(ts >> 32) != kSentKey;
-        const bool big = tot > kRsCap && tot >= a.k;  // (a union that fits the buffer is band-narrowed there)
-        if (spec || big) {
+        // Otherwise the pools may miss part of the top-k: exact fallback.  (The count is taken
+        // during the gather below; without a speculative bound a union larger than the buffer
+        // is first bounded by a radix scan.)
+        if (spec) {
+            T0 = ts < T0 ? ts : T0;  // (provisional: verified after the gather)
+        } else if (tot > kRsCap && tot >= a.k) {
             int le = 0;
-            const uint32_t kk = lists_kth_key(a.pools, a.cnt, a.S, a.Q, q, a.P, big ? (uint32_t)a.k : 0u, hist_all[w], ts,
-                                              &le);
-            if (spec) {
-                if (le >= a.k) {
-                    T0 = ts < T0 ? ts : T0;
-                } else if (!(T0 <= ts)) {
-                    if (lane == 0) { a.qfail[q] = 1; a.ccount[q] = -1; }
-                    return;
-                }
-            }
-            if (big) {
+            const uint32_t kk = lists_kth_key(a.pools, a.cnt, a.S, a.Q, q, a.P, (uint32_t)a.k, hist_all[w], ts, &le);
+            {
                 const unsigned long long t = ((unsigned long long)kk << 32) | 0xffffffffull;
                 T0 = t < T0 ? t : T0;
             }
@@ -254,6 +249,7 @@ __global__ void __launch_bounds__(32 * rs_warps(R), 4) knn_rescore_kernel(const 
         }
         __syncwarp();
     };
+    int le_spec = 0;  // pooled pairs <= T_spec (the speculative bound's verification)
     // one pair of the gather (phase A / B); x: its slot, ns: the list's length
     auto gather_one = [&](unsigned long long v, int x, int ns) {
             if (!exact_mode) {
@@ -314,12 +310,21 @@ __global__ void __launch_bounds__(32 * rs_warps(R), 4) knn_rescore_kernel(const 
             for (int j = 0; j < 4; ++j) {
                 const int x = base + j * 32 + (int)lane;
                 v[j] = (x < ns) ? __ldcg(pr + x) : ~0ull;
+                le_spec += (x < ns && v[j] <= ts) ? 1 : 0;
             }
 #pragma unroll 1
             for (int j = 0; j < 4 && base + j * 32 < ns; ++j) {
                 const unsigned long long vj = j == 0 ? v[0] : j == 1 ? v[1] : j == 2 ? v[2] : v[3];  // (no local array)
                 gather_one(vj, base + j * 32 + (int)lane, ns);
             }
+        }
+    }
+    if (spec) {
+        le_spec = __reduce_add_sync(kFull, le_spec);
+        const unsigned long long thr = a.thr[q];
+        if (le_spec < a.k && !(thr <= ts)) {  // T_spec not verified and no published bound below it
+            if (lane == 0) { a.qfail[q] = 1; a.ccount[q] = -1; }
+            return;
         }
     }
     if (!exact_mode) {  // phase A ended: the band set, rescored exactly by knn_exact_kernel
