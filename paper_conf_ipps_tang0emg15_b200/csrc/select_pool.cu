@@ -547,13 +547,12 @@ __global__ void __launch_bounds__(PoolCfg<R, WPR, RPC, SD>::kThreads, (R < 16 &&
                 // value cannot precede the bound pair, so the test is strict: rows with heavy
                 // ties then skip the sub-steps that only hold copies of the bound value.
                 // (a tree, not a 15-deep chain: the sub-step is latency-bound when few warps run)
+                // (3-input minima, FMNMX3 on sm_100: 10 instructions per 16 values instead of 15)
+                static_assert(G == 4, "min tree shape");
                 float gm[G];
 #pragma unroll
-                for (int u = 0; u < G; ++u)
-                    gm[u] = fminf(fminf(x[4 * u], x[4 * u + 1]), fminf(x[4 * u + 2], x[4 * u + 3]));
-                float mn = gm[0];
-#pragma unroll
-                for (int u = 1; u < G; ++u) mn = fminf(mn, gm[u]);
+                for (int u = 0; u < G; ++u) gm[u] = fminf(fmin3f(x[4 * u], x[4 * u + 1], x[4 * u + 2]), x[4 * u + 3]);
+                const float mn = fminf(fmin3f(gm[0], gm[1], gm[2]), gm[3]);
                 go = __any_sync(kFull, col0 >= Ti ? mn < tv : mn <= tv);
             }
             // The stage is refilled as soon as nothing reads it any more: right after the
