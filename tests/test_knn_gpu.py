@@ -216,6 +216,26 @@ def test_knn_search_ignores_experiment_knobs(oracle_mod, tmp_path, kind, k):
     check_knn(oracle_mod, ref, qry[sample], k, gv[sample], gi[sample])
 
 
+@pytest.mark.parametrize("knobs", [{"KSEL_KNN_SPEC": "0"}, {"KSEL_KNN_SPEC": "8", "KSEL_KNN_NSTRIDE": "4"},
+                                   {"KSEL_KNN_EW": "8"}, {"KSEL_KNN_SPEC": "2000"}])
+def test_knn_search_result_preserving_knobs(oracle_mod, tmp_path, knobs):
+    """The late-r2 launch knobs of the product library -- speculative pre-pass off / its sample
+    size, bound-refresh stride, epilogue warps -- change only the time, never the result."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    N, Q, k = 70000, 600, 50
+    env = dict(os.environ, **knobs)
+    subprocess.run([sys.executable, "-c", _KNOB_SCRIPT, root, str(tmp_path), "knn-U", str(N), str(Q), str(k)],
+                   check=True, env=env, timeout=300)
+    gv, gi = np.load(tmp_path / "v.npy"), np.load(tmp_path / "i.npy")
+    ref = synth.knn_points("knn-U", 61, 0, N, 128)
+    qry = synth.knn_points("knn-U", 62, 0, Q, 128)
+    sample = list(range(16)) + list(range(40, Q, 37))
+    check_knn(oracle_mod, ref, qry[sample], k, gv[sample], gi[sample])
+
+
 @pytest.mark.parametrize("kind,N,D,k", [("knn-S", 700, 128, 16), ("knn-U", 900, 64, 10), ("knn-U", 2, 5, 1),
                                         ("knn-U", 333, 3, 332), ("knn-S", 1500, 96, 100)])
 def test_knn_graph_vs_oracle(K, oracle_mod, kind, N, D, k):

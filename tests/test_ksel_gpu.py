@@ -451,16 +451,19 @@ np.savez(sys.argv[2], **out)
 """
 
 
-@pytest.mark.parametrize("order", ["0", "1", "2", "3"])
+@pytest.mark.parametrize("order", ["0", "1", "2", "3", "3-nospec"])
 def test_chunk_visit_orders_bit_exact(oracle_mod, order, tmp_path):
-    # the chunk visit order (KSEL_ORDER, read once per process; default 3) changes only
-    # which candidates are admitted when, never the result
+    # the chunk visit order (KSEL_ORDER, read once per process; default 3) and the speculative
+    # starting bound (KSEL_SPEC=0: off) change only which candidates are admitted when, never
+    # the result
     import os
     import subprocess
     import sys
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     f = str(tmp_path / "res.npz")
-    env = dict(os.environ, KSEL_ORDER=order)
+    env = dict(os.environ, KSEL_ORDER=order[0])
+    if order.endswith("nospec"):
+        env["KSEL_SPEC"] = "0"
     subprocess.run([sys.executable, "-c", _ORDER_CHILD, root, f], env=env, check=True, timeout=600)
     res = np.load(f)
     for dist in ("U", "T", "SA", "SD", "X"):
