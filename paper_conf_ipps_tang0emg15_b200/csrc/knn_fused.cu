@@ -1234,10 +1234,11 @@ struct KnnWork {
 // points would otherwise need tens of GB of workspace).
 constexpr size_t kPoolBudget = 2ull << 30;
 
-// sampled tiles: up to 64 (KSEL_KNN_SPEC, 0: off), at most 1/16 of the references, at
-// least 8 (N >= 32768; smaller sets start cold)
+// sampled tiles: up to 128 (KSEL_KNN_SPEC, 0: off), at most 1/16 of the references, at
+// least 8 (N >= 32768; smaller sets start cold).  C4 A/B (profiles/r02_knn_spec_size_ab.txt):
+// 32 / 64 / 96 / 128 tiles -> filter 3.64 / 3.59 / 3.40 / 3.31 ms, call 4.55 / 4.59 / 4.47 / 4.48 ms
 static int knn_spec_tiles(const KnnGeom& g) {
-    static const int env = env_int("KSEL_KNN_SPEC", 64);
+    static const int env = env_int("KSEL_KNN_SPEC", 128);
     if (env <= 0 || g.tstride != 1) return 0;
     const int ms = std::min(env, g.NT / 16);
     return ms >= 8 ? ms : 0;
@@ -1366,8 +1367,8 @@ static KnnGeom knn_geometry(int64_t N, int64_t Q, int D, int k, int num_sms, int
 // references (S = 1, target j) yields T_spec = the j-th smallest sampled d~.  The count
 // of ALL references with d~ <= T_spec is ~ (N / m) Gamma(j); the verification fails when
 // >= j of the k nearest fall in the sample: P = P(Poisson(lambda) >= j), lambda = k m / N.
-// j = lambda + 5 sqrt(lambda) + 5 keeps it below ~3e-9 per query at C4 (lambda = 1.64,
-// j = 14) and ~1e-6 at k = 1024 (lambda = 16.8, j = 43); 6 sigma was measured ~3 % slower.  The main pass admits against T_spec from its first
+// j = lambda + 5 sqrt(lambda) + 5 keeps it below ~1e-8 per query at C4 (128 sampled tiles:
+// lambda = 3.3, j = 18); 6 sigma was measured ~1-2 % slower.  The main pass admits against T_spec from its first
 // tile; knn_rescore_kernel verifies it (>= k pooled pairs <= T_spec, or a published
 // bound <= T_spec), else the query takes the exact fallback -- exact either way.
 static KnnGeom knn_spec_geometry(const KnnGeom& g, int ms) {

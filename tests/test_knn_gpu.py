@@ -380,8 +380,8 @@ def test_knn_outlier_tiles_rebuilt(K, oracle_mod, k):
 
 def test_knn_speculative_bound_fails_verification(K, oracle_mod):
     """knn_search's speculative start (reading R23): T_spec is the j-th smallest filter
-    distance of a strided sample of 64 reference tiles.  Here every sampled tile holds two
-    near copies of query 0 (128 near references in all, k = 200 > 128), so query 0's T_spec
+    distance of a strided sample of reference tiles.  Here every sampled tile holds two near
+    copies of query 0 (2 x 73 near references in all, k = 200), so query 0's T_spec
     is one of them and fewer than k references lie below it: the rescore's verification
     fails and the query takes the exact fallback; every other query is verified normally.
     All results must be the oracle's."""
@@ -389,8 +389,10 @@ def test_knn_speculative_bound_fails_verification(K, oracle_mod):
     ref = synth.knn_points("knn-U", 51, 0, N, D).clone()
     qry = synth.knn_points("knn-U", 52, 0, Q, D).clone()
     NT = (N + 255) // 256
-    ts = NT // 64                      # knn_spec_geometry: tiles 0, ts, 2 ts, ... are sampled
-    for i in range(64):
+    ms = min(128, NT // 16)            # knn_spec_tiles: sampled tiles
+    ts = NT // ms                      # knn_spec_geometry: tiles 0, ts, 2 ts, ... are sampled
+    assert 2 * ms < k
+    for i in range(ms):
         r0 = i * ts * 256
         ref[r0:r0 + 2] = qry[0] + 1e-3 * (ref[r0:r0 + 2] - 0.5)
     gv, gi = K.knn_search(ref.cuda(), qry.cuda(), k)
