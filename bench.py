@@ -635,7 +635,7 @@ def bench_knn(args, rank, world, local_rank, dev, K, tdist):
                          "frac": achieved / peaks_bf16, "traffic": load_traffic(workload), "peak_source": src,
                          "kernel": "knn_fused_kernel", "kernel_ms": kern_ms,
                          "flops_per_launch": flops, "flops_formula": "2*Q*N_rank*D (algorithmic, 1 pass; "
-                                                                     "executed: 1 fp16 pass + a bf16 norm block; the speculative pre-pass launch over 64 sampled tiles is counted in the call, not in this kernel)",
+                                                                     "executed: 1 fp16 pass + a bf16 norm block; the speculative pre-pass launch over up to 128 sampled tiles is counted in the call, not in this kernel)",
                          "note": "kernel = the fused filter; the call adds the prologue and the exact "
                                  "rescoring (bit-identical to the oracle)"},
             "gpu_launches": launches,

@@ -8,16 +8,16 @@
 // exists.  d~(q, r) = |q|^2 + |r|^2 - 2 q.r (reading R9: squared L2), with the dot
 // products on the 5th-gen tensor cores:
 //
-//   * operands split once into bf16 hi/lo pairs (x ~ hi + lo, hi = bf16(x),
-//     lo = bf16(x - hi)); q.r ~ qh.rh + qh.rl + ql.rh -- three kind::f16 MMAs
-//     into one fp32 TMEM accumulator (the dropped ql.rl term is ~2^-16 relative).
-//   * the norms ride in the same accumulation: A holds -2q and one extra
-//     16-wide K block [n1, n2, n3, 1, 1, 1, 0...] with |q|^2 = n1+n2+n3 split
-//     three ways in bf16 (24 significant bits), B holds [1, 1, 1, m1, m2, m3, 0...]
-//     for |r|^2 -- so the accumulator IS d~(q, r) and the epilogue touches each
-//     distance once (no per-element norm adds).
+//   * points are centred (x' = x - c, c a rounded sample mean) and each tile scaled by a
+//     power of two, then rounded to fp16 once: ONE kind::f16 MMA pass (fp16 x fp16 ->
+//     fp32 TMEM accumulator); the error of that rounding is in the bound eps_q below.
+//   * the norms ride in the same accumulation: A holds -2 s_q q' and one extra
+//     16-wide bf16 K block [s n1, s n2, s n3, s, s, s, 0...] with |q'|^2 = n1+n2+n3 split
+//     three ways (24 significant bits), B holds [s, s, s, s m1, s m2, s m3, 0...] for
+//     |r'|^2 -- so the accumulator IS s_q s_t d~(q, r) and the epilogue touches each
+//     distance once (it compares against the bound scaled the same way).
 //   * d~ only FILTERS: |d~ - d| <= eps_q (a rigorous bound, knn_common.cuh knn_eps,
-//     DESIGN.md reading R21, ~1e-3 of the distance on the paper's workload), so a
+//     DESIGN.md reading R21, ~0.4 % of the k-th distance on the paper's workload), so a
 //     reference can be in the exact top-k only if d~ <= T + 2 eps_q for any k-th
 //     value T of d~ over k references; the epilogue admits exactly those, pools keep
 //     that band above their k-th d~, and knn_rescore.cu recomputes every survivor in
@@ -28,8 +28,10 @@
 //     memory) x a contiguous range of 256-reference tiles (TMEM columns, B
 //     operand streamed by 1-D TMA bulk copies from a pre-tiled image);
 //     warp 0 = producer, warp 1 = TMEM allocator + single-thread MMA issuer,
-//     warps 2-5 = epilogue (one thread per query: the paper's thread-per-query
-//     layout, L243), double-buffered 2 x 256-column accumulators.
+//     warps 2-17 = epilogue (four per TMEM lane quadrant; one thread per query: the
+//     paper's thread-per-query layout, L243), double-buffered 2 x 256-column accumulators.
+//   * a speculative pre-pass of the same kernel over a strided sample of reference tiles
+//     gives each query a starting bound T_spec (verified later in knn_rescore.cu).
 //   * epilogue: tcgen05.ld 32 columns at a time, an fp32 min/vote pre-filter against
 //     the running bound plus the band, a rare path that appends packed
 //     (key(d~) << 32 | index) pairs to a per-query pool in global memory,
@@ -530,7 +532,7 @@ __device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint
            ((uint64_t)((sbo >> 4) & 0x3FFFu) << 32) | (1ull << 46);
 }
 
-// kind::f16 instruction descriptor: bf16 x bf16 -> fp32, K-major A and B, M x N
+// kind::f16 instruction descriptor: bf16 x bf16 -> fp32, K-major A and B, M x N (the norm block)
 __host__ __device__ constexpr uint32_t umma_idesc_bf16(int M, int N) {
     return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
 }
@@ -540,6 +542,7 @@ __host__ __device__ constexpr uint32_t umma_idesc_f16(int M, int N) {
     return (1u << 4) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
 }
 
+// one tcgen05.mma kind::f16 (fp16 or bf16 operands, per the instruction descriptor)
 __device__ __forceinline__ void umma_bf16(uint32_t d_tmem, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
     asm volatile(
         "{\n\t.reg .pred p;\n\t"
